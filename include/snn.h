@@ -1,0 +1,162 @@
+/*
+ * snn.h -- C ABI of the B200 (sm_100a) simulate-and-learn path of
+ *   She, Long & Mukhopadhyay, "Fast and Low-Precision Learning in GPU-Accelerated Spiking
+ *   Neural Network", DATE 2019.  Paper text: /root/reference/PAPER.md, cited as P:<line>.
+ *
+ * One call of snn_present* runs, for every image and every timestep t, the four steps of the
+ * paper's per-timestep loop (Fig. 2 flowchart, §III-A) entirely in CUDA kernels:
+ *   (a1) Poisson rate encoding of the 8-bit image        P:88 §III-B
+ *   (a2) synaptic integration I_a = sum_n g_{n,a} v_pre  P:83 eq.(3)
+ *   (a3) LIF update dv/dt = a + b v + c I, reset          P:83 eqs.(1)(2), P:90 constants
+ *   (a4) winner-take-all lateral inhibition for t_inh     P:88 §III-B
+ *   (a5) stochastic STDP, eqs.(6)(7), dG = 1 LSB          P:85 §II-C, §III-C
+ *   (a6) deterministic STDP arm, eqs.(4)(5) + rounding     P:84 §II-B, eq.(8)
+ * The exact semantics (every reading of a silent or garbled passage, the Philox counter
+ * layout, the fixed-point recipe) are DESIGN.md §2-§3.
+ *
+ * Conventions
+ *  - Every function returns SNN_OK (0) or a negative SNN_E* code; snn_last_error() returns a
+ *    thread-local message for the last failure on the calling thread.
+ *  - The caller owns every buffer it passes; the library never retains a caller pointer past
+ *    the call (asynchronous calls: past the completion of the work they enqueue, see SNN_ASYNC).
+ *  - "host or device" pointers are classified with cudaPointerGetAttributes; host memory may be
+ *    pageable or pinned.
+ *  - A handle owns all of its device memory and is bound to the device current at snn_create.
+ *    Handles are not thread-safe; distinct handles may be used from distinct threads.
+ *  - Weights persist across presentations (online learning).  v, refractory counters and
+ *    spike timers are reset at the start of each presentation unless SNN_KEEP_STATE (R5).
+ */
+#ifndef SNN_H
+#define SNN_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SNN_OK       0
+#define SNN_EINVAL  (-1)   /* invalid argument or parameter                       */
+#define SNN_ENOMEM  (-2)   /* host or device allocation failed                    */
+#define SNN_ECUDA   (-3)   /* CUDA runtime error (message in snn_last_error)      */
+#define SNN_ENCCL   (-4)   /* NCCL error (sharded handles)                        */
+#define SNN_ESIZE   (-5)   /* caller buffer too small, or network exceeds the on-chip capacity */
+#define SNN_ECOOP   (-6)   /* cluster / co-residency launch not possible          */
+
+/* wta_mode */
+#define SNN_WTA_HARD   0   /* at most one spike per step: the largest v - v_th wins, ties -> lowest j (R7) */
+#define SNN_WTA_LAYER  1   /* every crossing neuron spikes (one-to-one inhibitory layer, R7)              */
+/* inh_mode */
+#define SNN_INH_RESET  0   /* inhibited neurons are reset to v_reset and held for t_inh steps */
+#define SNN_INH_HOLD   1   /* inhibited neurons keep v and are held for t_inh steps           */
+/* stdp_mode */
+#define SNN_STDP_STOCH 0   /* eqs.(6)(7) gate a one-LSB step ("dG is set to 1/2^n")     */
+#define SNN_STDP_DET   1   /* eqs.(4)(5) at each post spike, rounded to the grid (R16)        */
+/* rounding (deterministic arm, "three available rounding options") */
+#define SNN_ROUND_TRUNC   0
+#define SNN_ROUND_NEAREST 1
+#define SNN_ROUND_STOCH   2   /* eq.(8) */
+/* membrane_mode */
+#define SNN_MEM_FP32   0   /* explicit fmaf recipe */
+#define SNN_MEM_FIXED  1   /* Q15.16 integer recipe */
+
+/* Parameter block.  Field order and types are part of the ABI. */
+typedef struct snn_params {
+  /* LIF, §III-D: a=-6.77, b=-0.0989, c=0.314, V_th=-60.2, V_reset=-74.7, v_init=-70.0 */
+  double a, b, c, v_th, v_reset, v_init;
+  double dt_ms;          /* Euler step, ms (R1: 1.0)                                   */
+  double v_spike;        /* pre-synaptic "voltage spike" v_pre of eq.(3) (R3: 2.0)      */
+  double i_ext;          /* constant external current, test hook (0)                   */
+  int32_t t_ref_steps;   /* refractory steps after a spike (R6: 5)                     */
+  int32_t t_inh_steps;   /* lateral-inhibition steps, "t_inh" (R7: 10)            */
+  int32_t wta_mode, inh_mode;
+  double f_min_hz, f_max_hz;   /* encoder range, P:88 / Table I                         */
+  int32_t stdp_mode, rounding;
+  int32_t t_ltp_steps;   /* deterministic arm LTP window (R16: 20)                     */
+  int32_t membrane_mode;
+  double gamma_pot, tau_pot, gamma_dep, tau_dep;        /* eqs.(6)(7), Table I (ms)      */
+  double alpha_p, beta_p, alpha_d, beta_d, g_min, g_max; /* eqs.(4)(5), Table I "16 bit" */
+  int32_t frac_bits;     /* 0 = bits (LSB = 2^-bits); Q1.7-style grids: 7       */
+  int32_t init_mode;     /* 0: uniform codes from Philox TAG_INIT (R4)                 */
+  uint64_t init_seed;
+  int32_t cluster_size;  /* 0 = auto; else CTAs per network (1..16)                    */
+  int32_t reserved0;
+} snn_params;
+
+/* Table I rows */
+#define SNN_PRESET_2B  0
+#define SNN_PRESET_4B  1
+#define SNN_PRESET_8B  2
+#define SNN_PRESET_16B 3   /* parameters only: 16-bit codes are not built (SNN_EINVAL at create) */
+#define SNN_PRESET_HF  4   /* "high frequency": 5-78 Hz, tau_pot 80, tau_dep 5 */
+int snn_params_preset(snn_params* p, int preset);
+
+typedef struct snn_handle snn_handle;
+
+/* Create a network n_in -> n_exc with `bits`-bit conductance codes (2, 4 or 8).
+ * Conductances are initialised on the device (R4).  SNN_ESIZE if the network does not fit the
+ * on-chip layout.  *out receives the handle. */
+int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** out);
+int snn_destroy(snn_handle* h);
+
+/* Stream used by every subsequent call on h (a cudaStream_t; NULL = the handle's own stream). */
+int snn_set_stream(snn_handle* h, void* cuda_stream);
+/* Block until all work enqueued on h has finished. */
+int snn_synchronize(snn_handle* h);
+
+/* flags */
+#define SNN_RASTER_INPUT  1   /* `input` is a T x ceil(n_in/32) u32 input spike raster (encoder bypassed) */
+#define SNN_KEEP_STATE    2   /* keep v / counters / timers; steps are numbered t0 .. t0+T-1              */
+#define SNN_RECORD_INPUT  4   /* also record the input raster of the last image (snn_get_input_raster)    */
+#define SNN_ASYNC         8   /* return after enqueueing; host buffers must stay valid until synchronize  */
+
+/* Present one image (n_in bytes, host or device) for T steps with learning on ("Each image is
+ * presented to the network for t_learn ms").  `seed` keys every random draw of the presentation. */
+int snn_present(snn_handle* h, const uint8_t* image, int T, uint64_t seed);
+
+/* Present n_images images back to back in ONE kernel launch (weights stay resident on chip
+ * between images).  images: n_images x n_in bytes; seeds: n_images (both host or device).
+ * spike_counts (optional, host or device, n_images int32): post spikes per image. */
+int snn_present_batch(snn_handle* h, const uint8_t* images, int n_images, int T, const uint64_t* seeds,
+                      int32_t* spike_counts, int flags);
+
+/* General form: input is an image (n_in bytes) or, with SNN_RASTER_INPUT, a T x ceil(n_in/32)
+ * u32 raster (host or device); t0 is the first step index (only meaningful with SNN_KEEP_STATE). */
+int snn_present_ex(snn_handle* h, const void* input, int T, uint64_t seed, int flags, int t0);
+
+/* Test hook: present a given input raster (T x ceil(n_in/32) u32), encoder bypassed. */
+int snn_present_raster(snn_handle* h, const uint32_t* raster, int T, uint64_t seed);
+
+/* Ensemble: n independent handles (equal n_in, n_exc, cluster size; bits and parameters may
+ * differ) each present n_images images in ONE launch.  images[k]: n_images x n_in bytes and
+ * seeds[k]: n_images seeds for handle k (arrays of host pointers to host or device buffers). */
+int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images, int n_images, int T,
+                     const uint64_t* const* seeds);
+
+/* Readout.  codes: n_in x n_exc bytes, row-major [i][j], one code per byte (G = code * 2^-frac_bits). */
+int snn_get_weights(snn_handle* h, uint8_t* codes, size_t cap);
+int snn_set_weights(snn_handle* h, const uint8_t* codes, size_t n);
+/* Output raster of the last presented image: T x ceil(n_exc/32) u32, bit j%32 of word j/32. */
+int snn_get_spikes(snn_handle* h, uint32_t* raster, size_t cap_words);
+/* Input raster of the last presented image (requires SNN_RECORD_INPUT): T x ceil(n_in/32) u32. */
+int snn_get_input_raster(snn_handle* h, uint32_t* raster, size_t cap_words);
+/* State blob: int32 {n_in, n_exc, t_next, membrane_mode}, v[n_exc] (fp32 bits
+ * or Q15.16), cnt[n_exc], last_post[n_exc], last_pre[n_in]. */
+size_t snn_state_bytes(const snn_handle* h);
+int snn_get_state(snn_handle* h, void* buf, size_t cap);
+int snn_set_state(snn_handle* h, const void* buf, size_t n);
+/* Counters accumulated since the last snn_reset_stats: [0] sum_t act(t) (active input rows),
+ * [1] post spikes, [2] LTD trials, [3] LTD events, [4] LTP trials, [5] LTP events,
+ * [6] images presented, [7] steps simulated. */
+int snn_get_stats(snn_handle* h, uint64_t stats[8]);
+int snn_reset_stats(snn_handle* h);
+/* Introspection: [0] cluster size, [1] threads per CTA, [2] dynamic smem bytes per CTA,
+ * [3] words per weight row in a CTA slice, [4] q_max, [5] L_pot, [6] L_dep, [7] kernel launches so far. */
+int snn_get_info(const snn_handle* h, int64_t info[8]);
+
+const char* snn_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SNN_H */
