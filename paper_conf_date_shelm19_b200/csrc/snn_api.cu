@@ -1,0 +1,703 @@
+// snn_api.cu -- host runtime behind include/snn.h: parameter validation, host-side probability
+// tables (built here in double precision, independently of the CPU oracle), device allocation,
+// the on-chip layout choice, launches and readout.
+#include "snn.h"
+#include "snn_internal.h"
+
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+using snn::NetDesc;
+
+namespace {
+
+thread_local std::string g_err;
+
+int fail(int code, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return code;
+}
+
+#define CUDA_TRY(expr)                                                                          \
+  do {                                                                                          \
+    cudaError_t _e = (expr);                                                                    \
+    if (_e != cudaSuccess) return fail(SNN_ECUDA, "%s: %s (%s:%d)", #expr, cudaGetErrorString(_e), \
+                                       __FILE__, __LINE__);                                     \
+  } while (0)
+
+template <class T>
+cudaError_t dalloc(T** p, size_t n) {
+  *p = nullptr;
+  if (n == 0) n = 1;
+  return cudaMalloc(reinterpret_cast<void**>(p), n * sizeof(T));
+}
+
+bool is_device_ptr(const void* p) {
+  if (!p) return false;
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+// threshold of an event of probability P: floor(P * 2^32) (R13)
+unsigned long long prob_thr(double P) { return (unsigned long long)std::floor(std::ldexp(P, 32)); }
+
+}  // namespace
+
+struct snn_handle {
+  int dev = 0;
+  int n_in = 0, n_exc = 0, bits = 0, frac_bits = 0, q_max = 0;
+  snn_params p{};
+  int cs = 1, nthr = 128, wpr = 0, ngroups = 0, slice_words = 0;
+  size_t smem = 0;
+  int L_pot = 0, L_dep = 0;
+  // fixed / fp32 constants
+  long long A = 0, B = 0, C = 0, E = 0;
+  int Vth = 0, Vreset = 0, Vinit = 0;
+  // device memory
+  uint32_t* d_w = nullptr;
+  unsigned long long* d_enc = nullptr;
+  uint32_t* d_pot = nullptr;
+  uint32_t* d_dep = nullptr;
+  int* d_dbp = nullptr;
+  int* d_dbd = nullptr;
+  uint32_t* d_dtp = nullptr;
+  uint32_t* d_dtd = nullptr;
+  int* d_v = nullptr;
+  int* d_cnt = nullptr;
+  int* d_lpost = nullptr;
+  int* d_lpre = nullptr;
+  unsigned long long* d_stats = nullptr;
+  uint32_t* d_raster = nullptr;  size_t raster_cap = 0;
+  uint32_t* d_inrec = nullptr;   size_t inrec_cap = 0;
+  uint8_t* d_img = nullptr;      size_t img_cap = 0;
+  uint32_t* d_rin = nullptr;     size_t rin_cap = 0;
+  unsigned long long* d_seeds = nullptr; size_t seeds_cap = 0;
+  int* d_counts = nullptr;       size_t counts_cap = 0;
+  uint8_t* d_codes = nullptr;
+  int* d_bad = nullptr;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  int last_T = 0;
+  bool last_recorded = false;
+  int t_next = 0;
+  long long launches = 0;
+};
+
+namespace {
+
+int validate(int n_in, int n_exc, int bits, const snn_params* p) {
+  if (!p) return fail(SNN_EINVAL, "params is NULL");
+  if (n_in < 1 || n_in > 8192) return fail(SNN_EINVAL, "n_in=%d outside [1, 8192]", n_in);
+  if (n_exc < 1 || n_exc > (1 << 20)) return fail(SNN_EINVAL, "n_exc=%d outside [1, 2^20]", n_exc);
+  if (bits != 2 && bits != 4 && bits != 8) return fail(SNN_EINVAL, "bits=%d not in {2,4,8}", bits);
+  if (!(p->dt_ms > 0.0)) return fail(SNN_EINVAL, "dt_ms must be > 0");
+  if (!(p->f_min_hz >= 0.0 && p->f_max_hz >= p->f_min_hz)) return fail(SNN_EINVAL, "need 0 <= f_min <= f_max");
+  if (p->f_max_hz * p->dt_ms * 1e-3 > 1.0) return fail(SNN_EINVAL, "f_max * dt > 1 (spike probability > 1)");
+  if (!(p->gamma_pot >= 0.0 && p->gamma_pot <= 1.0 && p->gamma_dep >= 0.0 && p->gamma_dep <= 1.0))
+    return fail(SNN_EINVAL, "gamma must lie in [0, 1]");
+  if (!(p->tau_pot > 0.0 && p->tau_dep > 0.0)) return fail(SNN_EINVAL, "tau must be > 0");
+  if (p->t_ref_steps < 0 || p->t_inh_steps < 0 || p->t_ltp_steps < 0) return fail(SNN_EINVAL, "negative step count");
+  if (p->wta_mode < 0 || p->wta_mode > 1 || p->inh_mode < 0 || p->inh_mode > 1) return fail(SNN_EINVAL, "bad wta/inh mode");
+  if (p->stdp_mode < 0 || p->stdp_mode > 1 || p->rounding < 0 || p->rounding > 2) return fail(SNN_EINVAL, "bad stdp/rounding mode");
+  if (p->membrane_mode < 0 || p->membrane_mode > 1) return fail(SNN_EINVAL, "bad membrane_mode");
+  if (p->g_min != 0.0 || !(p->g_max > 0.0)) return fail(SNN_EINVAL, "need g_min == 0 and g_max > 0 (R9)");
+  if (p->frac_bits < 0 || p->frac_bits > 16) return fail(SNN_EINVAL, "frac_bits outside [0, 16]");
+  if (p->init_mode != 0) return fail(SNN_EINVAL, "init_mode must be 0");
+  if (p->stdp_mode == 1 && !(p->alpha_p >= 0 && p->alpha_d >= 0 && p->beta_p >= 0 && p->beta_d >= 0))
+    return fail(SNN_EINVAL, "alpha/beta must be >= 0");
+  if (p->cluster_size < 0 || p->cluster_size > snn::kMaxCluster) return fail(SNN_EINVAL, "cluster_size outside [0, 16]");
+  return SNN_OK;
+}
+
+// eqs.(6)(7) tables (R10, R19): u32 (thr - 1) for D < L, where thr = floor(gamma e^{-D dt/tau} 2^32) >= 1
+int exp_table(double gamma, double tau, double dt, std::vector<uint32_t>& out) {
+  out.clear();
+  if (gamma == 0.0) return SNN_OK;
+  for (int D = 0; D < snn::kLutMax; ++D) {
+    const unsigned long long thr = prob_thr(gamma * std::exp(-((double)D * dt) / tau));
+    if (thr == 0) return SNN_OK;
+    out.push_back((uint32_t)(thr - 1ull));
+  }
+  return fail(SNN_EINVAL, "STDP horizon exceeds %d steps (R19): gamma=%g tau=%g", snn::kLutMax, gamma, tau);
+}
+
+void fill_static(const snn_handle* h, NetDesc& d) {
+  std::memset(&d, 0, sizeof(d));
+  const snn_params& p = h->p;
+  d.n_in = h->n_in; d.n_exc = h->n_exc; d.bits = h->bits; d.q_max = h->q_max;
+  d.cs = h->cs; d.ngroups = h->ngroups; d.wpr = h->wpr;
+  d.nwi = (h->n_in + 31) / 32; d.nwe = (h->n_exc + 31) / 32;
+  d.membrane_mode = p.membrane_mode;
+  const double lsb = std::ldexp(1.0, -h->frac_bits);
+  d.af = (float)p.a; d.bf = (float)p.b; d.cf = (float)p.c; d.dtf = (float)p.dt_ms;
+  d.kI = (float)(p.v_spike * lsb); d.ief = (float)p.i_ext;
+  d.vthf = (float)p.v_th; d.vresetf = (float)p.v_reset; d.vinitf = (float)p.v_init;
+  d.A = h->A; d.B = h->B; d.C = h->C; d.E = h->E;
+  d.Vth = h->Vth; d.Vreset = h->Vreset; d.Vinit = h->Vinit;
+  d.t_ref = p.t_ref_steps; d.t_inh = p.t_inh_steps; d.wta_mode = p.wta_mode; d.inh_mode = p.inh_mode;
+  d.stdp_mode = p.stdp_mode; d.t_ltp = p.t_ltp_steps;
+  d.L_pot = h->L_pot; d.L_dep = h->L_dep;
+  d.thr_enc = h->d_enc; d.pot_m1 = h->d_pot; d.dep_m1 = h->d_dep;
+  d.det_base_p = h->d_dbp; d.det_thr_p = h->d_dtp; d.det_base_d = h->d_dbd; d.det_thr_d = h->d_dtd;
+  d.wslices = h->d_w;
+  d.v = h->d_v; d.cnt = h->d_cnt; d.last_post = h->d_lpost; d.last_pre = h->d_lpre;
+  d.stats = h->d_stats;
+}
+
+void free_all(snn_handle* h) {
+  void* ptrs[] = {h->d_w, h->d_enc, h->d_pot, h->d_dep, h->d_dbp, h->d_dbd, h->d_dtp, h->d_dtd,
+                  h->d_v, h->d_cnt, h->d_lpost, h->d_lpre, h->d_stats, h->d_raster, h->d_inrec,
+                  h->d_img, h->d_rin, h->d_seeds, h->d_counts, h->d_codes, h->d_bad};
+  for (void* q : ptrs) if (q) cudaFree(q);
+  if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
+}
+
+template <class T>
+int ensure(snn_handle* h, T** buf, size_t* cap, size_t need) {
+  if (*cap >= need && *buf) return SNN_OK;
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  if (*buf) cudaFree(*buf);
+  *buf = nullptr;
+  *cap = 0;
+  CUDA_TRY(dalloc(buf, need));
+  *cap = need;
+  return SNN_OK;
+}
+
+struct DevGuard {
+  int prev = -1;
+  explicit DevGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DevGuard() { if (prev >= 0) cudaSetDevice(prev); }
+};
+
+// Stage one input array onto the device (returns a device pointer valid on h->stream).
+template <class T>
+int stage(snn_handle* h, const T* src, size_t n, T** dbuf, size_t* cap, const T** out) {
+  if (is_device_ptr(src)) { *out = src; return SNN_OK; }
+  int rc = ensure(h, dbuf, cap, n);
+  if (rc) return rc;
+  CUDA_TRY(cudaMemcpyAsync(*dbuf, src, n * sizeof(T), cudaMemcpyHostToDevice, h->stream));
+  *out = *dbuf;
+  return SNN_OK;
+}
+
+int check_handle(const snn_handle* h) {
+  if (!h) return fail(SNN_EINVAL, "handle is NULL");
+  return SNN_OK;
+}
+
+int finish(snn_handle* h, int flags) {
+  CUDA_TRY(cudaGetLastError());
+  if (!(flags & SNN_ASYNC)) CUDA_TRY(cudaStreamSynchronize(h->stream));
+  return SNN_OK;
+}
+
+// Common path of every single-handle presentation.
+int present_impl(snn_handle* h, const void* input, int n_images, int T, const uint64_t* seeds, int32_t* counts,
+                 int flags, int t0) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  if (n_images < 0 || T < 0 || t0 < 0) return fail(SNN_EINVAL, "negative n_images / T / t0");
+  if ((flags & SNN_KEEP_STATE) && n_images > 1) return fail(SNN_EINVAL, "SNN_KEEP_STATE needs n_images == 1");
+  if ((flags & SNN_RASTER_INPUT) && n_images > 1) return fail(SNN_EINVAL, "SNN_RASTER_INPUT needs n_images == 1");
+  if (!(flags & SNN_KEEP_STATE) && t0 != 0) return fail(SNN_EINVAL, "t0 != 0 requires SNN_KEEP_STATE");
+  if (n_images == 0) {   // nothing to present (a T == 0 presentation still runs: it resets the state, R5)
+    h->last_T = 0;
+    return SNN_OK;
+  }
+  if (!input || !seeds) return fail(SNN_EINVAL, "input / seeds is NULL");
+  DevGuard g(h->dev);
+  NetDesc d;
+  fill_static(h, d);
+  d.n_images = n_images; d.T = T; d.flags = flags & 0x7; d.t0 = t0;
+  const int nwi = d.nwi, nwe = d.nwe;
+  if (flags & SNN_RASTER_INPUT) {
+    const uint32_t* rin = nullptr;
+    rc = stage(h, static_cast<const uint32_t*>(input), (size_t)T * nwi, &h->d_rin, &h->rin_cap, &rin);
+    if (rc) return rc;
+    d.in_raster = rin;
+  } else {
+    const uint8_t* img = nullptr;
+    rc = stage(h, static_cast<const uint8_t*>(input), (size_t)n_images * h->n_in, &h->d_img, &h->img_cap, &img);
+    if (rc) return rc;
+    d.images = img;
+  }
+  const unsigned long long* sd = nullptr;
+  rc = stage(h, reinterpret_cast<const unsigned long long*>(seeds), (size_t)n_images, &h->d_seeds, &h->seeds_cap, &sd);
+  if (rc) return rc;
+  d.seeds = sd;
+  rc = ensure(h, &h->d_raster, &h->raster_cap, (size_t)T * nwe);
+  if (rc) return rc;
+  d.raster_out = h->d_raster;
+  if (flags & SNN_RECORD_INPUT) {
+    rc = ensure(h, &h->d_inrec, &h->inrec_cap, (size_t)T * nwi);
+    if (rc) return rc;
+    d.in_raster_out = h->d_inrec;
+  }
+  const bool counts_dev = counts && is_device_ptr(counts);
+  if (counts && !counts_dev) {
+    rc = ensure(h, &h->d_counts, &h->counts_cap, (size_t)n_images);
+    if (rc) return rc;
+    d.spike_counts = h->d_counts;
+  } else {
+    d.spike_counts = counts;
+  }
+  snn::LaunchParams lp;
+  lp.descs = nullptr;
+  lp.single = d;
+  CUDA_TRY(snn::launch_present(lp, 1, h->cs, h->nthr, h->smem, h->stream));
+  h->launches++;
+  if (counts && !counts_dev)
+    CUDA_TRY(cudaMemcpyAsync(counts, h->d_counts, sizeof(int32_t) * n_images, cudaMemcpyDeviceToHost, h->stream));
+  h->last_T = T;
+  h->last_recorded = (flags & SNN_RECORD_INPUT) != 0;
+  h->t_next = ((flags & SNN_KEEP_STATE) ? t0 : 0) + T;
+  return finish(h, flags);
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* snn_last_error(void) { return g_err.c_str(); }
+
+int snn_params_preset(snn_params* p, int preset) {
+  if (!p) return fail(SNN_EINVAL, "params is NULL");
+  std::memset(p, 0, sizeof(*p));
+  // P:90 §III-D
+  p->a = -6.77; p->b = -0.0989; p->c = 0.314; p->v_th = -60.2; p->v_reset = -74.7; p->v_init = -70.0;
+  p->dt_ms = 1.0; p->v_spike = 2.0; p->i_ext = 0.0;          // R1, R3
+  p->t_ref_steps = 5; p->t_inh_steps = 10;                     // R6, R7
+  p->wta_mode = SNN_WTA_HARD; p->inh_mode = SNN_INH_RESET;
+  p->stdp_mode = SNN_STDP_STOCH; p->rounding = SNN_ROUND_NEAREST; p->t_ltp_steps = 20;
+  p->membrane_mode = SNN_MEM_FP32;
+  // Table I "16 bit" row alpha/beta (R16) for the deterministic arm at every width
+  p->alpha_p = 0.01; p->beta_p = 3.0; p->alpha_d = 0.005; p->beta_d = 3.0; p->g_min = 0.0; p->g_max = 1.0;
+  p->frac_bits = 0; p->init_mode = 0; p->init_seed = 1; p->cluster_size = 0;
+  p->f_min_hz = 1.0; p->f_max_hz = 22.0;
+  switch (preset) {   // Table I
+    case SNN_PRESET_2B:  p->gamma_pot = 0.2; p->tau_pot = 20; p->gamma_dep = 0.2; p->tau_dep = 10; break;
+    case SNN_PRESET_4B:  p->gamma_pot = 0.3; p->tau_pot = 30; p->gamma_dep = 0.3; p->tau_dep = 10; break;
+    case SNN_PRESET_8B:  p->gamma_pot = 0.5; p->tau_pot = 30; p->gamma_dep = 0.5; p->tau_dep = 10; break;
+    case SNN_PRESET_16B: p->gamma_pot = 0.9; p->tau_pot = 30; p->gamma_dep = 0.9; p->tau_dep = 10; break;
+    case SNN_PRESET_HF:
+      p->gamma_pot = 0.3; p->tau_pot = 80; p->gamma_dep = 0.2; p->tau_dep = 5;
+      p->f_min_hz = 5.0; p->f_max_hz = 78.0;
+      break;
+    default: return fail(SNN_EINVAL, "unknown preset %d", preset);
+  }
+  return SNN_OK;
+}
+
+int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** out) {
+  if (!out) return fail(SNN_EINVAL, "out is NULL");
+  *out = nullptr;
+  int rc = validate(n_in, n_exc, bits, p);
+  if (rc) return rc;
+  snn_handle* h = new (std::nothrow) snn_handle();
+  if (!h) return fail(SNN_ENOMEM, "host allocation failed");
+  h->p = *p;
+  h->n_in = n_in; h->n_exc = n_exc; h->bits = bits;
+  h->frac_bits = p->frac_bits > 0 ? p->frac_bits : bits;
+  h->q_max = (1 << bits) - 1;
+  if (h->frac_bits != bits) {
+    const double cap = std::floor(std::ldexp(p->g_max, h->frac_bits));
+    if (cap < h->q_max) h->q_max = (int)cap;
+  }
+  const double lsb = std::ldexp(1.0, -h->frac_bits);
+
+  // ---- host tables, built in double precision
+  unsigned long long enc[256];
+  for (int x = 0; x < 256; ++x)
+    enc[x] = prob_thr((p->f_min_hz + (p->f_max_hz - p->f_min_hz) * (double)x / 255.0) * p->dt_ms * 1e-3);
+  std::vector<uint32_t> pot, dep;
+  if ((rc = exp_table(p->gamma_pot, p->tau_pot, p->dt_ms, pot)) || (rc = exp_table(p->gamma_dep, p->tau_dep, p->dt_ms, dep))) {
+    delete h;
+    return rc;
+  }
+  h->L_pot = (int)pot.size();
+  h->L_dep = (int)dep.size();
+  std::vector<int> dbp(h->q_max + 1), dbd(h->q_max + 1);
+  std::vector<uint32_t> dtp(h->q_max + 1), dtd(h->q_max + 1);
+  for (int q = 0; q <= h->q_max; ++q) {     // eqs.(4)(5) in LSB units, R16/R17
+    const double G = (double)q * lsb;
+    const double x_p = std::ldexp(p->alpha_p * std::exp(-p->beta_p * (G - p->g_min) / (p->g_max - p->g_min)), h->frac_bits);
+    const double x_d = std::ldexp(p->alpha_d * std::exp(-p->beta_d * (p->g_max - G) / (p->g_max - p->g_min)), h->frac_bits);
+    for (int s = 0; s < 2; ++s) {
+      const double x = s == 0 ? x_p : x_d;
+      double base;
+      unsigned long long thr = 0;
+      if (p->rounding == SNN_ROUND_TRUNC) base = std::floor(x);
+      else if (p->rounding == SNN_ROUND_NEAREST) base = std::floor(x + 0.5);
+      else { base = std::floor(x); thr = prob_thr(x - std::floor(x)); }
+      const int bi = base > 1e9 ? 1000000000 : (int)base;
+      if (s == 0) { dbp[q] = bi; dtp[q] = (uint32_t)thr; } else { dbd[q] = bi; dtd[q] = (uint32_t)thr; }
+    }
+  }
+  h->A = std::llround(p->dt_ms * p->a * 65536.0);
+  h->B = std::llround(p->dt_ms * p->b * 4294967296.0);
+  h->C = std::llround(p->dt_ms * p->c * p->v_spike * lsb * 4294967296.0);
+  h->E = std::llround(p->dt_ms * p->c * p->i_ext * 65536.0);
+  h->Vth = (int)std::llround(p->v_th * 65536.0);
+  h->Vreset = (int)std::llround(p->v_reset * 65536.0);
+  h->Vinit = (int)std::llround(p->v_init * 65536.0);
+
+  // ---- device + on-chip layout
+  int ndev = 0;
+  cudaError_t ce = cudaGetDeviceCount(&ndev);
+  if (ce != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    delete h;
+    return fail(SNN_ECUDA, "no CUDA device: %s", cudaGetErrorString(ce));
+  }
+  cudaGetDevice(&h->dev);
+  int smem_optin = 0;
+  cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, h->dev);
+  h->ngroups = (n_exc + 31) / 32;
+  int chosen = 0;
+  const int cs_lo = p->cluster_size > 0 ? p->cluster_size : 1;
+  const int cs_hi = p->cluster_size > 0 ? p->cluster_size : snn::kMaxCluster;
+  for (int cs = cs_lo; cs <= cs_hi; ++cs) {
+    if (cs > h->ngroups) break;
+    const int max_groups = (h->ngroups + cs - 1) / cs;
+    if (max_groups * 32 > snn::kMaxThreads) continue;
+    const int nthr = max_groups * 32 < 128 ? 128 : max_groups * 32;
+    const int wpr = max_groups * bits;
+    const int sw = ((n_in * wpr) + 3) & ~3;
+    const size_t smem = snn::present_smem_bytes(n_in, sw, h->L_pot, h->L_dep, h->q_max, nthr);
+    if (smem > (size_t)smem_optin) continue;
+    h->cs = cs; h->nthr = nthr; h->wpr = wpr; h->slice_words = sw; h->smem = smem;
+    chosen = 1;
+    break;
+  }
+  if (!chosen) {
+    delete h;
+    return fail(SNN_ESIZE, "network %dx%d at %d bits does not fit one cluster of <= 16 CTAs (%d B smem/CTA)",
+                n_in, n_exc, bits, smem_optin);
+  }
+  int nclusters = 0;
+  ce = snn::query_max_clusters(h->cs, h->nthr, h->smem, &nclusters);
+  if (ce != cudaSuccess || nclusters < 1) {
+    cudaGetLastError();
+    delete h;
+    return fail(SNN_ECOOP, "cluster of %d CTAs x %zu B smem cannot be co-resident (%s)", h->cs, h->smem,
+                cudaGetErrorString(ce));
+  }
+
+#define ALLOC(ptr, n)                                                            \
+  do {                                                                           \
+    if (dalloc(&(ptr), (n)) != cudaSuccess) {                                    \
+      cudaGetLastError();                                                        \
+      free_all(h);                                                               \
+      delete h;                                                                  \
+      return fail(SNN_ENOMEM, "cudaMalloc failed for " #ptr);                    \
+    }                                                                            \
+  } while (0)
+  ALLOC(h->d_w, (size_t)h->cs * h->slice_words);
+  ALLOC(h->d_enc, 256);
+  ALLOC(h->d_pot, pot.size());
+  ALLOC(h->d_dep, dep.size());
+  ALLOC(h->d_dbp, (size_t)h->q_max + 1);
+  ALLOC(h->d_dbd, (size_t)h->q_max + 1);
+  ALLOC(h->d_dtp, (size_t)h->q_max + 1);
+  ALLOC(h->d_dtd, (size_t)h->q_max + 1);
+  ALLOC(h->d_v, (size_t)n_exc);
+  ALLOC(h->d_cnt, (size_t)n_exc);
+  ALLOC(h->d_lpost, (size_t)n_exc);
+  ALLOC(h->d_lpre, (size_t)n_in);
+  ALLOC(h->d_stats, 8);
+  ALLOC(h->d_codes, (size_t)n_in * n_exc);
+  ALLOC(h->d_bad, 1);
+#undef ALLOC
+  if (cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking) != cudaSuccess) {
+    free_all(h);
+    delete h;
+    return fail(SNN_ECUDA, "cudaStreamCreate failed");
+  }
+  h->own_stream = true;
+  auto up = [&](void* dst, const void* src, size_t bytes) {
+    return bytes ? cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, h->stream) : cudaSuccess;
+  };
+  cudaError_t e = cudaSuccess;
+  if (e == cudaSuccess) e = up(h->d_enc, enc, sizeof(enc));
+  if (e == cudaSuccess) e = up(h->d_pot, pot.data(), pot.size() * 4);
+  if (e == cudaSuccess) e = up(h->d_dep, dep.data(), dep.size() * 4);
+  if (e == cudaSuccess) e = up(h->d_dbp, dbp.data(), dbp.size() * 4);
+  if (e == cudaSuccess) e = up(h->d_dbd, dbd.data(), dbd.size() * 4);
+  if (e == cudaSuccess) e = up(h->d_dtp, dtp.data(), dtp.size() * 4);
+  if (e == cudaSuccess) e = up(h->d_dtd, dtd.data(), dtd.size() * 4);
+  // state after a reset (R5)
+  std::vector<int> v0(n_exc), m1(std::max(n_in, n_exc), snn::kNever);
+  if (p->membrane_mode == SNN_MEM_FIXED) std::fill(v0.begin(), v0.end(), h->Vinit);
+  else { float f = (float)p->v_init; int bitsf; std::memcpy(&bitsf, &f, 4); std::fill(v0.begin(), v0.end(), bitsf); }
+  if (e == cudaSuccess) e = up(h->d_v, v0.data(), (size_t)n_exc * 4);
+  if (e == cudaSuccess) e = cudaMemsetAsync(h->d_cnt, 0, (size_t)n_exc * 4, h->stream);
+  if (e == cudaSuccess) e = up(h->d_lpost, m1.data(), (size_t)n_exc * 4);
+  if (e == cudaSuccess) e = up(h->d_lpre, m1.data(), (size_t)n_in * 4);
+  if (e == cudaSuccess) e = cudaMemsetAsync(h->d_stats, 0, 8 * sizeof(unsigned long long), h->stream);
+  NetDesc d;
+  fill_static(h, d);
+  if (e == cudaSuccess) e = snn::launch_init_weights(d, p->init_seed, h->stream);   // R4
+  if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+  if (e != cudaSuccess) {
+    free_all(h);
+    delete h;
+    return fail(SNN_ECUDA, "create: %s", cudaGetErrorString(e));
+  }
+  h->launches = 1;
+  *out = h;
+  return SNN_OK;
+}
+
+int snn_destroy(snn_handle* h) {
+  if (!h) return SNN_OK;
+  DevGuard g(h->dev);
+  if (h->stream) cudaStreamSynchronize(h->stream);
+  free_all(h);
+  delete h;
+  return SNN_OK;
+}
+
+int snn_set_stream(snn_handle* h, void* s) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  DevGuard g(h->dev);
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  if (s) {
+    if (h->own_stream) cudaStreamDestroy(h->stream);
+    h->stream = static_cast<cudaStream_t>(s);
+    h->own_stream = false;
+  } else if (!h->own_stream) {
+    CUDA_TRY(cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking));
+    h->own_stream = true;
+  }
+  return SNN_OK;
+}
+
+int snn_synchronize(snn_handle* h) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  DevGuard g(h->dev);
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  return SNN_OK;
+}
+
+int snn_present(snn_handle* h, const uint8_t* image, int T, uint64_t seed) {
+  return present_impl(h, image, 1, T, &seed, nullptr, 0, 0);
+}
+
+int snn_present_ex(snn_handle* h, const void* input, int T, uint64_t seed, int flags, int t0) {
+  if (flags & SNN_ASYNC) return fail(SNN_EINVAL, "snn_present_ex is synchronous (seed is passed by value)");
+  return present_impl(h, input, 1, T, &seed, nullptr, flags, t0);
+}
+
+int snn_present_raster(snn_handle* h, const uint32_t* raster, int T, uint64_t seed) {
+  return present_impl(h, raster, 1, T, &seed, nullptr, SNN_RASTER_INPUT, 0);
+}
+
+int snn_present_batch(snn_handle* h, const uint8_t* images, int n_images, int T, const uint64_t* seeds,
+                      int32_t* spike_counts, int flags) {
+  if (flags & (SNN_RASTER_INPUT | SNN_KEEP_STATE)) return fail(SNN_EINVAL, "batch presentations take images, fresh state");
+  return present_impl(h, images, n_images, T, seeds, spike_counts, flags, 0);
+}
+
+int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images, int n_images, int T,
+                     const uint64_t* const* seeds) {
+  if (!hs || n < 1 || !images || !seeds) return fail(SNN_EINVAL, "bad ensemble arguments");
+  if (n_images < 0 || T < 0) return fail(SNN_EINVAL, "negative n_images / T");
+  for (int k = 0; k < n; ++k) {
+    if (!hs[k]) return fail(SNN_EINVAL, "handle %d is NULL", k);
+    if (hs[k]->n_in != hs[0]->n_in || hs[k]->cs != hs[0]->cs || hs[k]->nthr != hs[0]->nthr ||
+        hs[k]->dev != hs[0]->dev)
+      return fail(SNN_EINVAL, "ensemble handles must share n_in, cluster size, CTA shape and device");
+  }
+  if (n_images == 0 || T == 0) return SNN_OK;
+  snn_handle* h0 = hs[0];
+  DevGuard g(h0->dev);
+  size_t smem = 0;
+  for (int k = 0; k < n; ++k) smem = std::max(smem, hs[k]->smem);
+  std::vector<NetDesc> descs(n);
+  for (int k = 0; k < n; ++k) {
+    snn_handle* h = hs[k];
+    if (h != h0) CUDA_TRY(cudaStreamSynchronize(h->stream));
+    NetDesc& d = descs[k];
+    fill_static(h, d);
+    d.n_images = n_images; d.T = T; d.flags = 0; d.t0 = 0;
+    const uint8_t* img = nullptr;
+    int rc = stage(h0, images[k], (size_t)n_images * h->n_in, &h->d_img, &h->img_cap, &img);
+    if (rc) return rc;
+    const unsigned long long* sd = nullptr;
+    rc = stage(h0, reinterpret_cast<const unsigned long long*>(seeds[k]), (size_t)n_images, &h->d_seeds, &h->seeds_cap, &sd);
+    if (rc) return rc;
+    rc = ensure(h, &h->d_raster, &h->raster_cap, (size_t)T * d.nwe);
+    if (rc) return rc;
+    d.images = img; d.seeds = sd; d.raster_out = h->d_raster;
+  }
+  NetDesc* d_descs = nullptr;
+  CUDA_TRY(cudaMalloc(&d_descs, sizeof(NetDesc) * n));
+  CUDA_TRY(cudaMemcpyAsync(d_descs, descs.data(), sizeof(NetDesc) * n, cudaMemcpyHostToDevice, h0->stream));
+  snn::LaunchParams lp;
+  std::memset(&lp, 0, sizeof(lp));
+  lp.descs = d_descs;
+  cudaError_t e = snn::launch_present(lp, n, h0->cs, h0->nthr, smem, h0->stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(h0->stream);
+  cudaFree(d_descs);
+  if (e != cudaSuccess) return fail(SNN_ECUDA, "present_many: %s", cudaGetErrorString(e));
+  for (int k = 0; k < n; ++k) {
+    hs[k]->last_T = T;
+    hs[k]->last_recorded = false;
+    hs[k]->t_next = T;
+    hs[k]->launches++;
+  }
+  return SNN_OK;
+}
+
+int snn_get_weights(snn_handle* h, uint8_t* codes, size_t cap) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  const size_t n = (size_t)h->n_in * h->n_exc;
+  if (!codes) return fail(SNN_EINVAL, "codes is NULL");
+  if (cap < n) return fail(SNN_ESIZE, "need %zu bytes", n);
+  DevGuard g(h->dev);
+  NetDesc d;
+  fill_static(h, d);
+  CUDA_TRY(snn::launch_unpack_weights(d, h->d_codes, h->stream));
+  CUDA_TRY(cudaMemcpyAsync(codes, h->d_codes, n, is_device_ptr(codes) ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost,
+                           h->stream));
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  return SNN_OK;
+}
+
+int snn_set_weights(snn_handle* h, const uint8_t* codes, size_t n) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  const size_t need = (size_t)h->n_in * h->n_exc;
+  if (!codes) return fail(SNN_EINVAL, "codes is NULL");
+  if (n < need) return fail(SNN_ESIZE, "need %zu bytes", need);
+  DevGuard g(h->dev);
+  CUDA_TRY(cudaMemcpyAsync(h->d_codes, codes, need, is_device_ptr(codes) ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice,
+                           h->stream));
+  CUDA_TRY(cudaMemsetAsync(h->d_bad, 0, sizeof(int), h->stream));
+  CUDA_TRY(snn::launch_check_codes(h->d_codes, need, h->q_max, h->d_bad, h->stream));
+  int bad = 0;
+  CUDA_TRY(cudaMemcpyAsync(&bad, h->d_bad, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  if (bad) return fail(SNN_EINVAL, "%d codes exceed q_max=%d", bad, h->q_max);
+  NetDesc d;
+  fill_static(h, d);
+  CUDA_TRY(snn::launch_pack_weights(d, h->d_codes, h->stream));
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  return SNN_OK;
+}
+
+int snn_get_spikes(snn_handle* h, uint32_t* raster, size_t cap_words) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  const size_t need = (size_t)h->last_T * ((h->n_exc + 31) / 32);
+  if (cap_words < need) return fail(SNN_ESIZE, "need %zu words", need);
+  if (!need) return SNN_OK;
+  if (!raster) return fail(SNN_EINVAL, "raster is NULL");
+  DevGuard g(h->dev);
+  CUDA_TRY(cudaMemcpyAsync(raster, h->d_raster, need * 4, cudaMemcpyDefault, h->stream));
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  return SNN_OK;
+}
+
+int snn_get_input_raster(snn_handle* h, uint32_t* raster, size_t cap_words) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  if (!h->last_recorded) return fail(SNN_EINVAL, "last presentation did not set SNN_RECORD_INPUT");
+  const size_t need = (size_t)h->last_T * ((h->n_in + 31) / 32);
+  if (cap_words < need) return fail(SNN_ESIZE, "need %zu words", need);
+  if (!need) return SNN_OK;
+  if (!raster) return fail(SNN_EINVAL, "raster is NULL");
+  DevGuard g(h->dev);
+  CUDA_TRY(cudaMemcpyAsync(raster, h->d_inrec, need * 4, cudaMemcpyDefault, h->stream));
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  return SNN_OK;
+}
+
+size_t snn_state_bytes(const snn_handle* h) {
+  if (!h) return 0;
+  return sizeof(int32_t) * (4 + 3 * (size_t)h->n_exc + (size_t)h->n_in);
+}
+
+int snn_get_state(snn_handle* h, void* buf, size_t cap) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  if (!buf) return fail(SNN_EINVAL, "buf is NULL");
+  if (cap < snn_state_bytes(h)) return fail(SNN_ESIZE, "need %zu bytes", snn_state_bytes(h));
+  DevGuard g(h->dev);
+  int32_t* w = static_cast<int32_t*>(buf);
+  const size_t ne = (size_t)h->n_exc;
+  CUDA_TRY(cudaMemcpyAsync(w + 4, h->d_v, ne * 4, cudaMemcpyDeviceToHost, h->stream));
+  CUDA_TRY(cudaMemcpyAsync(w + 4 + ne, h->d_cnt, ne * 4, cudaMemcpyDeviceToHost, h->stream));
+  CUDA_TRY(cudaMemcpyAsync(w + 4 + 2 * ne, h->d_lpost, ne * 4, cudaMemcpyDeviceToHost, h->stream));
+  CUDA_TRY(cudaMemcpyAsync(w + 4 + 3 * ne, h->d_lpre, (size_t)h->n_in * 4, cudaMemcpyDeviceToHost, h->stream));
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  w[0] = h->n_in; w[1] = h->n_exc; w[2] = h->t_next; w[3] = h->p.membrane_mode;
+  return SNN_OK;
+}
+
+int snn_set_state(snn_handle* h, const void* buf, size_t n) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  if (!buf) return fail(SNN_EINVAL, "buf is NULL");
+  if (n < snn_state_bytes(h)) return fail(SNN_ESIZE, "need %zu bytes", snn_state_bytes(h));
+  const int32_t* w = static_cast<const int32_t*>(buf);
+  if (w[0] != h->n_in || w[1] != h->n_exc || w[3] != h->p.membrane_mode || w[2] < 0)
+    return fail(SNN_EINVAL, "state header does not match this handle");
+  DevGuard g(h->dev);
+  const size_t ne = (size_t)h->n_exc;
+  CUDA_TRY(cudaMemcpyAsync(h->d_v, w + 4, ne * 4, cudaMemcpyHostToDevice, h->stream));
+  CUDA_TRY(cudaMemcpyAsync(h->d_cnt, w + 4 + ne, ne * 4, cudaMemcpyHostToDevice, h->stream));
+  CUDA_TRY(cudaMemcpyAsync(h->d_lpost, w + 4 + 2 * ne, ne * 4, cudaMemcpyHostToDevice, h->stream));
+  CUDA_TRY(cudaMemcpyAsync(h->d_lpre, w + 4 + 3 * ne, (size_t)h->n_in * 4, cudaMemcpyHostToDevice, h->stream));
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  h->t_next = w[2];
+  return SNN_OK;
+}
+
+int snn_get_stats(snn_handle* h, uint64_t stats[8]) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  if (!stats) return fail(SNN_EINVAL, "stats is NULL");
+  DevGuard g(h->dev);
+  CUDA_TRY(cudaMemcpyAsync(stats, h->d_stats, 8 * sizeof(uint64_t), cudaMemcpyDeviceToHost, h->stream));
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  return SNN_OK;
+}
+
+int snn_reset_stats(snn_handle* h) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  DevGuard g(h->dev);
+  CUDA_TRY(cudaMemsetAsync(h->d_stats, 0, 8 * sizeof(unsigned long long), h->stream));
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  return SNN_OK;
+}
+
+int snn_get_info(const snn_handle* h, int64_t info[8]) {
+  if (!h || !info) return fail(SNN_EINVAL, "NULL argument");
+  info[0] = h->cs; info[1] = h->nthr; info[2] = (int64_t)h->smem; info[3] = h->wpr;
+  info[4] = h->q_max; info[5] = h->L_pot; info[6] = h->L_dep; info[7] = h->launches;
+  return SNN_OK;
+}
+
+}  // extern "C"

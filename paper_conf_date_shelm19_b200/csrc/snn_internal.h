@@ -1,0 +1,72 @@
+// snn_internal.h -- descriptor shared by the host runtime (snn_api.cu) and the kernels
+// (snn_kernels.cu).  CUDA path only; the CPU oracle (oracle/) shares nothing with it.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace snn {
+
+constexpr int kMaxCluster = 16;     // non-portable cluster size limit on B200
+constexpr int kMaxThreads = 1024;   // one column per thread -> <= 32 groups of 32 columns per CTA
+constexpr int kLutMax = 4096;       // R19
+constexpr int kNever = -1;
+
+enum : uint32_t { TAG_ENC = 1, TAG_LTD = 2, TAG_LTP = 3, TAG_ROUND = 4, TAG_INIT = 5 };
+enum : int { FLAG_RASTER_INPUT = 1, FLAG_KEEP_STATE = 2, FLAG_RECORD_INPUT = 4, FLAG_ASYNC = 8 };
+
+// Everything one network needs inside the persistent kernel.  Built per launch on the host.
+struct NetDesc {
+  // geometry
+  int n_in, n_exc, bits, q_max;
+  int cs;          // CTAs per network (= cluster size)
+  int ngroups;     // ceil(n_exc / 32): columns are sliced across CTAs in groups of 32
+  int wpr;         // u32 words per weight row of one CTA slice (max_groups * bits)
+  int nwi, nwe;    // u32 words per input / output raster row
+  // LIF
+  int membrane_mode;
+  float af, bf, cf, dtf, kI, ief, vthf, vresetf, vinitf;
+  long long A, B, C, E;
+  int Vth, Vreset, Vinit;
+  int t_ref, t_inh, wta_mode, inh_mode, stdp_mode, t_ltp;
+  int L_pot, L_dep;
+  // tables (device)
+  const unsigned long long* thr_enc;   // [256]      event iff u <  thr
+  const uint32_t* pot_m1;              // [L_pot]    event iff u <= thr - 1   (thr >= 1 for D < L)
+  const uint32_t* dep_m1;              // [L_dep]
+  const int* det_base_p;               // [q_max+1]  deterministic arm (R16/R17)
+  const uint32_t* det_thr_p;
+  const int* det_base_d;
+  const uint32_t* det_thr_d;
+  // persistent device state
+  uint32_t* wslices;                   // [cs][n_in][wpr] packed codes (the smem image of each CTA)
+  int* v;                              // [n_exc] fp32 bits or Q15.16
+  int* cnt;                            // [n_exc]
+  int* last_post;                      // [n_exc]
+  int* last_pre;                       // [n_in]
+  unsigned long long* stats;           // [8]
+  // per-launch I/O
+  const uint8_t* images;               // [n_images][n_in]
+  const uint32_t* in_raster;           // [T][nwi] with FLAG_RASTER_INPUT (n_images == 1)
+  const unsigned long long* seeds;     // [n_images]
+  uint32_t* raster_out;                // [T][nwe] output raster of the last image (may be null)
+  uint32_t* in_raster_out;             // [T][nwi] input raster of the last image (may be null)
+  int* spike_counts;                   // [n_images] (may be null)
+  int n_images, T, flags, t0;
+};
+
+struct LaunchParams {
+  const NetDesc* descs;   // device array (ensembles) or null -> use `single`
+  NetDesc single;
+};
+
+// kernels.cu entry points (host side)
+cudaError_t launch_present(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, cudaStream_t s);
+cudaError_t configure_present_kernel(size_t smem, int cs);
+cudaError_t query_max_clusters(int cs, int nthr, size_t smem, int* out);
+cudaError_t launch_init_weights(const NetDesc& d, uint64_t init_seed, cudaStream_t s);
+cudaError_t launch_pack_weights(const NetDesc& d, const uint8_t* codes, cudaStream_t s);
+cudaError_t launch_unpack_weights(const NetDesc& d, uint8_t* codes, cudaStream_t s);
+cudaError_t launch_check_codes(const uint8_t* codes, size_t n, int q_max, int* bad, cudaStream_t s);
+size_t present_smem_bytes(int n_in, int wpr, int L_pot, int L_dep, int q_max, int nthr);
+
+}  // namespace snn

@@ -1,0 +1,245 @@
+"""Thin ctypes binding of include/snn.h (libsnn_b200.so).  Argument marshalling only: every step
+of the simulate-and-learn path runs in the library's CUDA kernels.  There is no CPU fallback:
+if the in-tree extension is missing this module raises on import of the library."""
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import Optional, Sequence
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libsnn_b200.so")
+
+SNN_OK, SNN_EINVAL, SNN_ENOMEM, SNN_ECUDA, SNN_ENCCL, SNN_ESIZE, SNN_ECOOP = 0, -1, -2, -3, -4, -5, -6
+SNN_RASTER_INPUT, SNN_KEEP_STATE, SNN_RECORD_INPUT, SNN_ASYNC = 1, 2, 4, 8
+PRESETS = {"2b": 0, "4b": 1, "8b": 2, "16b": 3, "hf": 4}
+
+# Every function declared in include/snn.h (checked by tests/test_abi.py).
+EXPORTS = [
+    "snn_params_preset", "snn_create", "snn_destroy", "snn_set_stream", "snn_synchronize",
+    "snn_present", "snn_present_batch", "snn_present_ex", "snn_present_raster", "snn_present_many",
+    "snn_get_weights", "snn_set_weights", "snn_get_spikes", "snn_get_input_raster",
+    "snn_state_bytes", "snn_get_state", "snn_set_state", "snn_get_stats", "snn_reset_stats",
+    "snn_get_info", "snn_last_error",
+]
+
+
+class SnnParams(ctypes.Structure):
+    """snn_params (include/snn.h)."""
+    _fields_ = [
+        ("a", ctypes.c_double), ("b", ctypes.c_double), ("c", ctypes.c_double),
+        ("v_th", ctypes.c_double), ("v_reset", ctypes.c_double), ("v_init", ctypes.c_double),
+        ("dt_ms", ctypes.c_double), ("v_spike", ctypes.c_double), ("i_ext", ctypes.c_double),
+        ("t_ref_steps", ctypes.c_int32), ("t_inh_steps", ctypes.c_int32),
+        ("wta_mode", ctypes.c_int32), ("inh_mode", ctypes.c_int32),
+        ("f_min_hz", ctypes.c_double), ("f_max_hz", ctypes.c_double),
+        ("stdp_mode", ctypes.c_int32), ("rounding", ctypes.c_int32),
+        ("t_ltp_steps", ctypes.c_int32), ("membrane_mode", ctypes.c_int32),
+        ("gamma_pot", ctypes.c_double), ("tau_pot", ctypes.c_double),
+        ("gamma_dep", ctypes.c_double), ("tau_dep", ctypes.c_double),
+        ("alpha_p", ctypes.c_double), ("beta_p", ctypes.c_double),
+        ("alpha_d", ctypes.c_double), ("beta_d", ctypes.c_double),
+        ("g_min", ctypes.c_double), ("g_max", ctypes.c_double),
+        ("frac_bits", ctypes.c_int32), ("init_mode", ctypes.c_int32),
+        ("init_seed", ctypes.c_uint64),
+        ("cluster_size", ctypes.c_int32), ("reserved0", ctypes.c_int32),
+    ]
+
+    def as_dict(self) -> dict:
+        return {name: getattr(self, name) for name, _ in self._fields_}
+
+
+_lib = None
+
+
+def lib():
+    """Load the in-tree CUDA library (raises if it was not built: no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"CUDA extension not built: {LIB_PATH} (run __graft_entry__.build())")
+        L = ctypes.CDLL(LIB_PATH)
+        vp, i32, u64, sz = ctypes.c_void_p, ctypes.c_int, ctypes.c_uint64, ctypes.c_size_t
+        pp = ctypes.POINTER(SnnParams)
+        sig = {
+            "snn_params_preset": ([pp, i32], i32),
+            "snn_create": ([i32, i32, i32, pp, ctypes.POINTER(vp)], i32),
+            "snn_destroy": ([vp], i32),
+            "snn_set_stream": ([vp, vp], i32),
+            "snn_synchronize": ([vp], i32),
+            "snn_present": ([vp, vp, i32, u64], i32),
+            "snn_present_batch": ([vp, vp, i32, i32, vp, vp, i32], i32),
+            "snn_present_ex": ([vp, vp, i32, u64, i32, i32], i32),
+            "snn_present_raster": ([vp, vp, i32, u64], i32),
+            "snn_present_many": ([vp, i32, vp, i32, i32, vp], i32),
+            "snn_get_weights": ([vp, vp, sz], i32),
+            "snn_set_weights": ([vp, vp, sz], i32),
+            "snn_get_spikes": ([vp, vp, sz], i32),
+            "snn_get_input_raster": ([vp, vp, sz], i32),
+            "snn_state_bytes": ([vp], sz),
+            "snn_get_state": ([vp, vp, sz], i32),
+            "snn_set_state": ([vp, vp, sz], i32),
+            "snn_get_stats": ([vp, vp], i32),
+            "snn_reset_stats": ([vp], i32),
+            "snn_get_info": ([vp, vp], i32),
+            "snn_last_error": ([], ctypes.c_char_p),
+        }
+        for name, (args, res) in sig.items():
+            f = getattr(L, name)
+            f.argtypes = args
+            f.restype = res
+        _lib = L
+    return _lib
+
+
+class SnnError(RuntimeError):
+    def __init__(self, rc: int, what: str):
+        msg = lib().snn_last_error().decode(errors="replace")
+        super().__init__(f"{what} failed rc={rc}: {msg}")
+        self.rc = rc
+
+
+def _check(rc: int, what: str):
+    if rc != SNN_OK:
+        raise SnnError(rc, what)
+
+
+def preset(name: str = "8b", **overrides) -> SnnParams:
+    p = SnnParams()
+    _check(lib().snn_params_preset(ctypes.byref(p), PRESETS[name]), "snn_params_preset")
+    for k, v in overrides.items():
+        if not hasattr(p, k):
+            raise KeyError(k)
+        setattr(p, k, v)
+    return p
+
+
+def params_from_dict(d: dict) -> SnnParams:
+    p = SnnParams()
+    for name, _ in SnnParams._fields_:
+        setattr(p, name, d[name])
+    return p
+
+
+def _ptr(x) -> ctypes.c_void_p:
+    """Host numpy array or torch tensor (host or CUDA) -> raw pointer."""
+    if x is None:
+        return ctypes.c_void_p(0)
+    if isinstance(x, np.ndarray):
+        assert x.flags["C_CONTIGUOUS"]
+        return ctypes.c_void_p(x.ctypes.data)
+    if hasattr(x, "data_ptr"):
+        assert x.is_contiguous()
+        return ctypes.c_void_p(x.data_ptr())
+    raise TypeError(type(x))
+
+
+class Network:
+    """One snn_handle: n_in -> n_exc network with `bits`-bit conductance codes on the GPU."""
+
+    def __init__(self, n_in: int, n_exc: int, bits: int, params: Optional[SnnParams] = None, **overrides):
+        self.n_in, self.n_exc, self.bits = n_in, n_exc, bits
+        self.params = params if params is not None else preset({2: "2b", 4: "4b", 8: "8b"}[bits])
+        for k, v in overrides.items():
+            setattr(self.params, k, v)
+        self._h = ctypes.c_void_p()
+        _check(lib().snn_create(n_in, n_exc, bits, ctypes.byref(self.params), ctypes.byref(self._h)), "snn_create")
+        self.last_T = 0
+
+    @property
+    def handle(self) -> ctypes.c_void_p:
+        return self._h
+
+    def close(self):
+        if getattr(self, "_h", None) is not None and self._h.value:
+            lib().snn_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def info(self) -> dict:
+        a = (ctypes.c_int64 * 8)()
+        _check(lib().snn_get_info(self._h, a), "snn_get_info")
+        keys = ["cluster_size", "threads", "smem_bytes", "words_per_row", "q_max", "L_pot", "L_dep", "launches"]
+        return dict(zip(keys, [int(x) for x in a]))
+
+    def set_stream(self, stream_ptr: int):
+        _check(lib().snn_set_stream(self._h, ctypes.c_void_p(stream_ptr)), "snn_set_stream")
+
+    def synchronize(self):
+        _check(lib().snn_synchronize(self._h), "snn_synchronize")
+
+    def present(self, image, T: int, seed: int):
+        _check(lib().snn_present(self._h, _ptr(image), T, seed), "snn_present")
+        self.last_T = T
+
+    def present_ex(self, inp, T: int, seed: int, flags: int = 0, t0: int = 0):
+        _check(lib().snn_present_ex(self._h, _ptr(inp), T, seed, flags, t0), "snn_present_ex")
+        self.last_T = T
+
+    def present_raster(self, raster, T: int, seed: int, keep_state: bool = False, t0: int = 0):
+        flags = SNN_RASTER_INPUT | (SNN_KEEP_STATE if keep_state else 0)
+        self.present_ex(raster, T, seed, flags, t0)
+
+    def present_batch(self, images, T: int, seeds, spike_counts=None, flags: int = 0):
+        n = int(images.shape[0])
+        _check(lib().snn_present_batch(self._h, _ptr(images), n, T, _ptr(seeds), _ptr(spike_counts), flags),
+               "snn_present_batch")
+        self.last_T = T
+
+    def weights(self) -> np.ndarray:
+        out = np.empty((self.n_in, self.n_exc), dtype=np.uint8)
+        _check(lib().snn_get_weights(self._h, _ptr(out), out.nbytes), "snn_get_weights")
+        return out
+
+    def set_weights(self, codes: np.ndarray):
+        c = np.ascontiguousarray(codes, dtype=np.uint8).reshape(self.n_in, self.n_exc)
+        _check(lib().snn_set_weights(self._h, _ptr(c), c.nbytes), "snn_set_weights")
+
+    def spikes(self) -> np.ndarray:
+        we = (self.n_exc + 31) // 32
+        out = np.zeros((self.last_T, we), dtype=np.uint32)
+        _check(lib().snn_get_spikes(self._h, _ptr(out), out.size), "snn_get_spikes")
+        return out
+
+    def input_raster(self) -> np.ndarray:
+        wi = (self.n_in + 31) // 32
+        out = np.zeros((self.last_T, wi), dtype=np.uint32)
+        _check(lib().snn_get_input_raster(self._h, _ptr(out), out.size), "snn_get_input_raster")
+        return out
+
+    def state(self) -> np.ndarray:
+        n = int(lib().snn_state_bytes(self._h))
+        out = np.zeros(n // 4, dtype=np.int32)
+        _check(lib().snn_get_state(self._h, _ptr(out), out.nbytes), "snn_get_state")
+        return out
+
+    def set_state(self, blob: np.ndarray):
+        b = np.ascontiguousarray(blob, dtype=np.int32)
+        _check(lib().snn_set_state(self._h, _ptr(b), b.nbytes), "snn_set_state")
+
+    def stats(self) -> np.ndarray:
+        out = np.zeros(8, dtype=np.uint64)
+        _check(lib().snn_get_stats(self._h, _ptr(out)), "snn_get_stats")
+        return out
+
+    def reset_stats(self):
+        _check(lib().snn_reset_stats(self._h), "snn_reset_stats")
+
+
+def present_many(nets: Sequence[Network], images: Sequence, T: int, seeds: Sequence):
+    """Ensemble: every network presents its own image batch, all in one kernel launch."""
+    n = len(nets)
+    hs = (ctypes.c_void_p * n)(*[x.handle.value for x in nets])
+    imgs = (ctypes.c_void_p * n)(*[_ptr(a).value for a in images])
+    sds = (ctypes.c_void_p * n)(*[_ptr(s).value for s in seeds])
+    n_images = int(images[0].shape[0])
+    _check(lib().snn_present_many(hs, n, imgs, n_images, T, sds), "snn_present_many")
+    for x in nets:
+        x.last_T = T

@@ -1,5 +1,4 @@
 import os
-import subprocess
 import sys
 
 import pytest
@@ -22,7 +21,18 @@ def _ensure_oracle_built():
         __graft_entry__.build_oracle()
 
 
+def _ensure_cuda_built():
+    lib = os.path.join(ROOT, "paper_conf_date_shelm19_b200", "libsnn_b200.so")
+    csrc = os.path.join(ROOT, "paper_conf_date_shelm19_b200", "csrc")
+    newest = max(os.path.getmtime(os.path.join(csrc, f)) for f in os.listdir(csrc))
+    newest = max(newest, os.path.getmtime(os.path.join(ROOT, "include", "snn.h")))
+    if (not os.path.exists(lib)) or os.path.getmtime(lib) < newest:
+        import __graft_entry__  # noqa: E402
+        __graft_entry__.build_cuda()
+
+
 _ensure_oracle_built()
+_ensure_cuda_built()
 
 
 def cuda_available() -> bool:
