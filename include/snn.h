@@ -109,6 +109,7 @@ int snn_synchronize(snn_handle* h);
 #define SNN_KEEP_STATE    2   /* keep v / counters / timers; steps are numbered t0 .. t0+T-1              */
 #define SNN_RECORD_INPUT  4   /* also record the input raster of the last image (snn_get_input_raster)    */
 #define SNN_ASYNC         8   /* return after enqueueing; host buffers must stay valid until synchronize  */
+#define SNN_FLOOR_PROBE  16   /* benchmark probe: same launch shape, per-step barriers/exchange only, no work */
 
 /* Present one image (n_in bytes, host or device) for T steps with learning on ("Each image is
  * presented to the network for t_learn ms").  `seed` keys every random draw of the presentation. */

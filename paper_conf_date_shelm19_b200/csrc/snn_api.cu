@@ -225,7 +225,7 @@ int present_impl(snn_handle* h, const void* input, int n_images, int T, const ui
   DevGuard g(h->dev);
   NetDesc d;
   fill_static(h, d);
-  d.n_images = n_images; d.T = T; d.flags = flags & 0x7; d.t0 = t0;
+  d.n_images = n_images; d.T = T; d.flags = flags & 0x17; d.t0 = t0;
   const int nwi = d.nwi, nwe = d.nwe;
   if (flags & SNN_RASTER_INPUT) {
     const uint32_t* rin = nullptr;
@@ -514,6 +514,7 @@ int snn_present_raster(snn_handle* h, const uint32_t* raster, int T, uint64_t se
 int snn_present_batch(snn_handle* h, const uint8_t* images, int n_images, int T, const uint64_t* seeds,
                       int32_t* spike_counts, int flags) {
   if (flags & (SNN_RASTER_INPUT | SNN_KEEP_STATE)) return fail(SNN_EINVAL, "batch presentations take images, fresh state");
+  // SNN_FLOOR_PROBE (16): benchmark-only probe of the per-step synchronisation floor (no learning work)
   return present_impl(h, images, n_images, T, seeds, spike_counts, flags, 0);
 }
 

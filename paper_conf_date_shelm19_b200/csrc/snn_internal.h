@@ -12,7 +12,7 @@ constexpr int kLutMax = 4096;       // R19
 constexpr int kNever = -1;
 
 enum : uint32_t { TAG_ENC = 1, TAG_LTD = 2, TAG_LTP = 3, TAG_ROUND = 4, TAG_INIT = 5 };
-enum : int { FLAG_RASTER_INPUT = 1, FLAG_KEEP_STATE = 2, FLAG_RECORD_INPUT = 4, FLAG_ASYNC = 8 };
+enum : int { FLAG_RASTER_INPUT = 1, FLAG_KEEP_STATE = 2, FLAG_RECORD_INPUT = 4, FLAG_ASYNC = 8, FLAG_FLOOR = 16 };
 
 // Everything one network needs inside the persistent kernel.  Built per launch on the host.
 struct NetDesc {

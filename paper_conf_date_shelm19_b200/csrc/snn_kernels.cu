@@ -145,6 +145,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
   const bool hard = d.wta_mode == 0;
   const bool stoch = d.stdp_mode == 0;
   const bool inh_reset = d.inh_mode == 0;
+  const bool floor_mode = (flags & FLAG_FLOOR) != 0;   // bench: same launch shape, barriers + exchange only
 
   // ---- one-time staging: tables + this CTA's weight slice -> SMEM
   for (int k = tid; k < 256; k += nthr) s_enc[k] = d.thr_enc[k];
@@ -190,7 +191,9 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
       const int par = k & 1;
 
       // (a1) ENCODE: s_i = u_ENC(t, i) < thr_enc[x_i]   (R8, R13)
-      if (flags & FLAG_RASTER_INPUT) {
+      if (floor_mode) {
+        for (int w = tid; w < nwi; w += nthr) s_spk[w] = 0u;
+      } else if (flags & FLAG_RASTER_INPUT) {
         for (int w = tid; w < nwi; w += nthr) s_spk[w] = d.in_raster[(size_t)k * nwi + w];
       } else {
         for (int base = warp * 32; base < nq4; base += nthr) {     // warp-uniform trip count
@@ -246,7 +249,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
 
       // (a2) INTEGRATE eq.(3): S_j = sum_{active i} q_ij      (a3) LIF eqs.(1)(2)
       bool cand = false;
-      if (mycol) {
+      if (mycol && !floor_mode) {
         int S = 0;
         const uint32_t* wcol = s_w + wj;
         for (int a = 0; a < nact; ++a) S += (int)((wcol[(int)s_alist[a] * wpr] >> sh) & fmask);

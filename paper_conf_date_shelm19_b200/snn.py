@@ -13,7 +13,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libsnn_b200.so")
 
 SNN_OK, SNN_EINVAL, SNN_ENOMEM, SNN_ECUDA, SNN_ENCCL, SNN_ESIZE, SNN_ECOOP = 0, -1, -2, -3, -4, -5, -6
-SNN_RASTER_INPUT, SNN_KEEP_STATE, SNN_RECORD_INPUT, SNN_ASYNC = 1, 2, 4, 8
+SNN_RASTER_INPUT, SNN_KEEP_STATE, SNN_RECORD_INPUT, SNN_ASYNC, SNN_FLOOR_PROBE = 1, 2, 4, 8, 16
 PRESETS = {"2b": 0, "4b": 1, "8b": 2, "16b": 3, "hf": 4}
 
 # Every function declared in include/snn.h (checked by tests/test_abi.py).
