@@ -80,8 +80,12 @@ typedef struct snn_params {
   int32_t init_mode;     /* 0: uniform codes from Philox TAG_INIT (R4)                 */
   uint64_t init_seed;
   int32_t cluster_size;  /* 0 = auto; else CTAs per network (1..16)                    */
-  int32_t reserved0;
+  int32_t engine;        /* SNN_ENGINE_EVENT (0, default) or SNN_ENGINE_STEP (1) */
 } snn_params;
+
+/* engine: both give bit-identical results */
+#define SNN_ENGINE_EVENT 0   /* one cluster exchange per post-spike epoch; T <= 32767 */
+#define SNN_ENGINE_STEP  1   /* one cluster exchange per timestep */
 
 /* Table I rows */
 #define SNN_PRESET_2B  0

@@ -94,6 +94,13 @@ struct snn_handle {
   bool last_recorded = false;
   int t_next = 0;
   long long launches = 0;
+  // event engine
+  int engine = SNN_ENGINE_EVENT;
+  int rows_cap = 0, offs_cap = 0, logn = 0;
+  uint32_t* d_words = nullptr;   size_t words_cap = 0;
+  uint32_t* d_ecnt = nullptr;    size_t ecnt_cap = 0;
+  uint32_t* d_offs = nullptr;    size_t offs_buf_cap = 0;
+  uint16_t* d_rows = nullptr;    size_t rows_buf_cap = 0;
 };
 
 namespace {
@@ -119,6 +126,7 @@ int validate(int n_in, int n_exc, int bits, const snn_params* p) {
   if (p->stdp_mode == 1 && !(p->alpha_p >= 0 && p->alpha_d >= 0 && p->beta_p >= 0 && p->beta_d >= 0))
     return fail(SNN_EINVAL, "alpha/beta must be >= 0");
   if (p->cluster_size < 0 || p->cluster_size > snn::kMaxCluster) return fail(SNN_EINVAL, "cluster_size outside [0, 16]");
+  if (p->engine != SNN_ENGINE_EVENT && p->engine != SNN_ENGINE_STEP) return fail(SNN_EINVAL, "engine must be 0 or 1");
   return SNN_OK;
 }
 
@@ -155,12 +163,14 @@ void fill_static(const snn_handle* h, NetDesc& d) {
   d.wslices = h->d_w;
   d.v = h->d_v; d.cnt = h->d_cnt; d.last_post = h->d_lpost; d.last_pre = h->d_lpre;
   d.stats = h->d_stats;
+  d.rows_cap = h->rows_cap; d.offs_cap = h->offs_cap; d.logn = h->logn;
 }
 
 void free_all(snn_handle* h) {
   void* ptrs[] = {h->d_w, h->d_enc, h->d_pot, h->d_dep, h->d_dbp, h->d_dbd, h->d_dtp, h->d_dtd,
                   h->d_v, h->d_cnt, h->d_lpost, h->d_lpre, h->d_stats, h->d_raster, h->d_inrec,
-                  h->d_img, h->d_rin, h->d_seeds, h->d_counts, h->d_codes, h->d_bad};
+                  h->d_img, h->d_rin, h->d_seeds, h->d_counts, h->d_codes, h->d_bad,
+                  h->d_words, h->d_ecnt, h->d_offs, h->d_rows};
   for (void* q : ptrs) if (q) cudaFree(q);
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
 }
@@ -208,6 +218,37 @@ int finish(snn_handle* h, int flags) {
   return SNN_OK;
 }
 
+// Event engine pre-pass: encoder (or the given raster) -> per-step active-row lists.
+int event_prepass(snn_handle* h, NetDesc& d, const uint8_t* images, const uint32_t* raster, int n_images, int T,
+                  int t0, const unsigned long long* seeds) {
+  const int nwi = d.nwi;
+  int rc;
+  const uint32_t* words = nullptr;
+  if ((rc = ensure(h, &h->d_ecnt, &h->ecnt_cap, (size_t)n_images * T))) return rc;
+  if (raster) {
+    words = raster;
+    CUDA_TRY(snn::launch_counts_from_raster(raster, h->n_in, T, h->d_ecnt, h->stream));
+  } else {
+    if ((rc = ensure(h, &h->d_words, &h->words_cap, (size_t)n_images * T * nwi))) return rc;
+    CUDA_TRY(snn::launch_encode(images, h->d_enc, seeds, h->n_in, T, n_images, t0, h->d_words, h->d_ecnt, h->stream));
+    words = h->d_words;
+    h->launches++;
+  }
+  const long long stride = ((long long)T * h->n_in + 7) & ~7LL;
+  if ((rc = ensure(h, &h->d_offs, &h->offs_buf_cap, (size_t)n_images * (T + 1)))) return rc;
+  if ((rc = ensure(h, &h->d_rows, &h->rows_buf_cap, (size_t)n_images * stride))) return rc;
+  CUDA_TRY(snn::launch_compact(words, h->d_ecnt, h->n_in, T, n_images, stride, h->d_offs, h->d_rows, h->stream));
+  h->launches++;
+  d.ev_offs = h->d_offs;
+  d.ev_rows = h->d_rows;
+  d.rows_stride = stride;
+  if (d.in_raster_out)
+    CUDA_TRY(cudaMemcpyAsync(d.in_raster_out, words + (size_t)(n_images - 1) * T * nwi, (size_t)T * nwi * 4,
+                             cudaMemcpyDeviceToDevice, h->stream));
+  if (d.raster_out) CUDA_TRY(cudaMemsetAsync(d.raster_out, 0, (size_t)T * d.nwe * 4, h->stream));
+  return SNN_OK;
+}
+
 // Common path of every single-handle presentation.
 int present_impl(snn_handle* h, const void* input, int n_images, int T, const uint64_t* seeds, int32_t* counts,
                  int flags, int t0) {
@@ -217,6 +258,9 @@ int present_impl(snn_handle* h, const void* input, int n_images, int T, const ui
   if ((flags & SNN_KEEP_STATE) && n_images > 1) return fail(SNN_EINVAL, "SNN_KEEP_STATE needs n_images == 1");
   if ((flags & SNN_RASTER_INPUT) && n_images > 1) return fail(SNN_EINVAL, "SNN_RASTER_INPUT needs n_images == 1");
   if (!(flags & SNN_KEEP_STATE) && t0 != 0) return fail(SNN_EINVAL, "t0 != 0 requires SNN_KEEP_STATE");
+  const bool ev = h->engine == SNN_ENGINE_EVENT;
+  if (ev && T > snn::kEvMaxT) return fail(SNN_EINVAL, "T=%d exceeds %d for the event engine", T, snn::kEvMaxT);
+  if (ev && (flags & SNN_FLOOR_PROBE)) return fail(SNN_EINVAL, "SNN_FLOOR_PROBE applies to the per-step engine");
   if (n_images == 0) {   // nothing to present (a T == 0 presentation still runs: it resets the state, R5)
     h->last_T = 0;
     return SNN_OK;
@@ -227,13 +271,13 @@ int present_impl(snn_handle* h, const void* input, int n_images, int T, const ui
   fill_static(h, d);
   d.n_images = n_images; d.T = T; d.flags = flags & 0x17; d.t0 = t0;
   const int nwi = d.nwi, nwe = d.nwe;
+  const uint32_t* rin = nullptr;
+  const uint8_t* img = nullptr;
   if (flags & SNN_RASTER_INPUT) {
-    const uint32_t* rin = nullptr;
     rc = stage(h, static_cast<const uint32_t*>(input), (size_t)T * nwi, &h->d_rin, &h->rin_cap, &rin);
     if (rc) return rc;
     d.in_raster = rin;
   } else {
-    const uint8_t* img = nullptr;
     rc = stage(h, static_cast<const uint8_t*>(input), (size_t)n_images * h->n_in, &h->d_img, &h->img_cap, &img);
     if (rc) return rc;
     d.images = img;
@@ -260,8 +304,15 @@ int present_impl(snn_handle* h, const void* input, int n_images, int T, const ui
   }
   snn::LaunchParams lp;
   lp.descs = nullptr;
-  lp.single = d;
-  CUDA_TRY(snn::launch_present(lp, 1, h->cs, h->nthr, h->smem, h->stream));
+  if (ev) {
+    rc = event_prepass(h, d, img, rin, n_images, T, (flags & SNN_KEEP_STATE) ? t0 : 0, sd);
+    if (rc) return rc;
+    lp.single = d;
+    CUDA_TRY(snn::launch_present_event(lp, 1, h->cs, h->nthr, h->smem, h->stream));
+  } else {
+    lp.single = d;
+    CUDA_TRY(snn::launch_present(lp, 1, h->cs, h->nthr, h->smem, h->stream));
+  }
   h->launches++;
   if (counts && !counts_dev)
     CUDA_TRY(cudaMemcpyAsync(counts, h->d_counts, sizeof(int32_t) * n_images, cudaMemcpyDeviceToHost, h->stream));
@@ -370,19 +421,37 @@ int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** 
   int smem_optin = 0;
   cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, h->dev);
   h->ngroups = (n_exc + 31) / 32;
+  h->engine = p->engine;
   int chosen = 0;
   const int cs_lo = p->cluster_size > 0 ? p->cluster_size : 1;
   const int cs_hi = p->cluster_size > 0 ? p->cluster_size : snn::kMaxCluster;
+  const bool ev = h->engine == SNN_ENGINE_EVENT;
+  const int max_thr = ev ? snn::kEvMaxThreads : snn::kMaxThreads;
   for (int cs = cs_lo; cs <= cs_hi; ++cs) {
     if (cs > h->ngroups) break;
     const int max_groups = (h->ngroups + cs - 1) / cs;
-    if (max_groups * 32 > snn::kMaxThreads) continue;
+    if (max_groups * 32 > max_thr) continue;
     const int nthr = max_groups * 32 < 128 ? 128 : max_groups * 32;
     const int wpr = max_groups * bits;
     const int sw = ((n_in * wpr) + 3) & ~3;
-    const size_t smem = snn::present_smem_bytes(n_in, sw, h->L_pot, h->L_dep, h->q_max, nthr);
+    size_t smem;
+    int rows_cap = 0, offs_cap = 0, logn = 0;
+    if (ev) {
+      // on-chip window of active-row lists + LTD undo log
+      offs_cap = 1024;
+      logn = p->stdp_mode == SNN_STDP_STOCH ? 8 : 1;
+      rows_cap = std::max(n_in, 8192);
+      smem = snn::event_smem_bytes(n_in, sw, h->L_pot, h->L_dep, h->q_max, nthr, rows_cap, offs_cap, logn);
+      if (smem > (size_t)smem_optin) {         // shrink the row window down to one step's worth
+        rows_cap = n_in;
+        smem = snn::event_smem_bytes(n_in, sw, h->L_pot, h->L_dep, h->q_max, nthr, rows_cap, offs_cap, logn);
+      }
+    } else {
+      smem = snn::present_smem_bytes(n_in, sw, h->L_pot, h->L_dep, h->q_max, nthr);
+    }
     if (smem > (size_t)smem_optin) continue;
     h->cs = cs; h->nthr = nthr; h->wpr = wpr; h->slice_words = sw; h->smem = smem;
+    h->rows_cap = rows_cap; h->offs_cap = offs_cap; h->logn = logn;
     chosen = 1;
     break;
   }
@@ -392,7 +461,8 @@ int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** 
                 n_in, n_exc, bits, smem_optin);
   }
   int nclusters = 0;
-  ce = snn::query_max_clusters(h->cs, h->nthr, h->smem, &nclusters);
+  ce = ev ? snn::query_max_clusters_event(h->cs, h->nthr, h->smem, &nclusters)
+          : snn::query_max_clusters(h->cs, h->nthr, h->smem, &nclusters);
   if (ce != cudaSuccess || nclusters < 1) {
     cudaGetLastError();
     delete h;
@@ -525,10 +595,14 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
   for (int k = 0; k < n; ++k) {
     if (!hs[k]) return fail(SNN_EINVAL, "handle %d is NULL", k);
     if (hs[k]->n_in != hs[0]->n_in || hs[k]->cs != hs[0]->cs || hs[k]->nthr != hs[0]->nthr ||
-        hs[k]->dev != hs[0]->dev)
-      return fail(SNN_EINVAL, "ensemble handles must share n_in, cluster size, CTA shape and device");
+        hs[k]->dev != hs[0]->dev || hs[k]->engine != hs[0]->engine)
+      return fail(SNN_EINVAL, "ensemble handles must share n_in, cluster size, CTA shape, engine and device");
+    for (int m = 0; m < k; ++m)
+      if (hs[m] == hs[k]) return fail(SNN_EINVAL, "handle %d appears twice", k);
   }
-  if (n_images == 0 || T == 0) return SNN_OK;
+  const bool ev = hs[0]->engine == SNN_ENGINE_EVENT;
+  if (ev && T > snn::kEvMaxT) return fail(SNN_EINVAL, "T=%d exceeds %d for the event engine", T, snn::kEvMaxT);
+  if (n_images == 0) return SNN_OK;
   snn_handle* h0 = hs[0];
   DevGuard g(h0->dev);
   size_t smem = 0;
@@ -537,18 +611,23 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
   for (int k = 0; k < n; ++k) {
     snn_handle* h = hs[k];
     if (h != h0) CUDA_TRY(cudaStreamSynchronize(h->stream));
+    cudaStream_t own = h->stream;
+    h->stream = h0->stream;            // all pre-pass work is ordered on the launching stream
     NetDesc& d = descs[k];
     fill_static(h, d);
     d.n_images = n_images; d.T = T; d.flags = 0; d.t0 = 0;
     const uint8_t* img = nullptr;
-    int rc = stage(h0, images[k], (size_t)n_images * h->n_in, &h->d_img, &h->img_cap, &img);
-    if (rc) return rc;
     const unsigned long long* sd = nullptr;
-    rc = stage(h0, reinterpret_cast<const unsigned long long*>(seeds[k]), (size_t)n_images, &h->d_seeds, &h->seeds_cap, &sd);
+    int rc = stage(h, images[k], (size_t)n_images * h->n_in, &h->d_img, &h->img_cap, &img);
+    if (!rc) rc = stage(h, reinterpret_cast<const unsigned long long*>(seeds[k]), (size_t)n_images, &h->d_seeds,
+                        &h->seeds_cap, &sd);
+    if (!rc) rc = ensure(h, &h->d_raster, &h->raster_cap, (size_t)T * d.nwe);
+    if (!rc) {
+      d.images = img; d.seeds = sd; d.raster_out = h->d_raster;
+      if (ev) rc = event_prepass(h, d, img, nullptr, n_images, T, 0, sd);
+    }
+    h->stream = own;
     if (rc) return rc;
-    rc = ensure(h, &h->d_raster, &h->raster_cap, (size_t)T * d.nwe);
-    if (rc) return rc;
-    d.images = img; d.seeds = sd; d.raster_out = h->d_raster;
   }
   NetDesc* d_descs = nullptr;
   CUDA_TRY(cudaMalloc(&d_descs, sizeof(NetDesc) * n));
@@ -556,7 +635,8 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
   snn::LaunchParams lp;
   std::memset(&lp, 0, sizeof(lp));
   lp.descs = d_descs;
-  cudaError_t e = snn::launch_present(lp, n, h0->cs, h0->nthr, smem, h0->stream);
+  cudaError_t e = ev ? snn::launch_present_event(lp, n, h0->cs, h0->nthr, smem, h0->stream)
+                     : snn::launch_present(lp, n, h0->cs, h0->nthr, smem, h0->stream);
   if (e == cudaSuccess) e = cudaStreamSynchronize(h0->stream);
   cudaFree(d_descs);
   if (e != cudaSuccess) return fail(SNN_ECUDA, "present_many: %s", cudaGetErrorString(e));

@@ -52,6 +52,11 @@ struct NetDesc {
   uint32_t* in_raster_out;             // [T][nwi] input raster of the last image (may be null)
   int* spike_counts;                   // [n_images] (may be null)
   int n_images, T, flags, t0;
+  // event engine: per-image active-row lists from the encoder pre-pass
+  const uint32_t* ev_offs;             // [n_images][T+1] prefix offsets into ev_rows
+  const uint16_t* ev_rows;             // [n_images][rows_stride] active input rows, step-major, ascending
+  long long rows_stride;
+  int rows_cap, offs_cap, logn;        // on-chip window of the lists, per-thread LTD undo-log entries
 };
 
 struct LaunchParams {
@@ -61,6 +66,18 @@ struct LaunchParams {
 
 // kernels.cu entry points (host side)
 cudaError_t launch_present(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, cudaStream_t s);
+// event engine (snn_event.cu)
+constexpr int kEvMaxThreads = 512;
+constexpr int kEvMaxT = 32767;
+size_t event_smem_bytes(int n_in, int slice_words, int L_pot, int L_dep, int q_max, int nthr, int rows_cap,
+                        int offs_cap, int logn);
+cudaError_t query_max_clusters_event(int cs, int nthr, size_t smem, int* out);
+cudaError_t launch_encode(const uint8_t* images, const unsigned long long* thr_enc, const unsigned long long* seeds,
+                          int n_in, int T, int n_images, int t0, uint32_t* words, uint32_t* counts, cudaStream_t s);
+cudaError_t launch_counts_from_raster(const uint32_t* raster, int n_in, int T, uint32_t* counts, cudaStream_t s);
+cudaError_t launch_compact(const uint32_t* words, const uint32_t* counts, int n_in, int T, int n_images,
+                           long long rows_stride, uint32_t* offs, uint16_t* rows, cudaStream_t s);
+cudaError_t launch_present_event(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, cudaStream_t s);
 cudaError_t configure_present_kernel(size_t smem, int cs);
 cudaError_t query_max_clusters(int cs, int nthr, size_t smem, int* out);
 cudaError_t launch_init_weights(const NetDesc& d, uint64_t init_seed, cudaStream_t s);

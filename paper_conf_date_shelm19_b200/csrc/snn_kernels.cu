@@ -14,52 +14,10 @@
 //   (a5) LTP (or the deterministic arm, a6) on the winner's column, rows spread over threads
 // Citations: P:<line> of /root/reference/PAPER.md; readings R<n> of DESIGN.md §2.
 #include "snn_internal.h"
+#include "snn_device.cuh"
 #include <cstdint>
 
 namespace snn {
-
-// ------------------------------------------------------------------ Philox4x32-10 (R13), device copy
-__device__ __forceinline__ uint4 philox(uint32_t c0, uint32_t c1, uint32_t c2, uint32_t c3,
-                                        unsigned long long seed) {
-  uint32_t k0 = (uint32_t)seed, k1 = (uint32_t)(seed >> 32);
-#pragma unroll
-  for (int r = 0; r < 10; ++r) {
-    if (r) { k0 += 0x9E3779B9u; k1 += 0xBB67AE85u; }
-    const uint32_t lo0 = 0xD2511F53u * c0, hi0 = __umulhi(0xD2511F53u, c0);
-    const uint32_t lo1 = 0xCD9E8D57u * c2, hi1 = __umulhi(0xCD9E8D57u, c2);
-    const uint32_t n0 = hi1 ^ c1 ^ k0, n2 = hi0 ^ c3 ^ k1;
-    c0 = n0; c1 = lo1; c2 = n2; c3 = lo0;
-  }
-  return make_uint4(c0, c1, c2, c3);
-}
-
-__device__ __forceinline__ uint32_t pick(const uint4& u, int l) {
-  return l == 0 ? u.x : (l == 1 ? u.y : (l == 2 ? u.z : u.w));
-}
-
-// ------------------------------------------------------------------ cluster primitives
-__device__ __forceinline__ void cluster_arrive() {
-  asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
-}
-__device__ __forceinline__ void cluster_wait() {
-  asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
-}
-// store v into the same shared-memory variable of CTA `rank` of this cluster (DSMEM)
-__device__ __forceinline__ void st_cluster_u64(unsigned long long* local, uint32_t rank, unsigned long long v) {
-  const uint32_t a = (uint32_t)__cvta_generic_to_shared(local);
-  uint32_t ra;
-  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(a), "r"(rank));
-  asm volatile("st.shared::cluster.u64 [%0], %1;" ::"r"(ra), "l"(v) : "memory");
-}
-
-// order-preserving map of an fp32 bit pattern to u32 (for the WTA argmax key)
-__device__ __forceinline__ uint32_t float_ord(uint32_t u) {
-  return (u & 0x80000000u) ? ~u : (u | 0x80000000u);
-}
-
-constexpr unsigned FULL = 0xFFFFFFFFu;
-
-__host__ __device__ inline size_t align16(size_t x) { return (x + 15) & ~size_t(15); }
 
 struct SmemLayout {
   size_t enc, wkey, slots, w, pot, dep, dbp, dbd, dtp, dtd, lpre, spk, misc, alist, splist, img, total;

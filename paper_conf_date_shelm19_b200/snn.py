@@ -44,7 +44,7 @@ class SnnParams(ctypes.Structure):
         ("g_min", ctypes.c_double), ("g_max", ctypes.c_double),
         ("frac_bits", ctypes.c_int32), ("init_mode", ctypes.c_int32),
         ("init_seed", ctypes.c_uint64),
-        ("cluster_size", ctypes.c_int32), ("reserved0", ctypes.c_int32),
+        ("cluster_size", ctypes.c_int32), ("engine", ctypes.c_int32),
     ]
 
     def as_dict(self) -> dict:
@@ -116,10 +116,16 @@ def preset(name: str = "8b", **overrides) -> SnnParams:
     return p
 
 
-def params_from_dict(d: dict) -> SnnParams:
+def params_from_dict(d: dict, **overrides) -> SnnParams:
+    """Parameter block from a dict of DESIGN.md §3.1 fields (`engine` defaults to event-driven)."""
     p = SnnParams()
     for name, _ in SnnParams._fields_:
-        setattr(p, name, d[name])
+        if name == "engine":
+            p.engine = int(d.get("engine", 0))
+        else:
+            setattr(p, name, d[name])
+    for k, v in overrides.items():
+        setattr(p, k, v)
     return p
 
 

@@ -14,9 +14,12 @@ from oracle import oracle as O
 pytestmark = pytest.mark.gpu
 
 
-def _pair(n_in, n_exc, bits, p):
+ENGINES = [0, 1]   # SNN_ENGINE_EVENT (event-driven epochs), SNN_ENGINE_STEP (per-step exchange)
+
+
+def _pair(n_in, n_exc, bits, p, engine=0):
     import paper_conf_date_shelm19_b200 as P
-    g = P.Network(n_in, n_exc, bits, P.params_from_dict(p))
+    g = P.Network(n_in, n_exc, bits, P.params_from_dict(p, engine=engine))
     o = O.OracleNet(n_in, n_exc, bits, p)
     return g, o
 
@@ -65,7 +68,7 @@ def test_initial_weights_bit_exact(gpu, bits, n_exc, cs):
 
 def test_set_get_weights_roundtrip(gpu):
     import paper_conf_date_shelm19_b200 as P
-    g, _ = _pair(784, 1600, 4, O.params("4b", cluster_size=3))
+    g, _ = _pair(784, 1600, 4, O.params("4b", cluster_size=4))
     w = np.random.default_rng(0).integers(0, 16, size=(784, 1600)).astype(np.uint8)
     g.set_weights(w)
     assert np.array_equal(g.weights(), w)
@@ -75,20 +78,22 @@ def test_set_get_weights_roundtrip(gpu):
 
 # ------------------------------------------------------------------ C1: 784 -> 100, 8 bit, T = 100 (configs[0])
 @pytest.mark.parametrize("mode", [0, 1])
-def test_C1_784x100_8bit_20_images(gpu, mode):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_C1_784x100_8bit_20_images(gpu, engine, mode):
     p = O.params("8b", membrane_mode=mode, init_seed=1)
-    g, o = _pair(784, 100, 8, p)
+    g, o = _pair(784, 100, 8, p, engine=engine)
     imgs = synthdata.images(20, "mnist")
     seeds = synthdata.seeds(20, base_seed=1)
     _compare_presentations(g, o, imgs, 100, seeds, 784, 100, mode)
     assert o.stats()[1] > 0
 
 
-def test_C1_batch_launch_equals_per_image(gpu):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_C1_batch_launch_equals_per_image(gpu, engine):
     """snn_present_batch (one persistent launch, weights resident across images) == the oracle
     presenting the images one by one."""
     p = O.params("8b", membrane_mode=1, init_seed=1)
-    g, o = _pair(784, 100, 8, p)
+    g, o = _pair(784, 100, 8, p, engine=engine)
     imgs = synthdata.images(20, "mnist")
     seeds = synthdata.seeds(20, base_seed=1)
     counts = np.zeros(20, np.int32)
@@ -105,9 +110,10 @@ def test_C1_batch_launch_equals_per_image(gpu):
 
 # ------------------------------------------------------------------ C2: 784 -> 400 LAYER WTA, stochastic and deterministic arms
 @pytest.mark.parametrize("stdp,rounding", [(0, 1), (1, 0), (1, 1), (1, 2)])
-def test_C2_784x400_layer(gpu, stdp, rounding):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_C2_784x400_layer(gpu, engine, stdp, rounding):
     p = O.params("8b", wta_mode=1, stdp_mode=stdp, rounding=rounding, membrane_mode=1, init_seed=2)
-    g, o = _pair(784, 400, 8, p)
+    g, o = _pair(784, 400, 8, p, engine=engine)
     imgs = synthdata.images(3, "mnist", start=100)
     seeds = synthdata.seeds(3, base_seed=2)
     _compare_presentations(g, o, imgs, 350, seeds, 784, 400, 1)
@@ -115,51 +121,57 @@ def test_C2_784x400_layer(gpu, stdp, rounding):
 
 
 @pytest.mark.parametrize("mode", [0, 1])
-def test_C2_hard_det_fp32(gpu, mode):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_C2_hard_det_fp32(gpu, engine, mode):
     p = O.params("8b", stdp_mode=1, rounding=2, membrane_mode=mode, init_seed=3)
-    g, o = _pair(784, 400, 8, p)
+    g, o = _pair(784, 400, 8, p, engine=engine)
     _compare_presentations(g, o, synthdata.images(2, "mnist", start=7), 350, synthdata.seeds(2, 3), 784, 400, mode)
 
 
 # ------------------------------------------------------------------ C3: 784 -> 1600, 2 bit, rate sweep
 @pytest.mark.parametrize("fmin,fmax,T", [(1.0, 22.0, 350), (5.0, 78.0, 100), (5.0, 156.0, 100), (10.0, 312.0, 100)])
-def test_C3_784x1600_2bit_rate_sweep(gpu, fmin, fmax, T):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_C3_784x1600_2bit_rate_sweep(gpu, engine, fmin, fmax, T):
     p = O.params("2b", f_min_hz=fmin, f_max_hz=fmax, membrane_mode=1, init_seed=4)
-    g, o = _pair(784, 1600, 2, p)
+    g, o = _pair(784, 1600, 2, p, engine=engine)
     _compare_presentations(g, o, synthdata.images(2, "mnist", start=3), T, synthdata.seeds(2, 4), 784, 1600, 1)
 
 
 @pytest.mark.parametrize("cs", [1, 2, 3, 8, 16])
-def test_cluster_size_invariance(gpu, cs):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_cluster_size_invariance(gpu, engine, cs):
     """The same network sliced over 1..16 CTAs gives bit-identical results (global Philox indices)."""
     p = O.params("4b", membrane_mode=1, init_seed=5, cluster_size=cs)
-    g, o = _pair(784, 512, 4, p)        # 16 groups of 32 columns: 200 KB on one CTA, 1 group per CTA at 16
+    g, o = _pair(784, 512, 4, p, engine=engine)        # 16 groups of 32 columns: 200 KB on one CTA, 1 group per CTA at 16
     _compare_presentations(g, o, synthdata.images(2, "fashion"), 150, synthdata.seeds(2, 5), 784, 512, 1)
 
 
 # ------------------------------------------------------------------ C4: 784 -> 6400, 2 bit, fashion (the bench workload)
 @pytest.mark.parametrize("mode", [0, 1])
-def test_C4_784x6400_2bit_full_size(gpu, mode):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_C4_784x6400_2bit_full_size(gpu, engine, mode):
     p = O.params("2b", membrane_mode=mode, init_seed=1)
-    g, o = _pair(784, 6400, 2, p)
+    g, o = _pair(784, 6400, 2, p, engine=engine)
     _compare_presentations(g, o, synthdata.images(2, "fashion"), 350, synthdata.seeds(2, 1), 784, 6400, mode)
     assert o.stats()[1] > 0
 
 
-def test_C4_hf_variant(gpu):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_C4_hf_variant(gpu, engine):
     p = O.params("hf", membrane_mode=1, init_seed=1)
-    g, o = _pair(784, 6400, 2, p)
+    g, o = _pair(784, 6400, 2, p, engine=engine)
     _compare_presentations(g, o, synthdata.images(1, "fashion", start=5), 100, synthdata.seeds(1, 9), 784, 6400, 1)
 
 
 # ------------------------------------------------------------------ C5: ensemble, one launch
-def test_C5_ensemble_present_many(gpu):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_C5_ensemble_present_many(gpu, engine):
     import paper_conf_date_shelm19_b200 as P
     nets, oracles, imgs, seeds = [], [], [], []
     for k in range(6):
         bits = (2, 4, 8)[k % 3]
         p = O.params({2: "2b", 4: "4b", 8: "8b"}[bits], membrane_mode=1, init_seed=1 + k, cluster_size=2)
-        g, o = _pair(784, 400, bits, p)
+        g, o = _pair(784, 400, bits, p, engine=engine)
         nets.append(g)
         oracles.append(o)
         imgs.append(synthdata.images(3, "mnist", start=10 * k))
@@ -174,17 +186,19 @@ def test_C5_ensemble_present_many(gpu):
 
 # ------------------------------------------------------------------ edge cases
 @pytest.mark.parametrize("n_in,n_exc,bits", [(1, 1, 8), (33, 1, 2), (5, 65, 4), (784, 31, 2), (2000, 64, 8)])
-def test_ragged_shapes(gpu, n_in, n_exc, bits):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_ragged_shapes(gpu, engine, n_in, n_exc, bits):
     p = O.params("8b", membrane_mode=1, f_min_hz=20.0, f_max_hz=400.0, v_spike=30.0, init_seed=6)
-    g, o = _pair(n_in, n_exc, bits, p)
+    g, o = _pair(n_in, n_exc, bits, p, engine=engine)
     rng = np.random.default_rng(n_in * 7 + n_exc)
     imgs = rng.integers(0, 256, size=(2, n_in)).astype(np.uint8)
     _compare_presentations(g, o, imgs, 60, [3, 4], n_in, n_exc, 1)
 
 
-def test_zero_and_one_step(gpu):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_zero_and_one_step(gpu, engine):
     p = O.params("8b", membrane_mode=1)
-    g, o = _pair(784, 100, 8, p)
+    g, o = _pair(784, 100, 8, p, engine=engine)
     img = synthdata.images(1)[0]
     for T in (0, 1, 2):
         g.present(img, T, 5)
@@ -195,13 +209,14 @@ def test_zero_and_one_step(gpu):
 
 
 @pytest.mark.parametrize("mode", [0, 1])
-def test_stepwise_keep_state_and_reseed(gpu, mode):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_stepwise_keep_state_and_reseed(gpu, engine, mode):
     """North-star protocol: after each single step (SNN_KEEP_STATE, t0 = t) the GPU state equals the
     oracle's; in fp32 mode v agrees to 1e-5 relative per step; the GPU can be reseeded from the
     oracle state at any point and continue identically."""
     import paper_conf_date_shelm19_b200 as P
     p = O.params("8b", membrane_mode=mode, init_seed=8)
-    g, o = _pair(784, 64, 8, p)
+    g, o = _pair(784, 64, 8, p, engine=engine)
     img = synthdata.images(1, "mnist", start=4)[0]
     for t in range(80):
         fl = O.ORACLE_KEEP_STATE if t else 0
@@ -214,10 +229,11 @@ def test_stepwise_keep_state_and_reseed(gpu, mode):
             g.set_weights(o.weights())
 
 
-def test_raster_input_ltp_ltd_paths(gpu):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_raster_input_ltp_ltd_paths(gpu, engine):
     """Encoder bypass (SNN_RASTER_INPUT) with forced post spikes: LTP / LTD counters and codes equal."""
     p = O.params("8b", i_ext=60.0, v_spike=1e-9, t_ref_steps=7, membrane_mode=1)
-    g, o = _pair(784, 3, 8, p)
+    g, o = _pair(784, 3, 8, p, engine=engine)
     rng = np.random.default_rng(3)
     raster = rng.integers(0, 2 ** 32, size=(40, 25), dtype=np.uint64).astype(np.uint32)
     raster &= rng.integers(0, 2 ** 32, size=(40, 25), dtype=np.uint64).astype(np.uint32)
