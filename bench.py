@@ -149,6 +149,7 @@ def main():
     ap.add_argument("--membrane", type=int, default=0, help="0 fp32, 1 Q15.16")
     ap.add_argument("--cpu-images", type=int, default=10, help="oracle images for cpu_baseline (0 = skip)")
     ap.add_argument("--no-floor", action="store_true")
+    ap.add_argument("--engine", type=int, default=0, help="0 event-driven epochs, 1 per-step exchange")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -170,7 +171,8 @@ def main():
     torch.cuda.set_stream(stream)
 
     B = args.images_per_step
-    params = P.preset("2b", membrane_mode=args.membrane, init_seed=1 + rank, cluster_size=args.cluster_size)
+    params = P.preset("2b", membrane_mode=args.membrane, init_seed=1 + rank, cluster_size=args.cluster_size,
+                      engine=args.engine)
     net = P.Network(N_IN, N_EXC, BITS, params)
     net.set_stream(stream.cuda_stream)
     info = net.info()
@@ -230,7 +232,7 @@ def main():
 
     # ---- latency floor: same launch shape, barriers + exchange only (SNN_FLOOR_PROBE)
     floor = None
-    if not args.no_floor:
+    if not args.no_floor and args.engine == 1:
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
         step(args.warmup, flags=P.snn.SNN_FLOOR_PROBE)
@@ -245,7 +247,8 @@ def main():
     imgs_pin = torch.from_numpy(imgs_h).pin_memory()
     seeds_pin = torch.from_numpy(seeds_h.view(np.int64)).pin_memory()
     counts_pin = torch.zeros(pool_n, dtype=torch.int32).pin_memory()
-    net2_params = P.preset("2b", membrane_mode=args.membrane, init_seed=1 + rank, cluster_size=args.cluster_size)
+    net2_params = P.preset("2b", membrane_mode=args.membrane, init_seed=1 + rank, cluster_size=args.cluster_size,
+                      engine=args.engine)
     net2 = P.Network(N_IN, N_EXC, BITS, net2_params)
     net2.set_stream(stream.cuda_stream)
     for k in range(args.warmup):
@@ -298,7 +301,11 @@ def main():
                       "act_per_step": int(stats[0]) / (B * args.steps * T_STEPS),
                       "ltd_trials_per_image": int(stats[2]) / (B * args.steps),
                       "ltp_trials_per_image": int(stats[4]) / (B * args.steps),
-                      "step_ms_min": min(step_ms), "step_ms_max": max(step_ms)},
+                      "step_ms_min": min(step_ms), "step_ms_max": max(step_ms),
+                      "epochs_per_image": int(stats[8]) / (B * args.steps),
+                      "log_stops_per_image": int(stats[9]) / (B * args.steps),
+                      "resims_per_image": int(stats[10]) / (B * args.steps),
+                      "speculated_column_steps_ratio": int(stats[11]) / max(1, N_EXC * T_STEPS * B * args.steps)},
         "gpu_launches": launches,
         "clocks": clocks,
         "e2e": e2e,

@@ -152,12 +152,23 @@ int snn_get_state(snn_handle* h, void* buf, size_t cap);
 int snn_set_state(snn_handle* h, const void* buf, size_t n);
 /* Counters accumulated since the last snn_reset_stats: [0] sum_t act(t) (active input rows),
  * [1] post spikes, [2] LTD trials, [3] LTD events, [4] LTP trials, [5] LTP events,
- * [6] images presented, [7] steps simulated. */
-int snn_get_stats(snn_handle* h, uint64_t stats[8]);
+ * [6] images presented, [7] steps simulated; event engine only: [8] epochs
+ * (cluster exchanges), [9] speculation stops on a full undo log, [10] re-simulations,
+ * [11] speculated column-steps, [12] undone LTD events; [13..15] reserved (0). */
+#define SNN_NSTATS 16
+int snn_get_stats(snn_handle* h, uint64_t stats[SNN_NSTATS]);
 int snn_reset_stats(snn_handle* h);
 /* Introspection: [0] cluster size, [1] threads per CTA, [2] dynamic smem bytes per CTA,
  * [3] words per weight row in a CTA slice, [4] q_max, [5] L_pot, [6] L_dep, [7] kernel launches so far. */
 int snn_get_info(const snn_handle* h, int64_t info[8]);
+
+/* Tracing: with max_epochs > 0 the event engine records, per CTA and epoch,
+ * 8 u64 values: {image<<32 | k0, kind<<32 | P, t_spec_start, t_spec_end (max over warps),
+ * t_summary, t_exchanged, t_committed, t_end} (%globaltimer ns; kind 1 = post spike, 2 = no
+ * event / log stop, 0 = end of window).  snn_get_trace copies cluster_size x max_epochs x 8
+ * values of the last presentation call.  0 disables tracing. */
+int snn_set_trace(snn_handle* h, int max_epochs);
+int snn_get_trace(snn_handle* h, uint64_t* out, size_t cap);
 
 const char* snn_last_error(void);
 

@@ -101,6 +101,7 @@ struct snn_handle {
   uint32_t* d_ecnt = nullptr;    size_t ecnt_cap = 0;
   uint32_t* d_offs = nullptr;    size_t offs_buf_cap = 0;
   uint16_t* d_rows = nullptr;    size_t rows_buf_cap = 0;
+  unsigned long long* d_trace = nullptr; int trace_epochs = 0;
 };
 
 namespace {
@@ -164,13 +165,14 @@ void fill_static(const snn_handle* h, NetDesc& d) {
   d.v = h->d_v; d.cnt = h->d_cnt; d.last_post = h->d_lpost; d.last_pre = h->d_lpre;
   d.stats = h->d_stats;
   d.rows_cap = h->rows_cap; d.offs_cap = h->offs_cap; d.logn = h->logn;
+  d.trace = h->d_trace; d.trace_cap = h->trace_epochs;
 }
 
 void free_all(snn_handle* h) {
   void* ptrs[] = {h->d_w, h->d_enc, h->d_pot, h->d_dep, h->d_dbp, h->d_dbd, h->d_dtp, h->d_dtd,
                   h->d_v, h->d_cnt, h->d_lpost, h->d_lpre, h->d_stats, h->d_raster, h->d_inrec,
                   h->d_img, h->d_rin, h->d_seeds, h->d_counts, h->d_codes, h->d_bad,
-                  h->d_words, h->d_ecnt, h->d_offs, h->d_rows};
+                  h->d_words, h->d_ecnt, h->d_offs, h->d_rows, h->d_trace};
   for (void* q : ptrs) if (q) cudaFree(q);
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
 }
@@ -439,7 +441,7 @@ int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** 
     if (ev) {
       // on-chip window of active-row lists + LTD undo log
       offs_cap = 1024;
-      logn = p->stdp_mode == SNN_STDP_STOCH ? 8 : 1;
+      logn = p->stdp_mode == SNN_STDP_STOCH ? 16 : 1;
       rows_cap = std::max(n_in, 8192);
       smem = snn::event_smem_bytes(n_in, sw, h->L_pot, h->L_dep, h->q_max, nthr, rows_cap, offs_cap, logn);
       if (smem > (size_t)smem_optin) {         // shrink the row window down to one step's worth
@@ -491,7 +493,7 @@ int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** 
   ALLOC(h->d_cnt, (size_t)n_exc);
   ALLOC(h->d_lpost, (size_t)n_exc);
   ALLOC(h->d_lpre, (size_t)n_in);
-  ALLOC(h->d_stats, 8);
+  ALLOC(h->d_stats, SNN_NSTATS);
   ALLOC(h->d_codes, (size_t)n_in * n_exc);
   ALLOC(h->d_bad, 1);
 #undef ALLOC
@@ -520,7 +522,7 @@ int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** 
   if (e == cudaSuccess) e = cudaMemsetAsync(h->d_cnt, 0, (size_t)n_exc * 4, h->stream);
   if (e == cudaSuccess) e = up(h->d_lpost, m1.data(), (size_t)n_exc * 4);
   if (e == cudaSuccess) e = up(h->d_lpre, m1.data(), (size_t)n_in * 4);
-  if (e == cudaSuccess) e = cudaMemsetAsync(h->d_stats, 0, 8 * sizeof(unsigned long long), h->stream);
+  if (e == cudaSuccess) e = cudaMemsetAsync(h->d_stats, 0, SNN_NSTATS * sizeof(unsigned long long), h->stream);
   NetDesc d;
   fill_static(h, d);
   if (e == cudaSuccess) e = snn::launch_init_weights(d, p->init_seed, h->stream);   // R4
@@ -595,8 +597,9 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
   for (int k = 0; k < n; ++k) {
     if (!hs[k]) return fail(SNN_EINVAL, "handle %d is NULL", k);
     if (hs[k]->n_in != hs[0]->n_in || hs[k]->cs != hs[0]->cs || hs[k]->nthr != hs[0]->nthr ||
-        hs[k]->dev != hs[0]->dev || hs[k]->engine != hs[0]->engine)
-      return fail(SNN_EINVAL, "ensemble handles must share n_in, cluster size, CTA shape, engine and device");
+        hs[k]->dev != hs[0]->dev || hs[k]->engine != hs[0]->engine ||
+        hs[k]->p.membrane_mode != hs[0]->p.membrane_mode)
+      return fail(SNN_EINVAL, "ensemble handles must share n_in, cluster size, CTA shape, engine, membrane mode, device");
     for (int m = 0; m < k; ++m)
       if (hs[m] == hs[k]) return fail(SNN_EINVAL, "handle %d appears twice", k);
   }
@@ -635,7 +638,7 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
   snn::LaunchParams lp;
   std::memset(&lp, 0, sizeof(lp));
   lp.descs = d_descs;
-  cudaError_t e = ev ? snn::launch_present_event(lp, n, h0->cs, h0->nthr, smem, h0->stream)
+  cudaError_t e = ev ? snn::launch_present_event_mode(lp, n, h0->cs, h0->nthr, smem, h0->p.membrane_mode, h0->stream)
                      : snn::launch_present(lp, n, h0->cs, h0->nthr, smem, h0->stream);
   if (e == cudaSuccess) e = cudaStreamSynchronize(h0->stream);
   cudaFree(d_descs);
@@ -755,12 +758,12 @@ int snn_set_state(snn_handle* h, const void* buf, size_t n) {
   return SNN_OK;
 }
 
-int snn_get_stats(snn_handle* h, uint64_t stats[8]) {
+int snn_get_stats(snn_handle* h, uint64_t stats[SNN_NSTATS]) {
   int rc = check_handle(h);
   if (rc) return rc;
   if (!stats) return fail(SNN_EINVAL, "stats is NULL");
   DevGuard g(h->dev);
-  CUDA_TRY(cudaMemcpyAsync(stats, h->d_stats, 8 * sizeof(uint64_t), cudaMemcpyDeviceToHost, h->stream));
+  CUDA_TRY(cudaMemcpyAsync(stats, h->d_stats, SNN_NSTATS * sizeof(uint64_t), cudaMemcpyDeviceToHost, h->stream));
   CUDA_TRY(cudaStreamSynchronize(h->stream));
   return SNN_OK;
 }
@@ -769,7 +772,37 @@ int snn_reset_stats(snn_handle* h) {
   int rc = check_handle(h);
   if (rc) return rc;
   DevGuard g(h->dev);
-  CUDA_TRY(cudaMemsetAsync(h->d_stats, 0, 8 * sizeof(unsigned long long), h->stream));
+  CUDA_TRY(cudaMemsetAsync(h->d_stats, 0, SNN_NSTATS * sizeof(unsigned long long), h->stream));
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  return SNN_OK;
+}
+
+int snn_set_trace(snn_handle* h, int max_epochs) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  if (max_epochs < 0) return fail(SNN_EINVAL, "max_epochs < 0");
+  DevGuard g(h->dev);
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  if (h->d_trace) cudaFree(h->d_trace);
+  h->d_trace = nullptr;
+  h->trace_epochs = 0;
+  if (max_epochs > 0) {
+    const size_t n = (size_t)h->cs * max_epochs * 8;
+    CUDA_TRY(dalloc(&h->d_trace, n));
+    CUDA_TRY(cudaMemset(h->d_trace, 0, n * sizeof(unsigned long long)));
+    h->trace_epochs = max_epochs;
+  }
+  return SNN_OK;
+}
+
+int snn_get_trace(snn_handle* h, uint64_t* out, size_t cap) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  const size_t n = (size_t)h->cs * h->trace_epochs * 8;
+  if (!h->d_trace) return fail(SNN_EINVAL, "tracing is off (snn_set_trace)");
+  if (!out || cap < n) return fail(SNN_ESIZE, "need %zu values", n);
+  DevGuard g(h->dev);
+  CUDA_TRY(cudaMemcpyAsync(out, h->d_trace, n * sizeof(uint64_t), cudaMemcpyDeviceToHost, h->stream));
   CUDA_TRY(cudaStreamSynchronize(h->stream));
   return SNN_OK;
 }

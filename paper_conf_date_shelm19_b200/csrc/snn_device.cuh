@@ -50,10 +50,22 @@ __device__ __forceinline__ void st_cluster_u64(unsigned long long* local, uint32
 __device__ __forceinline__ void red_min_cluster(int* local, uint32_t rank, int v) {
   asm volatile("red.relaxed.cluster.shared::cluster.min.s32 [%0], %1;" ::"r"(map_cluster(local, rank)), "r"(v) : "memory");
 }
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ int ld_volatile_shared_u32addr(uint32_t a) {
+  int v;
+  asm volatile("ld.volatile.shared.s32 %0, [%1];" : "=r"(v) : "r"(a));
+  return v;
+}
 __device__ __forceinline__ int ld_volatile_shared(const int* p) {
   int v;
   asm volatile("ld.volatile.shared.s32 %0, [%1];" : "=r"(v) : "r"((uint32_t)__cvta_generic_to_shared(p)));
   return v;
+}
+
+__device__ __forceinline__ unsigned long long globaltimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
 }
 
 // order-preserving map of an fp32 bit pattern to u32 (WTA argmax key)
@@ -88,6 +100,25 @@ struct Lif {
     const float vn = __fmaf_rn(dtf, dv, vf);
     v = __float_as_int(vn);
     return vn > vthf;
+  }
+  template <bool FIXED>
+  __device__ __forceinline__ bool step_t(int& v, int S) const {
+    if constexpr (FIXED) {
+      const long long x = v;
+      const long long bv = (B * x + (1LL << 31)) >> 32;
+      const long long cterm = (C * (long long)S + (1LL << 15)) >> 16;
+      v = (int)(x + A + bv + cterm + E);
+      return v > Vth;
+    } else {
+      const float vf = __int_as_float(v);
+      const float I = __fmul_rn(__int2float_rn(S), kI);
+      const float xx = __fadd_rn(I, ief);
+      const float y = __fmaf_rn(cf, xx, af);
+      const float dv = __fmaf_rn(bf, vf, y);
+      const float vn = __fmaf_rn(dtf, dv, vf);
+      v = __float_as_int(vn);
+      return vn > vthf;
+    }
   }
   __device__ __forceinline__ uint32_t ord(int v) const {
     return fixed ? ((uint32_t)v ^ 0x80000000u) : float_ord((uint32_t)v);

@@ -150,6 +150,34 @@ __global__ void __launch_bounds__(256) compact_kernel(const uint32_t* __restrict
 }
 
 // ====================================================================== main kernel
+
+// S_j over the active rows [r0, r1) of one step: independent loads, unrolled for ILP (eq.(3))
+__device__ __forceinline__ int integrate(const uint32_t* __restrict__ wcol, const uint16_t* __restrict__ rows, int r0,
+                                        int r1, int wpr, int sh, uint32_t fmask) {
+  int S = 0;
+  int r = r0;
+  for (; r + 4 <= r1; r += 4) {
+    const int i0 = rows[r], i1 = rows[r + 1], i2 = rows[r + 2], i3 = rows[r + 3];
+    const uint32_t w0 = wcol[i0 * wpr], w1 = wcol[i1 * wpr], w2 = wcol[i2 * wpr], w3 = wcol[i3 * wpr];
+    S += (int)(((w0 >> sh) & fmask) + ((w1 >> sh) & fmask) + ((w2 >> sh) & fmask) + ((w3 >> sh) & fmask));
+  }
+  for (; r < r1; ++r) S += (int)((wcol[(int)rows[r] * wpr] >> sh) & fmask);
+  return S;
+}
+
+// LTD draws of column j against rows [r0, r0 + n), n <= 32: bit m set iff u_LTD(t, rows[r0+m], j) <= thr.
+// Branch-free so that the independent Philox blocks overlap (eq.(7), R13).
+__device__ __forceinline__ uint32_t ltd_draws(const uint16_t* __restrict__ rows, int r0, int n, uint32_t t, int j,
+                                              uint32_t thr, unsigned long long seed) {
+  uint32_t m = 0;
+  const int lanej = j & 3;
+#pragma unroll 4
+  for (int x = 0; x < n; ++x) {
+    const uint4 u = philox(t, (uint32_t)rows[r0 + x], (uint32_t)(j >> 2), TAG_LTD, seed);
+    m |= (pick(u, lanej) <= thr ? 1u : 0u) << x;
+  }
+  return m;
+}
 struct EvLayout {
   size_t slots, wsum, flags, misc, w, pot, dep, dbp, dbd, dtp, dtd, lpre, offs, rows, log, splist, total;
 };
@@ -161,7 +189,7 @@ __host__ __device__ inline EvLayout ev_layout(int n_in, int slice_words, int L_p
   L.slots = o;  o = align16(o + 2 * kMaxCluster * 2 * 8);   // [parity][rank][2] u64
   L.wsum = o;   o = align16(o + 32 * 2 * 8);                // per warp: summary, key
   L.flags = o;  o = align16(o + 4 * 4);                     // early-stop flag per epoch parity
-  L.misc = o;   o = align16(o + 16 * 4);
+  L.misc = o;   o = align16(o + 16 * 8);
   L.w = o;      o = align16(o + (size_t)slice_words * 4);
   L.pot = o;    o = align16(o + (size_t)(L_pot > 0 ? L_pot : 1) * 4);
   L.dep = o;    o = align16(o + (size_t)(L_dep > 0 ? L_dep : 1) * 4);
@@ -183,6 +211,7 @@ size_t event_smem_bytes(int n_in, int slice_words, int L_pot, int L_dep, int q_m
   return ev_layout(n_in, slice_words, L_pot, L_dep, q_max, nthr, rows_cap, offs_cap, logn).total;
 }
 
+template <bool FIXED>
 __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const __grid_constant__ LaunchParams lp) {
   extern __shared__ __align__(16) unsigned char smem[];
   const NetDesc& d0 = lp.descs ? lp.descs[0] : lp.single;
@@ -258,12 +287,16 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
     if (mycol) { v = d.v[j]; cnt = d.cnt[j]; lpost = d.last_post[j]; }
     for (int i = tid; i < n_in; i += nthr) s_lpre[i] = d.last_pre[i];
   }
-  unsigned long long ltd_trials = 0, ltd_events = 0, ltp_trials = 0, ltp_events = 0;
+  uint32_t ltd_trials = 0, ltd_events = 0, ltp_trials = 0, ltp_events = 0;   // per launch, < 2^32
   unsigned long long act_sum = 0, post_sum = 0;
+  uint32_t eng_epochs = 0, eng_hz = 0, eng_resim = 0, eng_spec = 0, eng_undo = 0;
   // every CTA of the cluster has initialised its flags before any remote red.min can target them
   if (cs > 1) { cluster_arrive(); cluster_wait(); } else { __syncthreads(); }
 
   int ep = 0;
+  unsigned long long* trace = d.trace ? d.trace + (size_t)rank * d.trace_cap * 8 : nullptr;
+  unsigned long long* s_tmax = reinterpret_cast<unsigned long long*>(s_misc + 8);   // max speculation end
+  unsigned long long tr0 = 0, tr2 = 0, tr3 = 0;
   for (int b = 0; b < n_images; ++b) {
     const unsigned long long seed = d.seeds[b];
     if (!keep) {
@@ -302,6 +335,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
       }
       const int kend = kb;
       const int fp = ep & 1;
+      if (trace && tid == 0) { tr0 = globaltimer(); *s_tmax = 0ull; }
 
       // ---------------------------------------------------------- speculation (column-local, no barriers)
       int p = kend;            // first step not fully processed by this thread
@@ -310,49 +344,105 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
       const int v0 = v, cnt0 = cnt;
       int v1 = v, cnt1 = cnt, vb = v;
       int nlog = 0;
-      if (mycol) {
+      {
+        // Warp-synchronous speculation: every lane of the warp walks the same step kk (lanes that
+        // stopped are predicated off), so the LTD Philox blocks of an LTD-active column can be
+        // spread over all 32 lanes (one block per row) instead of serialised in one lane.
+        const uint32_t flag_addr = smem_u32(&s_flag[fp]);
+        const bool ltd_col = mycol && stoch && lpost >= 0;
+        const int jw = col0 + warp * 32;                          // column of lane 0 of this warp
+        bool done = !mycol;
         int kk = k0;
-        for (; kk < kend; ++kk) {
-          if (kk > ld_volatile_shared(&s_flag[fp])) break;        // a crossing before kk exists in the cluster
-          const int r0 = (int)(s_offs[kk - ka] - wbase), r1 = (int)(s_offs[kk - ka + 1] - wbase);
-          const int t = tbase + kk;
-          const bool ltd_on = stoch && lpost >= 0 && (t - lpost) < L_dep;
-          if (ltd_on && kk > k0 && nlog + (r1 - r0) > logn) { hz = true; break; }
-          int S = 0;                                               // (a2) eq.(3)
-          for (int r = r0; r < r1; ++r) S += (int)((wcol[(int)s_rows[r] * wpr] >> sh) & fmask);
-          if (cnt > 0) {
-            --cnt;                                                 // (a3) refractory / inhibited: hold v
-          } else {
-            vb = v;
-            if (lif.step(v, S)) { cand = true; break; }            // (a3) eqs.(1)(2)
-          }
-          if (ltd_on) {                                            // (a5) LTD, eq.(7), exact (R10, R14)
-            const uint32_t thr = s_dep[t - lpost];
-            for (int r = r0; r < r1; ++r) {
-              const int i = s_rows[r];
-              const uint4 u = philox((uint32_t)t, (uint32_t)i, (uint32_t)(j >> 2), TAG_LTD, seed);
-              if (pick(u, j & 3) <= thr) {
-                uint32_t* pw = wcol + i * wpr;
-                const bool applied = ((*pw >> sh) & fmask) != 0u;
-                if (applied) atomicSub(pw, 1u << sh);
-                ++ltd_events;
-                if (kk > k0)
-                  s_log[nlog++ * nthr + tid] = ((uint32_t)(kk - k0) << 16) | (applied ? 0x8000u : 0u) | (uint32_t)i;
-              }
-            }
-            ltd_trials += (unsigned long long)(r1 - r0);
-          }
-          if (kk == k0) { v1 = v; cnt1 = cnt; }
-        }
-        p = kk;
-        if (cand || hz) {
-          const int f = cand ? kk : kk - 1;                         // tell the cluster where to stop
+        int r0 = (int)(s_offs[k0 - ka] - wbase);
+        auto signal = [&](int f) {                                // tell the cluster where to stop
           atomicMin(&s_flag[fp], f);
           for (int r = 0; r < cs; ++r)
             if (r != rank) red_min_cluster(&s_flag[fp], (uint32_t)r, f);
+        };
+        while (__any_sync(FULL, !done)) {
+          if (!done && (kk >= kend || kk > ld_volatile_shared_u32addr(flag_addr))) { done = true; p = kk; }
+          if (kk >= kend) break;                                  // warp-uniform
+          const int r1 = (int)(s_offs[kk - ka + 1] - wbase);
+          const int t = tbase + kk;
+          bool ltd_on = false;
+          int cb = cnt;
+          if (!done) {
+            const int S = integrate(wcol, s_rows, r0, r1, wpr, sh, fmask);   // (a2) eq.(3)
+            if (cnt > 0) {
+              --cnt;                                               // (a3) refractory / inhibited: hold v
+            } else {
+              vb = v;
+              if (lif.step_t<FIXED>(v, S)) { cand = true; done = true; p = kk; signal(kk); }   // (a3) eqs.(1)(2)
+            }
+            ltd_on = !done && ltd_col && (t - lpost) < L_dep;
+          }
+          // (a5) LTD, eq.(7), exact (R10, R14): cooperative draws, then this lane's events
+          const uint32_t lmask = __ballot_sync(FULL, ltd_on);
+          if (lmask) {
+            const uint32_t thr = ltd_on ? s_dep[t - lpost] : 0u;
+            const int nlog_step = nlog;
+            bool overflow = false;
+            uint32_t ev_step = 0;
+            for (int c0 = r0; c0 < r1; c0 += 32) {               // warp-uniform chunks of <= 32 rows
+              const int n = min(32, r1 - c0);
+              const uint32_t row_here = lane < n ? (uint32_t)s_rows[c0 + lane] : 0u;
+              uint32_t mine = 0;
+              for (uint32_t lm = lmask; lm; lm &= lm - 1) {
+                const int L = __ffs(lm) - 1;
+                const int jL = jw + L;
+                const uint32_t thrL = __shfl_sync(FULL, thr, L);
+                bool bit = false;
+                if (lane < n) {
+                  const uint4 u = philox((uint32_t)t, row_here, (uint32_t)(jL >> 2), TAG_LTD, seed);
+                  bit = pick(u, jL & 3) <= thrL;
+                }
+                const uint32_t m = __ballot_sync(FULL, bit);
+                if (lane == L) mine = m;
+              }
+              if (ltd_on && !overflow) {
+                while (mine) {
+                  const int x = __ffs(mine) - 1;
+                  mine &= mine - 1;
+                  if (kk > k0 && nlog == logn) { overflow = true; break; }
+                  const int i = s_rows[c0 + x];
+                  uint32_t* pw = wcol + i * wpr;
+                  const bool applied = ((*pw >> sh) & fmask) != 0u;
+                  if (applied) atomicSub(pw, 1u << sh);
+                  ++ev_step;
+                  if (kk > k0)
+                    s_log[nlog++ * nthr + tid] = ((uint32_t)(kk - k0) << 16) | (applied ? 0x8000u : 0u) | (uint32_t)i;
+                }
+              }
+            }
+            if (ltd_on) {
+              if (overflow) {                                      // undo this step entirely; stop before it
+                while (nlog > nlog_step) {
+                  const uint32_t e = s_log[(nlog - 1) * nthr + tid];
+                  if (e & 0x8000u) atomicAdd(wcol + (int)(e & 0x7FFFu) * wpr, 1u << sh);
+                  --nlog;
+                }
+                cnt = cb;
+                if (cb == 0) v = vb;
+                hz = true;
+                done = true;
+                p = kk;
+                ++eng_hz;
+                signal(kk - 1);
+              } else {
+                ltd_events += ev_step;
+                ltd_trials += (uint32_t)(r1 - r0);
+              }
+            }
+          }
+          if (!done && kk == k0) { v1 = v; cnt1 = cnt; }
+          ++kk;
+          r0 = r1;
         }
+        if (!mycol) p = kend;
+        if (mycol) eng_spec += (uint32_t)(p - k0 + (cand ? 1 : 0));
       }
 
+      if (trace && lane == 0) atomicMax(s_tmax, globaltimer());
       // ---------------------------------------------------------- CTA summary -> cluster exchange
       {
         const uint32_t w1 = ((uint32_t)(0xFFFF - min(p, kend)) << 1) | (hz ? 1u : 0u);
@@ -369,6 +459,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         }
       }
       __syncthreads();                                                               // S1
+      if (trace && tid == 0) tr2 = globaltimer();
       if (warp == 0) {
         const unsigned long long a = lane < nwarps ? s_wsum[2 * lane] : 0ull;
         const unsigned long long k = lane < nwarps ? s_wsum[2 * lane + 1] : 0ull;
@@ -389,6 +480,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         if (lane == 0) { s_flag[fp ^ 1] = INT_MAX; s_misc[1] = 0; }
       }
       if (cs > 1) { cluster_arrive(); cluster_wait(); } else { __syncthreads(); }   // the one cross-SM exchange
+      if (trace && tid == 0) tr3 = globaltimer();
 
       // ---------------------------------------------------------- global decision
       uint32_t W1 = 0, count = 0;
@@ -410,11 +502,11 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
 
       // ---------------------------------------------------------- per-thread resolution / rollback
       // resim(X): state after step k0 + undo of every logged LTD, then replay k0+1..X exactly.
-      auto count_trials = [&](int from, int to) -> unsigned long long {   // LTD trials of steps [from, to)
-        unsigned long long n = 0;
+      auto count_trials = [&](int from, int to) -> uint32_t {   // LTD trials of steps [from, to)
+        uint32_t n = 0;
         if (stoch && lpost >= 0)
           for (int kk = from; kk < to; ++kk)
-            if ((tbase + kk - lpost) < L_dep) n += (unsigned long long)(s_offs[kk - ka + 1] - s_offs[kk - ka]);
+            if ((tbase + kk - lpost) < L_dep) n += s_offs[kk - ka + 1] - s_offs[kk - ka];
         return n;
       };
       auto undo_after = [&](int rel_keep) {       // undo logged LTD of steps k0+rel > k0+rel_keep
@@ -424,30 +516,32 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
           if (e & 0x8000u) atomicAdd(wcol + (int)(e & 0x7FFFu) * wpr, 1u << sh);
           --ltd_events;
           --nlog;
+          ++eng_undo;
         }
       };
       auto resim = [&](int X) {
+        ++eng_resim;
         undo_after(0);
         ltd_trials -= count_trials(k0 + 1, p);
         v = v1; cnt = cnt1;
         for (int kk = k0 + 1; kk <= X; ++kk) {
           const int r0 = (int)(s_offs[kk - ka] - wbase), r1 = (int)(s_offs[kk - ka + 1] - wbase);
           const int t = tbase + kk;
-          int S = 0;
-          for (int r = r0; r < r1; ++r) S += (int)((wcol[(int)s_rows[r] * wpr] >> sh) & fmask);
-          if (cnt > 0) --cnt; else lif.step(v, S);
+          const int S = integrate(wcol, s_rows, r0, r1, wpr, sh, fmask);
+          if (cnt > 0) --cnt; else lif.step_t<FIXED>(v, S);
           if (stoch && lpost >= 0 && (t - lpost) < L_dep) {
             const uint32_t thr = s_dep[t - lpost];
-            for (int r = r0; r < r1; ++r) {
-              const int i = s_rows[r];
-              const uint4 u = philox((uint32_t)t, (uint32_t)i, (uint32_t)(j >> 2), TAG_LTD, seed);
-              if (pick(u, j & 3) <= thr) {
-                uint32_t* pw = wcol + i * wpr;
+            for (int c0 = r0; c0 < r1; c0 += 32) {
+              uint32_t m = ltd_draws(s_rows, c0, min(32, r1 - c0), (uint32_t)t, j, thr, seed);
+              while (m) {
+                const int x = __ffs(m) - 1;
+                m &= m - 1;
+                uint32_t* pw = wcol + (int)s_rows[c0 + x] * wpr;
                 if ((*pw >> sh) & fmask) atomicSub(pw, 1u << sh);
                 ++ltd_events;
               }
             }
-            ltd_trials += (unsigned long long)(r1 - r0);
+            ltd_trials += (uint32_t)(r1 - r0);
           }
         }
       };
@@ -493,16 +587,17 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         if (mycol && cand && p == P && stoch && lpost >= 0 && (tP - lpost) < L_dep) {
           const int r0 = (int)(s_offs[P - ka] - wbase), r1 = (int)(s_offs[P - ka + 1] - wbase);
           const uint32_t thr = s_dep[tP - lpost];
-          for (int r = r0; r < r1; ++r) {
-            const int i = s_rows[r];
-            const uint4 u = philox((uint32_t)tP, (uint32_t)i, (uint32_t)(j >> 2), TAG_LTD, seed);
-            if (pick(u, j & 3) <= thr) {
-              uint32_t* pw = wcol + i * wpr;
+          for (int c0 = r0; c0 < r1; c0 += 32) {
+            uint32_t m = ltd_draws(s_rows, c0, min(32, r1 - c0), (uint32_t)tP, j, thr, seed);
+            while (m) {
+              const int x = __ffs(m) - 1;
+              m &= m - 1;
+              uint32_t* pw = wcol + (int)s_rows[c0 + x] * wpr;
               if ((*pw >> sh) & fmask) atomicSub(pw, 1u << sh);
               ++ltd_events;
             }
           }
-          ltd_trials += (unsigned long long)(r1 - r0);
+          ltd_trials += (uint32_t)(r1 - r0);
         }
         if (rec_out) {
           const uint32_t bal = __ballot_sync(FULL, spiked);
@@ -519,6 +614,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
       }
       const bool local_spike = event && (hard ? (W >= (uint32_t)col0 && W < (uint32_t)(col0 + ncols)) : false);
       __syncthreads();                                                               // S3
+      if (trace && tid == 0 && ep < d.trace_cap) trace[(size_t)ep * 8 + 6] = globaltimer();
       const int nsp = hard ? (local_spike ? 1 : 0) : (event ? s_misc[1] : 0);
       if (nsp > 0) {
         // (a5) LTP eq.(6) / (a6) deterministic arm at t*, rows spread over threads (row words owned)
@@ -563,8 +659,15 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         __syncthreads();                                                             // S4
       }
       if (spiked) lpost = tP;
+      if (trace && tid == 0 && ep < d.trace_cap) {
+        unsigned long long* rec = trace + (size_t)ep * 8;
+        rec[0] = ((unsigned long long)b << 32) | (unsigned)k0;
+        rec[1] = ((unsigned long long)(event ? 1 : (unknown ? 2 : 0)) << 32) | (unsigned)P;
+        rec[2] = tr0; rec[3] = *s_tmax; rec[4] = tr2; rec[5] = tr3; rec[7] = globaltimer();
+      }
       k0 = k_last + 1;
       ++ep;
+      ++eng_epochs;
     }  // epochs
 
     if (rank == 0 && tid == 0) {
@@ -584,7 +687,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
     for (int k = tid; k < slice_words / 4; k += nthr) dst[k] = src[k];
   }
   {
-    unsigned long long a = ltd_trials, b2 = ltd_events, c = ltp_trials, e = ltp_events;
+    unsigned long long a = ltd_trials, b2 = ltd_events, c = ltp_trials, e = ltp_events;  // widen before the warp sum
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
       a += __shfl_xor_sync(FULL, a, o); b2 += __shfl_xor_sync(FULL, b2, o);
@@ -601,6 +704,19 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
       atomicAdd(&d.stats[1], post_sum);
       atomicAdd(&d.stats[6], (unsigned long long)n_images);
       atomicAdd(&d.stats[7], (unsigned long long)n_images * (unsigned long long)T);
+      atomicAdd(&d.stats[8], (unsigned long long)eng_epochs);
+    }
+    unsigned long long h2 = eng_hz, r2 = eng_resim, s2 = eng_spec, u2 = eng_undo;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      h2 += __shfl_xor_sync(FULL, h2, o); r2 += __shfl_xor_sync(FULL, r2, o);
+      s2 += __shfl_xor_sync(FULL, s2, o); u2 += __shfl_xor_sync(FULL, u2, o);
+    }
+    if (lane == 0) {
+      if (h2) atomicAdd(&d.stats[9], h2);
+      if (r2) atomicAdd(&d.stats[10], r2);
+      if (s2) atomicAdd(&d.stats[11], s2);
+      if (u2) atomicAdd(&d.stats[12], u2);
     }
   }
   if (cs > 1) { cluster_arrive(); cluster_wait(); }
@@ -630,10 +746,11 @@ cudaError_t launch_compact(const uint32_t* words, const uint32_t* counts, int n_
   return cudaGetLastError();
 }
 
+template <bool FIXED>
 static cudaError_t configure_event(size_t smem, int cs) {
-  cudaError_t e = cudaFuncSetAttribute(present_event_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaError_t e = cudaFuncSetAttribute(present_event_kernel<FIXED>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  if (cs > 8) e = cudaFuncSetAttribute(present_event_kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+  if (cs > 8) e = cudaFuncSetAttribute(present_event_kernel<FIXED>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
   return e;
 }
 
@@ -656,22 +773,36 @@ static void fill_cfg_ev(cudaLaunchConfig_t& cfg, cudaLaunchAttribute* attr, int 
 }
 
 cudaError_t query_max_clusters_event(int cs, int nthr, size_t smem, int* out) {
-  cudaError_t e = configure_event(smem, cs);
+  cudaError_t e = configure_event<false>(smem, cs);
+  if (e == cudaSuccess) e = configure_event<true>(smem, cs);
   if (e != cudaSuccess) return e;
-  if (cs == 1) return cudaOccupancyMaxActiveBlocksPerMultiprocessor(out, present_event_kernel, nthr, smem);
+  if (cs == 1) return cudaOccupancyMaxActiveBlocksPerMultiprocessor(out, present_event_kernel<false>, nthr, smem);
   cudaLaunchConfig_t cfg;
   cudaLaunchAttribute attr[1];
   fill_cfg_ev(cfg, attr, 1, cs, nthr, smem, 0);
-  return cudaOccupancyMaxActiveClusters(out, present_event_kernel, &cfg);
+  return cudaOccupancyMaxActiveClusters(out, present_event_kernel<false>, &cfg);
 }
 
 cudaError_t launch_present_event(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, cudaStream_t s) {
-  cudaError_t e = configure_event(smem, cs);
+  const bool fixed = (lp.descs ? 0 : lp.single.membrane_mode) == 1;   // ensembles: see launch_present_event_mode
+  cudaError_t e = fixed ? configure_event<true>(smem, cs) : configure_event<false>(smem, cs);
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg;
   cudaLaunchAttribute attr[1];
   fill_cfg_ev(cfg, attr, n_nets, cs, nthr, smem, s);
-  return cudaLaunchKernelEx(&cfg, present_event_kernel, lp);
+  return fixed ? cudaLaunchKernelEx(&cfg, present_event_kernel<true>, lp)
+               : cudaLaunchKernelEx(&cfg, present_event_kernel<false>, lp);
+}
+
+cudaError_t launch_present_event_mode(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, int fixed,
+                                      cudaStream_t s) {
+  cudaError_t e = fixed ? configure_event<true>(smem, cs) : configure_event<false>(smem, cs);
+  if (e != cudaSuccess) return e;
+  cudaLaunchConfig_t cfg;
+  cudaLaunchAttribute attr[1];
+  fill_cfg_ev(cfg, attr, n_nets, cs, nthr, smem, s);
+  return fixed ? cudaLaunchKernelEx(&cfg, present_event_kernel<true>, lp)
+               : cudaLaunchKernelEx(&cfg, present_event_kernel<false>, lp);
 }
 
 }  // namespace snn

@@ -57,6 +57,9 @@ struct NetDesc {
   const uint16_t* ev_rows;             // [n_images][rows_stride] active input rows, step-major, ascending
   long long rows_stride;
   int rows_cap, offs_cap, logn;        // on-chip window of the lists, per-thread LTD undo-log entries
+  // optional per-epoch trace: [cs][trace_cap][8] u64 (%globaltimer ns)
+  unsigned long long* trace;
+  int trace_cap;
 };
 
 struct LaunchParams {
@@ -78,6 +81,8 @@ cudaError_t launch_counts_from_raster(const uint32_t* raster, int n_in, int T, u
 cudaError_t launch_compact(const uint32_t* words, const uint32_t* counts, int n_in, int T, int n_images,
                            long long rows_stride, uint32_t* offs, uint16_t* rows, cudaStream_t s);
 cudaError_t launch_present_event(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, cudaStream_t s);
+cudaError_t launch_present_event_mode(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, int fixed,
+                                      cudaStream_t s);
 cudaError_t configure_present_kernel(size_t smem, int cs);
 cudaError_t query_max_clusters(int cs, int nthr, size_t smem, int* out);
 cudaError_t launch_init_weights(const NetDesc& d, uint64_t init_seed, cudaStream_t s);

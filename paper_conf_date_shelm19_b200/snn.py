@@ -22,7 +22,7 @@ EXPORTS = [
     "snn_present", "snn_present_batch", "snn_present_ex", "snn_present_raster", "snn_present_many",
     "snn_get_weights", "snn_set_weights", "snn_get_spikes", "snn_get_input_raster",
     "snn_state_bytes", "snn_get_state", "snn_set_state", "snn_get_stats", "snn_reset_stats",
-    "snn_get_info", "snn_last_error",
+    "snn_get_info", "snn_set_trace", "snn_get_trace", "snn_last_error",
 ]
 
 
@@ -84,6 +84,8 @@ def lib():
             "snn_get_stats": ([vp, vp], i32),
             "snn_reset_stats": ([vp], i32),
             "snn_get_info": ([vp, vp], i32),
+            "snn_set_trace": ([vp, i32], i32),
+            "snn_get_trace": ([vp, vp, sz], i32),
             "snn_last_error": ([], ctypes.c_char_p),
         }
         for name, (args, res) in sig.items():
@@ -231,8 +233,19 @@ class Network:
         _check(lib().snn_set_state(self._h, _ptr(b), b.nbytes), "snn_set_state")
 
     def stats(self) -> np.ndarray:
-        out = np.zeros(8, dtype=np.uint64)
+        out = np.zeros(16, dtype=np.uint64)
         _check(lib().snn_get_stats(self._h, _ptr(out)), "snn_get_stats")
+        return out
+
+    def set_trace(self, max_epochs: int):
+        _check(lib().snn_set_trace(self._h, max_epochs), "snn_set_trace")
+        self._trace_epochs = max_epochs
+
+    def trace(self) -> np.ndarray:
+        """(cluster_size, max_epochs, 8) u64 per-epoch records (include/snn.h snn_set_trace)."""
+        cs = self.info()["cluster_size"]
+        out = np.zeros((cs, self._trace_epochs, 8), dtype=np.uint64)
+        _check(lib().snn_get_trace(self._h, _ptr(out), out.size), "snn_get_trace")
         return out
 
     def reset_stats(self):

@@ -141,8 +141,8 @@ def test_C3_784x1600_2bit_rate_sweep(gpu, engine, fmin, fmax, T):
 @pytest.mark.parametrize("engine", ENGINES)
 def test_cluster_size_invariance(gpu, engine, cs):
     """The same network sliced over 1..16 CTAs gives bit-identical results (global Philox indices)."""
-    p = O.params("4b", membrane_mode=1, init_seed=5, cluster_size=cs)
-    g, o = _pair(784, 512, 4, p, engine=engine)        # 16 groups of 32 columns: 200 KB on one CTA, 1 group per CTA at 16
+    p = O.params("2b", membrane_mode=1, init_seed=5, cluster_size=cs)
+    g, o = _pair(784, 512, 2, p, engine=engine)        # 16 groups of 32 columns: 100 KB on one CTA, 1 group per CTA at 16
     _compare_presentations(g, o, synthdata.images(2, "fashion"), 150, synthdata.seeds(2, 5), 784, 512, 1)
 
 
@@ -244,3 +244,27 @@ def test_raster_input_ltp_ltd_paths(gpu, engine):
     assert np.array_equal(g.weights(), o.weights())
     assert np.array_equal(g.stats()[:6], o.stats()[:6])
     assert o.stats()[3] > 0 and o.stats()[5] > 0
+
+
+# ------------------------------------------------------------------ event-engine rollback paths
+@pytest.mark.parametrize("engine", ENGINES)
+@pytest.mark.parametrize("mode,wta,stdp", [(0, 0, 0), (1, 0, 0), (1, 1, 0), (1, 1, 1)])
+def test_inh_hold_mode(gpu, engine, mode, wta, stdp):
+    """HOLD inhibition (inhibited neurons keep v): the event engine must re-simulate overrunning
+    columns instead of the RESET shortcut."""
+    p = O.params("8b", inh_mode=1, wta_mode=wta, stdp_mode=stdp, membrane_mode=mode, init_seed=12)
+    g, o = _pair(784, 400, 8, p, engine=engine)
+    _compare_presentations(g, o, synthdata.images(2, "mnist", start=40), 250, synthdata.seeds(2, 12), 784, 400, mode)
+    assert o.stats()[1] > 0
+
+
+@pytest.mark.parametrize("engine", ENGINES)
+def test_undo_log_overflow_path(gpu, engine):
+    """High input rates + gamma_dep = 1, tau_dep = 50: many LTD events per column-step overflow the
+    per-thread undo log, exercising the partial-step undo and horizon epochs of the event engine."""
+    p = O.params("2b", f_min_hz=200.0, f_max_hz=1000.0, gamma_dep=1.0, tau_dep=50.0, v_spike=0.5,
+                 membrane_mode=1, init_seed=13)
+    g, o = _pair(784, 256, 2, p, engine=engine)
+    _compare_presentations(g, o, synthdata.images(2, "fashion", start=3), 120, synthdata.seeds(2, 13), 784, 256, 1)
+    if engine == 0:
+        assert int(g.stats()[9]) > 0, "undo-log overflow path not exercised"

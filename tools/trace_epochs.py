@@ -1,0 +1,72 @@
+#!/usr/bin/env python
+"""Per-epoch phase breakdown of the event engine from the %globaltimer trace (snn_set_trace).
+Usage: python tools/trace_epochs.py [--n-exc 6400 --bits 2 --images 4 --cluster-size 0]"""
+import argparse
+import os
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import synthdata  # noqa: E402
+import paper_conf_date_shelm19_b200 as P  # noqa: E402
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--n-exc", type=int, default=6400)
+    ap.add_argument("--bits", type=int, default=2)
+    ap.add_argument("--images", type=int, default=4)
+    ap.add_argument("--T", type=int, default=350)
+    ap.add_argument("--cluster-size", type=int, default=0)
+    ap.add_argument("--kind", default="fashion")
+    a = ap.parse_args()
+    pre = {2: "2b", 4: "4b", 8: "8b"}[a.bits]
+    net = P.Network(784, a.n_exc, a.bits, P.preset(pre, cluster_size=a.cluster_size))
+    imgs = synthdata.images(a.images + 2, a.kind)
+    seeds = synthdata.seeds(a.images + 2, 1)
+    net.present_batch(imgs[:2], a.T, seeds[:2])            # warm-up
+    net.set_trace(64 * a.images)
+    net.reset_stats()
+    net.present_batch(imgs[2:], a.T, seeds[2:])
+    tr = net.trace().astype(np.int64)                       # (cs, E, 8)
+    st = net.stats()
+    cs, E, _ = tr.shape
+    valid = tr[0, :, 7] > 0
+    tr = tr[:, valid]
+    E = tr.shape[1]
+    k0 = tr[0, :, 0] & 0xFFFFFFFF
+    kind = tr[0, :, 1] >> 32
+    Pst = tr[0, :, 1] & 0xFFFFFFFF
+    start = tr[:, :, 2].min(axis=0)
+    spec_end = tr[:, :, 3]
+    summ = tr[:, :, 4]
+    exch = tr[:, :, 5]
+    comm = tr[:, :, 6]
+    end = tr[:, :, 7]
+    tot = end.max(axis=0) - start
+    spec = spec_end.max(axis=0) - start
+    spread = spec_end.max(axis=0) - spec_end.min(axis=0)
+    wait = exch.max(axis=0) - summ.max(axis=0)
+    commit = comm.max(axis=0) - exch.min(axis=0)
+    ltp = end.max(axis=0) - comm.min(axis=0)
+    adv = np.diff(np.append(k0, k0[-1]))
+    print(f"cluster {cs}  epochs {E}  images {a.images}  epochs/image {E / a.images:.1f}  post spikes {int(st[1])}")
+    print(f"per-epoch mean ns: total {tot.mean():.0f}  speculation {spec.mean():.0f} (spread across CTAs {spread.mean():.0f})"
+          f"  summary->exchanged {wait.mean():.0f}  commit {commit.mean():.0f}  LTP+tail {ltp.mean():.0f}")
+    print(f"per-image us: {tot.sum() / a.images / 1e3:.1f}   sum of per-epoch speculation {spec.sum() / a.images / 1e3:.1f}")
+    print(f"steps per epoch (mean) {np.mean(adv[adv > 0]):.1f}; speculation ns/step {spec.sum() / max(1, a.T * a.images):.0f}")
+    own = spec_end - tr[:, :, 2]                         # per-CTA speculation duration
+    skew = tr[:, :, 2] - start[None, :]                    # per-CTA start skew
+    steps = (Pst - k0 + 1).astype(float)
+    print(f"per-CTA speculation ns: mean {own.mean():.0f}  max-over-CTAs mean {own.max(axis=0).mean():.0f}  "
+          f"-> {own.max(axis=0).sum() / steps.sum():.0f} ns/step (max CTA)  {own.mean(axis=0).sum() / steps.sum():.0f} ns/step (mean CTA)")
+    print(f"start skew ns: mean {skew.mean():.0f}  max {skew.max(axis=0).mean():.0f}")
+    print("first 12 epochs: k0 P kind | spec(ns) spread wait commit ltp")
+    for e in range(min(12, E)):
+        print(f"{k0[e]:4d} {Pst[e]:5d} {kind[e]} | {spec[e]:7d} {spread[e]:6d} {wait[e]:6d} {commit[e]:6d} {ltp[e]:6d}")
+
+
+if __name__ == "__main__":
+    main()
