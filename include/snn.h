@@ -159,8 +159,10 @@ int snn_set_state(snn_handle* h, const void* buf, size_t n);
 int snn_get_stats(snn_handle* h, uint64_t stats[SNN_NSTATS]);
 int snn_reset_stats(snn_handle* h);
 /* Introspection: [0] cluster size, [1] threads per CTA, [2] dynamic smem bytes per CTA,
- * [3] words per weight row in a CTA slice, [4] q_max, [5] L_pot, [6] L_dep, [7] kernel launches so far. */
-int snn_get_info(const snn_handle* h, int64_t info[8]);
+ * [3] words per weight row in a CTA slice, [4] q_max, [5] L_pot, [6] L_dep, [7] kernel launches so far,
+ * [8] engine, [9] columns per thread (event engine), [10] on-chip row window, [11] LTD undo-log depth. */
+#define SNN_NINFO 12
+int snn_get_info(const snn_handle* h, int64_t info[SNN_NINFO]);
 
 /* Tracing: with max_epochs > 0 the event engine records, per CTA and epoch,
  * 8 u64 values: {image<<32 | k0, kind<<32 | P, t_spec_start, t_spec_end (max over warps),

@@ -8,8 +8,10 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <cstdlib>
 #include <string>
 #include <vector>
+#include <algorithm>
 
 using snn::NetDesc;
 
@@ -97,10 +99,12 @@ struct snn_handle {
   // event engine
   int engine = SNN_ENGINE_EVENT;
   int rows_cap = 0, offs_cap = 0, logn = 0;
+  int cpt = 1;                    // columns per thread of the event engine
   uint32_t* d_words = nullptr;   size_t words_cap = 0;
   uint32_t* d_ecnt = nullptr;    size_t ecnt_cap = 0;
   uint32_t* d_offs = nullptr;    size_t offs_buf_cap = 0;
   uint16_t* d_rows = nullptr;    size_t rows_buf_cap = 0;
+  uint16_t* d_rows16 = nullptr;  size_t rows16_cap = 0;
   unsigned long long* d_trace = nullptr; int trace_epochs = 0;
 };
 
@@ -147,7 +151,7 @@ void fill_static(const snn_handle* h, NetDesc& d) {
   std::memset(&d, 0, sizeof(d));
   const snn_params& p = h->p;
   d.n_in = h->n_in; d.n_exc = h->n_exc; d.bits = h->bits; d.q_max = h->q_max;
-  d.cs = h->cs; d.ngroups = h->ngroups; d.wpr = h->wpr;
+  d.cs = h->cs; d.ngroups = h->ngroups; d.wpr = h->wpr; d.slice_words = h->slice_words;
   d.nwi = (h->n_in + 31) / 32; d.nwe = (h->n_exc + 31) / 32;
   d.membrane_mode = p.membrane_mode;
   const double lsb = std::ldexp(1.0, -h->frac_bits);
@@ -172,7 +176,7 @@ void free_all(snn_handle* h) {
   void* ptrs[] = {h->d_w, h->d_enc, h->d_pot, h->d_dep, h->d_dbp, h->d_dbd, h->d_dtp, h->d_dtd,
                   h->d_v, h->d_cnt, h->d_lpost, h->d_lpre, h->d_stats, h->d_raster, h->d_inrec,
                   h->d_img, h->d_rin, h->d_seeds, h->d_counts, h->d_codes, h->d_bad,
-                  h->d_words, h->d_ecnt, h->d_offs, h->d_rows, h->d_trace};
+                  h->d_words, h->d_ecnt, h->d_offs, h->d_rows, h->d_rows16, h->d_trace};
   for (void* q : ptrs) if (q) cudaFree(q);
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
 }
@@ -239,10 +243,13 @@ int event_prepass(snn_handle* h, NetDesc& d, const uint8_t* images, const uint32
   const long long stride = ((long long)T * h->n_in + 7) & ~7LL;
   if ((rc = ensure(h, &h->d_offs, &h->offs_buf_cap, (size_t)n_images * (T + 1)))) return rc;
   if ((rc = ensure(h, &h->d_rows, &h->rows_buf_cap, (size_t)n_images * stride))) return rc;
-  CUDA_TRY(snn::launch_compact(words, h->d_ecnt, h->n_in, T, n_images, stride, h->d_offs, h->d_rows, h->stream));
+  if ((rc = ensure(h, &h->d_rows16, &h->rows16_cap, (size_t)n_images * T * snn::kPadRows))) return rc;
+  CUDA_TRY(snn::launch_compact(words, h->d_ecnt, h->n_in, T, n_images, stride, h->d_offs, h->d_rows, h->d_rows16,
+                               h->stream));
   h->launches++;
   d.ev_offs = h->d_offs;
   d.ev_rows = h->d_rows;
+  d.ev_rows16 = h->d_rows16;
   d.rows_stride = stride;
   if (d.in_raster_out)
     CUDA_TRY(cudaMemcpyAsync(d.in_raster_out, words + (size_t)(n_images - 1) * T * nwi, (size_t)T * nwi * 4,
@@ -310,7 +317,8 @@ int present_impl(snn_handle* h, const void* input, int n_images, int T, const ui
     rc = event_prepass(h, d, img, rin, n_images, T, (flags & SNN_KEEP_STATE) ? t0 : 0, sd);
     if (rc) return rc;
     lp.single = d;
-    CUDA_TRY(snn::launch_present_event(lp, 1, h->cs, h->nthr, h->smem, h->stream));
+    CUDA_TRY(snn::launch_present_event_mode(lp, 1, h->cs, h->nthr, h->smem, h->bits, h->cpt, h->p.membrane_mode,
+                                            h->stream));
   } else {
     lp.single = d;
     CUDA_TRY(snn::launch_present(lp, 1, h->cs, h->nthr, h->smem, h->stream));
@@ -425,35 +433,49 @@ int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** 
   h->ngroups = (n_exc + 31) / 32;
   h->engine = p->engine;
   int chosen = 0;
-  const int cs_lo = p->cluster_size > 0 ? p->cluster_size : 1;
-  const int cs_hi = p->cluster_size > 0 ? p->cluster_size : snn::kMaxCluster;
   const bool ev = h->engine == SNN_ENGINE_EVENT;
   const int max_thr = ev ? snn::kEvMaxThreads : snn::kMaxThreads;
-  for (int cs = cs_lo; cs <= cs_hi; ++cs) {
-    if (cs > h->ngroups) break;
+  const int cs_lo = p->cluster_size > 0 ? p->cluster_size : 1;
+  const int cs_hi = p->cluster_size > 0 ? p->cluster_size : snn::kMaxCluster;
+  // event engine: the largest cluster that fits (one exchange per epoch, so more SMs per network win);
+  // per-step engine: the smallest (one exchange per step, cheaper with fewer CTAs)
+  std::vector<int> order;
+  for (int cs = cs_lo; cs <= cs_hi; ++cs) order.push_back(cs);
+  if (ev && p->cluster_size == 0) std::reverse(order.begin(), order.end());
+  for (int cs : order) {
+    if (cs > h->ngroups) continue;
     const int max_groups = (h->ngroups + cs - 1) / cs;
-    if (max_groups * 32 > max_thr) continue;
-    const int nthr = max_groups * 32 < 128 ? 128 : max_groups * 32;
+    // columns per thread: SWAR-maximal (8/bits) -- fewest warps, fewest per-step instructions per SM
+    // (measured faster than 2 columns/thread on C4, profiles/r01_event_engine.md); SNN_CPT overrides
+    int cpt = 1;
+    if (ev) {
+      const char* env = getenv("SNN_CPT");
+      const int cap = 8 / bits;
+      cpt = cap;
+      if (env && atoi(env) >= 1 && atoi(env) <= cap && (cap % atoi(env)) == 0) cpt = atoi(env);
+    }
+    const int nthr = ev ? snn::event_threads(max_groups, bits, cpt) : (max_groups * 32 < 128 ? 128 : max_groups * 32);
+    if ((ev ? nthr : max_groups * 32) > max_thr) continue;
     const int wpr = max_groups * bits;
-    const int sw = ((n_in * wpr) + 3) & ~3;
+    const int sw = snn::slice_words_for(n_in, wpr);
     size_t smem;
     int rows_cap = 0, offs_cap = 0, logn = 0;
     if (ev) {
-      // on-chip window of active-row lists + LTD undo log
-      offs_cap = 1024;
-      logn = p->stdp_mode == SNN_STDP_STOCH ? 16 : 1;
-      rows_cap = std::max(n_in, 8192);
-      smem = snn::event_smem_bytes(n_in, sw, h->L_pot, h->L_dep, h->q_max, nthr, rows_cap, offs_cap, logn);
-      if (smem > (size_t)smem_optin) {         // shrink the row window down to one step's worth
-        rows_cap = n_in;
+      // on-chip window of active-row lists + LTD undo log: shrink until it fits
+      const int plans[4][3] = {{std::max(n_in, 4096), 512, 16}, {n_in, 256, 16}, {n_in, 128, 8}, {n_in, 64, 4}};
+      smem = 0;
+      for (int k = 0; k < 4; ++k) {
+        rows_cap = plans[k][0]; offs_cap = plans[k][1];
+        logn = p->stdp_mode == SNN_STDP_STOCH ? plans[k][2] : 1;
         smem = snn::event_smem_bytes(n_in, sw, h->L_pot, h->L_dep, h->q_max, nthr, rows_cap, offs_cap, logn);
+        if (smem <= (size_t)smem_optin) break;
       }
     } else {
       smem = snn::present_smem_bytes(n_in, sw, h->L_pot, h->L_dep, h->q_max, nthr);
     }
     if (smem > (size_t)smem_optin) continue;
     h->cs = cs; h->nthr = nthr; h->wpr = wpr; h->slice_words = sw; h->smem = smem;
-    h->rows_cap = rows_cap; h->offs_cap = offs_cap; h->logn = logn;
+    h->rows_cap = rows_cap; h->offs_cap = offs_cap; h->logn = logn; h->cpt = cpt;
     chosen = 1;
     break;
   }
@@ -463,7 +485,7 @@ int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** 
                 n_in, n_exc, bits, smem_optin);
   }
   int nclusters = 0;
-  ce = ev ? snn::query_max_clusters_event(h->cs, h->nthr, h->smem, &nclusters)
+  ce = ev ? snn::query_max_clusters_event(bits, h->cpt, p->membrane_mode, h->cs, h->nthr, h->smem, &nclusters)
           : snn::query_max_clusters(h->cs, h->nthr, h->smem, &nclusters);
   if (ce != cudaSuccess || nclusters < 1) {
     cudaGetLastError();
@@ -596,7 +618,9 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
   if (n_images < 0 || T < 0) return fail(SNN_EINVAL, "negative n_images / T");
   for (int k = 0; k < n; ++k) {
     if (!hs[k]) return fail(SNN_EINVAL, "handle %d is NULL", k);
-    if (hs[k]->n_in != hs[0]->n_in || hs[k]->cs != hs[0]->cs || hs[k]->nthr != hs[0]->nthr ||
+    const bool same_shape = hs[k]->engine == SNN_ENGINE_EVENT ? (hs[k]->bits != hs[0]->bits || hs[k]->nthr == hs[0]->nthr)
+                                                              : hs[k]->nthr == hs[0]->nthr;
+    if (hs[k]->n_in != hs[0]->n_in || hs[k]->cs != hs[0]->cs || !same_shape ||
         hs[k]->dev != hs[0]->dev || hs[k]->engine != hs[0]->engine ||
         hs[k]->p.membrane_mode != hs[0]->p.membrane_mode)
       return fail(SNN_EINVAL, "ensemble handles must share n_in, cluster size, CTA shape, engine, membrane mode, device");
@@ -608,8 +632,6 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
   if (n_images == 0) return SNN_OK;
   snn_handle* h0 = hs[0];
   DevGuard g(h0->dev);
-  size_t smem = 0;
-  for (int k = 0; k < n; ++k) smem = std::max(smem, hs[k]->smem);
   std::vector<NetDesc> descs(n);
   for (int k = 0; k < n; ++k) {
     snn_handle* h = hs[k];
@@ -632,14 +654,65 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
     h->stream = own;
     if (rc) return rc;
   }
+  // event engine: one launch per bit width (the kernel is specialised on it), the groups run
+  // concurrently on forked streams; step engine: one launch for the whole ensemble.
+  std::vector<std::vector<int>> groups;
+  if (ev) {
+    for (int bw : {2, 4, 8}) {
+      std::vector<int> g;
+      for (int k = 0; k < n; ++k) if (hs[k]->bits == bw) g.push_back(k);
+      if (!g.empty()) groups.push_back(g);
+    }
+  } else {
+    std::vector<int> g;
+    for (int k = 0; k < n; ++k) g.push_back(k);
+    groups.push_back(g);
+  }
   NetDesc* d_descs = nullptr;
   CUDA_TRY(cudaMalloc(&d_descs, sizeof(NetDesc) * n));
-  CUDA_TRY(cudaMemcpyAsync(d_descs, descs.data(), sizeof(NetDesc) * n, cudaMemcpyHostToDevice, h0->stream));
-  snn::LaunchParams lp;
-  std::memset(&lp, 0, sizeof(lp));
-  lp.descs = d_descs;
-  cudaError_t e = ev ? snn::launch_present_event_mode(lp, n, h0->cs, h0->nthr, smem, h0->p.membrane_mode, h0->stream)
-                     : snn::launch_present(lp, n, h0->cs, h0->nthr, smem, h0->stream);
+  std::vector<NetDesc> ordered;
+  for (auto& g : groups) for (int k : g) ordered.push_back(descs[k]);
+  CUDA_TRY(cudaMemcpyAsync(d_descs, ordered.data(), sizeof(NetDesc) * n, cudaMemcpyHostToDevice, h0->stream));
+  cudaError_t e = cudaSuccess;
+  std::vector<cudaStream_t> forks;
+  cudaEvent_t ready = nullptr;
+  if (groups.size() > 1) {
+    e = cudaEventCreateWithFlags(&ready, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventRecord(ready, h0->stream);
+  }
+  size_t off = 0;
+  for (size_t gi = 0; gi < groups.size() && e == cudaSuccess; ++gi) {
+    const std::vector<int>& g = groups[gi];
+    snn::LaunchParams lp;
+    std::memset(&lp, 0, sizeof(lp));
+    lp.descs = d_descs + off;
+    size_t smem = 0;
+    for (int k : g) smem = std::max(smem, hs[k]->smem);
+    cudaStream_t st = h0->stream;
+    if (groups.size() > 1) {
+      e = cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking);
+      if (e != cudaSuccess) break;
+      forks.push_back(st);
+      e = cudaStreamWaitEvent(st, ready, 0);
+      if (e != cudaSuccess) break;
+    }
+    for (int k : g)
+      if (hs[k]->nthr != hs[g[0]]->nthr) { e = cudaErrorInvalidValue; break; }
+    if (e != cudaSuccess) break;
+    for (int k : g)
+      if (hs[k]->cpt != hs[g[0]]->cpt) { e = cudaErrorInvalidValue; break; }
+    if (e != cudaSuccess) break;
+    e = ev ? snn::launch_present_event_mode(lp, (int)g.size(), h0->cs, hs[g[0]]->nthr, smem, hs[g[0]]->bits,
+                                            hs[g[0]]->cpt, h0->p.membrane_mode, st)
+           : snn::launch_present(lp, (int)g.size(), h0->cs, h0->nthr, smem, st);
+    off += g.size();
+  }
+  for (cudaStream_t st : forks) {
+    cudaError_t e2 = cudaStreamSynchronize(st);
+    if (e == cudaSuccess) e = e2;
+    cudaStreamDestroy(st);
+  }
+  if (ready) cudaEventDestroy(ready);
   if (e == cudaSuccess) e = cudaStreamSynchronize(h0->stream);
   cudaFree(d_descs);
   if (e != cudaSuccess) return fail(SNN_ECUDA, "present_many: %s", cudaGetErrorString(e));
@@ -807,10 +880,11 @@ int snn_get_trace(snn_handle* h, uint64_t* out, size_t cap) {
   return SNN_OK;
 }
 
-int snn_get_info(const snn_handle* h, int64_t info[8]) {
+int snn_get_info(const snn_handle* h, int64_t info[SNN_NINFO]) {
   if (!h || !info) return fail(SNN_EINVAL, "NULL argument");
   info[0] = h->cs; info[1] = h->nthr; info[2] = (int64_t)h->smem; info[3] = h->wpr;
   info[4] = h->q_max; info[5] = h->L_pot; info[6] = h->L_dep; info[7] = h->launches;
+  info[8] = h->engine; info[9] = h->cpt; info[10] = h->rows_cap; info[11] = h->logn;
   return SNN_OK;
 }
 

@@ -88,7 +88,7 @@ __global__ void counts_from_raster_kernel(const uint32_t* __restrict__ raster, i
 // expands the bit-packed words into ascending row indices.
 __global__ void __launch_bounds__(256) compact_kernel(const uint32_t* __restrict__ words, const uint32_t* __restrict__ counts,
                                                       int n_in, int T, long long rows_stride, uint32_t* __restrict__ offs,
-                                                      uint16_t* __restrict__ rows) {
+                                                      uint16_t* __restrict__ rows, uint16_t* __restrict__ rows16) {
   __shared__ uint32_t s_warp[32];
   const int b = blockIdx.x, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int nthr = blockDim.x, nwarps = nthr >> 5;
@@ -126,6 +126,10 @@ __global__ void __launch_bounds__(256) compact_kernel(const uint32_t* __restrict
   uint16_t* rw = rows + (size_t)b * rows_stride;
   for (int k = warp; k < T; k += nwarps) {
     uint32_t base = off[k];
+    const uint32_t kbase = base;
+    uint16_t* r16 = rows16 + ((size_t)b * T + k) * kPadRows;
+    if (lane < kPadRows) r16[lane] = (uint16_t)n_in;          // padding -> the all-zero weight row
+    __syncwarp();
     const uint32_t* wk = words + ((size_t)b * T + k) * nwi;
     for (int w0 = 0; w0 < nwi; w0 += 32) {
       const int w = w0 + lane;
@@ -142,6 +146,7 @@ __global__ void __launch_bounds__(256) compact_kernel(const uint32_t* __restrict
       while (word) {
         const int bp = __ffs(word) - 1;
         word &= word - 1;
+        if (pos - kbase < (uint32_t)kPadRows) r16[pos - kbase] = (uint16_t)(w * 32 + bp);
         rw[pos++] = (uint16_t)(w * 32 + bp);
       }
       base += (uint32_t)__shfl_sync(FULL, inc, 31);
@@ -150,36 +155,92 @@ __global__ void __launch_bounds__(256) compact_kernel(const uint32_t* __restrict
 }
 
 // ====================================================================== main kernel
+// Thread -> column mapping: the slice is packed row-major, word w of a row holds
+// local columns w*cpw .. w*cpw+cpw-1 (cpw = 32/BITS).  Four threads share a word: thread
+// (w, f) owns the CPT = 8/BITS columns at fields f, f+4, f+8, f+12, which sit LW = 32/CPT bits
+// apart, so one shift+mask of the word yields all of the thread's codes in separate SWAR lanes
+// and one add integrates all of them (eq.(3)).
+constexpr int kBlk = 8;             // steps per speculation block
 
-// S_j over the active rows [r0, r1) of one step: independent loads, unrolled for ILP (eq.(3))
-__device__ __forceinline__ int integrate(const uint32_t* __restrict__ wcol, const uint16_t* __restrict__ rows, int r0,
-                                        int r1, int wpr, int sh, uint32_t fmask) {
-  int S = 0;
+// Swar<BITS, CPT>: a thread owns CPT columns of one packed word, LW = 32/CPT bits apart; TPW = CPW/CPT
+// threads share the word.  One shift+mask yields the thread's CPT codes in separate SWAR lanes.
+template <int BITS, int CPT_> struct Swar {
+  static constexpr int CPT = CPT_;
+  static constexpr int CPW = 32 / BITS;
+  static constexpr int TPW = CPW / CPT_;
+  static constexpr int LW = 32 / CPT_;
+  static constexpr uint32_t FM = (1u << BITS) - 1u;
+  static constexpr uint32_t LMASK = CPT_ == 1 ? FM : (CPT_ == 2 ? (FM | (FM << 16)) : (FM * 0x01010101u));
+  // rows that can be summed before a lane overflows
+  static constexpr int CHUNK = CPT_ == 1 ? (1 << 30) : (int)(((1u << (LW & 31)) - 1u) / FM);
+};
+// S[c] = sum over the active rows [r0, r1) of the thread's CPT codes (exact; lanes never overflow)
+template <int BITS, int CPT_>
+__device__ __forceinline__ void integrate_swar(const uint32_t* __restrict__ wcol, const uint16_t* __restrict__ rows,
+                                               int r0, int r1, int wpr, int fsh, int (&S)[CPT_]) {
+  using Z = Swar<BITS, CPT_>;
+#pragma unroll
+  for (int c = 0; c < Z::CPT; ++c) S[c] = 0;
   int r = r0;
-  for (; r + 4 <= r1; r += 4) {
-    const int i0 = rows[r], i1 = rows[r + 1], i2 = rows[r + 2], i3 = rows[r + 3];
-    const uint32_t w0 = wcol[i0 * wpr], w1 = wcol[i1 * wpr], w2 = wcol[i2 * wpr], w3 = wcol[i3 * wpr];
-    S += (int)(((w0 >> sh) & fmask) + ((w1 >> sh) & fmask) + ((w2 >> sh) & fmask) + ((w3 >> sh) & fmask));
+  while (r < r1) {
+    const int rend = min(r1, r + Z::CHUNK);
+    uint32_t acc = 0;
+    for (; r + 4 <= rend; r += 4) {
+      const int i0 = rows[r], i1 = rows[r + 1], i2 = rows[r + 2], i3 = rows[r + 3];
+      const uint32_t w0 = wcol[i0 * wpr], w1 = wcol[i1 * wpr], w2 = wcol[i2 * wpr], w3 = wcol[i3 * wpr];
+      acc += ((w0 >> fsh) & Z::LMASK) + ((w1 >> fsh) & Z::LMASK) + ((w2 >> fsh) & Z::LMASK) + ((w3 >> fsh) & Z::LMASK);
+    }
+    for (; r < rend; ++r) acc += (wcol[(int)rows[r] * wpr] >> fsh) & Z::LMASK;
+#pragma unroll
+    for (int c = 0; c < Z::CPT; ++c)
+      S[c] += (int)(Z::LW == 32 ? acc : ((acc >> (c * Z::LW)) & ((1u << (Z::LW & 31)) - 1u)));
   }
-  for (; r < r1; ++r) S += (int)((wcol[(int)rows[r] * wpr] >> sh) & fmask);
-  return S;
 }
 
-// LTD draws of column j against rows [r0, r0 + n), n <= 32: bit m set iff u_LTD(t, rows[r0+m], j) <= thr.
-// Branch-free so that the independent Philox blocks overlap (eq.(7), R13).
-__device__ __forceinline__ uint32_t ltd_draws(const uint16_t* __restrict__ rows, int r0, int n, uint32_t t, int j,
-                                              uint32_t thr, unsigned long long seed) {
-  uint32_t m = 0;
-  const int lanej = j & 3;
-#pragma unroll 4
-  for (int x = 0; x < n; ++x) {
-    const uint4 u = philox(t, (uint32_t)rows[r0 + x], (uint32_t)(j >> 2), TAG_LTD, seed);
-    m |= (pick(u, lanej) <= thr ? 1u : 0u) << x;
-  }
-  return m;
+// lane-wise max of two SWAR words (lanes of 32/CPT bits)
+template <int CPT>
+__device__ __forceinline__ uint32_t vmax_lanes(uint32_t a, uint32_t b) {
+  if constexpr (CPT == 4) return __vmaxu4(a, b);
+  else if constexpr (CPT == 2) return __vmaxu2(a, b);
+  else return a > b ? a : b;
 }
+
+
+// After an applied LTD decrement of row i at block step b (or its undo), add `delta` (one LSB of the
+// column's SWAR lane, two's complement for -1) to the running-sum slot of every later block step at
+// or after the first later step whose rows contain i, and to every later non-empty slot after it.
+// Rows r in [rlo, rhi) belong to steps > b (ascending).  Slots of empty steps stay 0.
+template <int CPT>
+__device__ __forceinline__ void block_correct(const uint16_t* __restrict__ rows, const uint16_t* __restrict__ rstep,
+                                              uint32_t* my_acc, int nthr, int rlo, int rhi, int sbase, int b, int nb,
+                                              int i, uint32_t delta) {
+  // first later step containing row i (one pass, 8 independent loads per group)
+  int first = nb;
+  for (int r = rlo; r < rhi && first == nb; r += 8) {
+    uint32_t rv[8];
+#pragma unroll
+    for (int x = 0; x < 8; ++x) rv[x] = r + x < rhi ? (uint32_t)rows[r + x] : 0xFFFFFFFFu;
+#pragma unroll
+    for (int x = 0; x < 8; ++x)
+      if (rv[x] == (uint32_t)i && first == nb) first = (int)rstep[r + x] - sbase;
+  }
+  if (first >= nb) return;
+  // each occurrence of i at step s2 lowers the running sums of every step >= s2: walk the later rows once
+  uint32_t cum = 0u;
+  int rr = rlo;
+  for (int b2 = b + 1; b2 < nb; ++b2) {
+    bool nonempty = false;
+    while (rr < rhi && (int)rstep[rr] - sbase == b2) {
+      if ((uint32_t)rows[rr] == (uint32_t)i) cum += delta;
+      nonempty = true;
+      ++rr;
+    }
+    if (nonempty && cum) my_acc[b2 * nthr] += cum;
+  }
+}
+
 struct EvLayout {
-  size_t slots, wsum, flags, misc, w, pot, dep, dbp, dbd, dtp, dtd, lpre, offs, rows, log, splist, total;
+  size_t slots, wsum, flags, misc, w, pot, dep, dbp, dbd, dtp, dtd, lpre, lpost, offs, rows, rows16, rstep, ev, acc, log, total;
 };
 
 __host__ __device__ inline EvLayout ev_layout(int n_in, int slice_words, int L_pot, int L_dep, int q_max, int nthr,
@@ -198,10 +259,14 @@ __host__ __device__ inline EvLayout ev_layout(int n_in, int slice_words, int L_p
   L.dtp = o;    o = align16(o + (size_t)(q_max + 1) * 4);
   L.dtd = o;    o = align16(o + (size_t)(q_max + 1) * 4);
   L.lpre = o;   o = align16(o + (size_t)n_in * 4);
+  L.lpost = o;  o = align16(o + (size_t)nthr * 4 * 4);        // last_post of the CTA's local columns
   L.offs = o;   o = align16(o + (size_t)(offs_cap + 1) * 4);
   L.rows = o;   o = align16(o + (size_t)rows_cap * 2);
+  L.rows16 = o; o = align16(o + (size_t)rows_cap * 4);               // word offset (row * wpr) of every window row
+  L.rstep = o;  o = align16(o + (size_t)rows_cap * 2);               // step (relative to the window) of every row
+  L.ev = o;     o = align16(o + (size_t)8 * nthr * 4);               // block LTD event masks [c][2][thread]
+  L.acc = o;    o = align16(o + (size_t)kBlk * nthr * 4);            // block SWAR sums [b][thread]
   L.log = o;    o = align16(o + (size_t)logn * nthr * 4);
-  L.splist = o; o = align16(o + (size_t)nthr * 2);
   L.total = o;
   return L;
 }
@@ -211,8 +276,18 @@ size_t event_smem_bytes(int n_in, int slice_words, int L_pot, int L_dep, int q_m
   return ev_layout(n_in, slice_words, L_pot, L_dep, q_max, nthr, rows_cap, offs_cap, logn).total;
 }
 
-template <bool FIXED>
+// undo-log entry: rel step (16) | column slot c (2) | applied (1) | row (13)
+__device__ __forceinline__ uint32_t log_entry(int rel, int c, bool applied, int row) {
+  return ((uint32_t)rel << 16) | ((uint32_t)c << 14) | (applied ? 0x2000u : 0u) | (uint32_t)row;
+}
+
+template <int BITS, int CPT_, bool FIXED>
 __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const __grid_constant__ LaunchParams lp) {
+  using Z = Swar<BITS, CPT_>;
+  constexpr int CPT = Z::CPT;
+  constexpr int CPW = Z::CPW;
+  constexpr int TPW = Z::TPW;
+  constexpr uint32_t FMASK = (1u << BITS) - 1u;
   extern __shared__ __align__(16) unsigned char smem[];
   const NetDesc& d0 = lp.descs ? lp.descs[0] : lp.single;
   const int cs = d0.cs;
@@ -220,10 +295,10 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
   const int rank = blockIdx.x - net * cs;
   const NetDesc& d = lp.descs ? lp.descs[net] : lp.single;
 
-  const int n_in = d.n_in, n_exc = d.n_exc, bits = d.bits, qmax = d.q_max, wpr = d.wpr, nwe = d.nwe;
+  const int n_in = d.n_in, n_exc = d.n_exc, qmax = d.q_max, wpr = d.wpr, nwe = d.nwe;
   const int T = d.T, flags = d.flags, n_images = d.n_images;
   const int L_pot = d.L_pot, L_dep = d.L_dep, rows_cap = d.rows_cap, offs_cap = d.offs_cap, logn = d.logn;
-  const int slice_words = ((n_in * wpr) + 3) & ~3;
+  const int slice_words = d.slice_words;
   const int nthr = blockDim.x;
   const EvLayout L = ev_layout(n_in, slice_words, L_pot, L_dep, qmax, nthr, rows_cap, offs_cap, logn);
   unsigned long long* s_slots = reinterpret_cast<unsigned long long*>(smem + L.slots);
@@ -238,30 +313,38 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
   uint32_t* s_dtp = reinterpret_cast<uint32_t*>(smem + L.dtp);
   uint32_t* s_dtd = reinterpret_cast<uint32_t*>(smem + L.dtd);
   int* s_lpre = reinterpret_cast<int*>(smem + L.lpre);
+  int* s_lpost = reinterpret_cast<int*>(smem + L.lpost);
   uint32_t* s_offs = reinterpret_cast<uint32_t*>(smem + L.offs);
   uint16_t* s_rows = reinterpret_cast<uint16_t*>(smem + L.rows);
+  uint32_t* s_woff = reinterpret_cast<uint32_t*>(smem + L.rows16);
+  uint16_t* s_rstep = reinterpret_cast<uint16_t*>(smem + L.rstep);
+  uint32_t* s_ev = reinterpret_cast<uint32_t*>(smem + L.ev);
+  uint32_t* s_acc = reinterpret_cast<uint32_t*>(smem + L.acc);
   uint32_t* s_log = reinterpret_cast<uint32_t*>(smem + L.log);
-  uint16_t* s_splist = reinterpret_cast<uint16_t*>(smem + L.splist);
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwarps = nthr >> 5;
   const int g0 = (rank * d.ngroups) / cs, g1 = ((rank + 1) * d.ngroups) / cs;
   const int col0 = g0 * 32;
   const int ncols = min(g1 * 32, n_exc) - col0;
-  const int ngrp_cta = g1 - g0;
-  const bool mycol = tid < ncols;
-  const int j = col0 + tid;
-  const int lg = bits == 2 ? 4 : (bits == 4 ? 3 : 2);
-  const int wj = tid >> lg;
-  const int sh = (tid & ((1 << lg) - 1)) * bits;
-  const uint32_t fmask = (1u << bits) - 1u;
-  const int nq4 = (n_in + 3) >> 2;
+  // this thread's word and columns
+  const int wj = tid / TPW, f = tid % TPW;
+  const int fsh = f * BITS;                                  // SWAR shift of the thread's lanes
   uint32_t* const wcol = s_w + wj;
+  int jcol[CPT];                                             // global column of slot c (or -1)
+  uint32_t valid = 0;
+#pragma unroll
+  for (int c = 0; c < CPT; ++c) {
+    const int jl = wj * CPW + f + TPW * c;
+    jcol[c] = (jl < ncols && wj < wpr) ? col0 + jl : -1;
+    if (jcol[c] >= 0) valid |= 1u << c;
+  }
+  const bool mycol = valid != 0;
+  const int nq4 = (n_in + 3) >> 2;
 
   Lif lif;
   lif.load(d);
-  const bool fixed = lif.fixed;
-  const int vreset = fixed ? d.Vreset : __float_as_int(d.vresetf);
-  const int vinit = fixed ? d.Vinit : __float_as_int(d.vinitf);
+  const int vreset = FIXED ? d.Vreset : __float_as_int(d.vresetf);
+  const int vinit = FIXED ? d.Vinit : __float_as_int(d.vinitf);
   const int t_ref = d.t_ref, t_inh = d.t_inh, t_ltp = d.t_ltp;
   const bool hard = d.wta_mode == 0;
   const bool stoch = d.stdp_mode == 0;
@@ -282,25 +365,40 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
     for (int k = tid; k < slice_words / 4; k += nthr) dst[k] = src[k];
   }
   if (tid == 0) { s_flag[0] = INT_MAX; s_flag[1] = INT_MAX; }
-  int v = vinit, cnt = 0, lpost = kNever;
-  if (keep) {
-    if (mycol) { v = d.v[j]; cnt = d.cnt[j]; lpost = d.last_post[j]; }
-    for (int i = tid; i < n_in; i += nthr) s_lpre[i] = d.last_pre[i];
+  int v[CPT], cnt[CPT], lpost[CPT];
+#pragma unroll
+  for (int c = 0; c < CPT; ++c) {
+    v[c] = vinit; cnt[c] = 0; lpost[c] = kNever;
+    if (keep && (valid >> c & 1u)) { v[c] = d.v[jcol[c]]; cnt[c] = d.cnt[jcol[c]]; lpost[c] = d.last_post[jcol[c]]; }
   }
+  if (keep) for (int i = tid; i < n_in; i += nthr) s_lpre[i] = d.last_pre[i];
+#pragma unroll
+  for (int c = 0; c < CPT; ++c)
+    if (valid >> c & 1u) s_lpost[jcol[c] - col0] = lpost[c];
   uint32_t ltd_trials = 0, ltd_events = 0, ltp_trials = 0, ltp_events = 0;   // per launch, < 2^32
   unsigned long long act_sum = 0, post_sum = 0;
   uint32_t eng_epochs = 0, eng_hz = 0, eng_resim = 0, eng_spec = 0, eng_undo = 0;
-  // every CTA of the cluster has initialised its flags before any remote red.min can target them
   if (cs > 1) { cluster_arrive(); cluster_wait(); } else { __syncthreads(); }
 
   int ep = 0;
   unsigned long long* trace = d.trace ? d.trace + (size_t)rank * d.trace_cap * 8 : nullptr;
-  unsigned long long* s_tmax = reinterpret_cast<unsigned long long*>(s_misc + 8);   // max speculation end
+  unsigned long long* s_tmax = reinterpret_cast<unsigned long long*>(s_misc + 8);
   unsigned long long tr0 = 0, tr2 = 0, tr3 = 0;
+  long long prof_int = 0, prof_ltd = 0, prof_seq = 0, prof_blk = 0, prof_loop0 = 0, prof_loop = 0;
+  const long long prof_clk0 = clock64();
+  const unsigned long long prof_ns0 = globaltimer();
+  // pending LTP of the previous epoch (owner warps run it while the others start speculating)
+  int pend_t = -1;
+  uint32_t pend_mask = 0;                                      // bit c: this thread's column c spiked
+
   for (int b = 0; b < n_images; ++b) {
     const unsigned long long seed = d.seeds[b];
     if (!keep) {
-      v = vinit; cnt = 0; lpost = kNever;
+#pragma unroll
+      for (int c = 0; c < CPT; ++c) {
+        v[c] = vinit; cnt[c] = 0; lpost[c] = kNever;
+        if (valid >> c & 1u) s_lpost[jcol[c] - col0] = kNever;
+      }
       for (int i = tid; i < n_in; i += nthr) s_lpre[i] = kNever;
     }
     const uint32_t* offs_g = d.ev_offs + (size_t)b * (T + 1);
@@ -315,8 +413,61 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
     __syncthreads();
 
     while (k0 < T) {
+      // ---------------------------------------------------------- (a5)/(a6) pending LTP of the last event
+      // Run by the warps that own a spiking column; the other warps go straight to speculation.
+      // Updates are atomic (other columns' LTD shares the words), and column W's own thread is in
+      // this warp, so it cannot speculate on W before W's potentiation is complete.
+      if (__any_sync(FULL, pend_mask != 0)) {
+        const int tP = pend_t;
+        for (uint32_t wm = __ballot_sync(FULL, pend_mask != 0); wm; wm &= wm - 1) {
+          const int Lsrc = __ffs(wm) - 1;
+          const uint32_t pm = __shfl_sync(FULL, pend_mask, Lsrc);
+          for (uint32_t cm = pm; cm; cm &= cm - 1) {
+            const int c = __ffs(cm) - 1;
+            const int tidL = warp * 32 + Lsrc;
+            const int jl = (tidL / TPW) * CPW + (tidL % TPW) + TPW * c;
+            const int Wg = col0 + jl;
+            const int ww = jl / CPW, wsh = (jl % CPW) * BITS;
+            for (int grp = lane; grp < nq4; grp += 32) {
+              const uint4 u = philox((uint32_t)tP, (uint32_t)Wg, (uint32_t)grp, stoch ? TAG_LTP : TAG_ROUND, seed);
+#pragma unroll
+              for (int r = 0; r < 4; ++r) {
+                const int i = 4 * grp + r;
+                if (i >= n_in) break;
+                const int lpi = s_lpre[i];
+                uint32_t* pw = s_w + i * wpr + ww;
+                if (stoch) {
+                  if (lpi < 0) continue;
+                  const int D = tP - lpi;
+                  if (D >= L_pot) continue;
+                  ++ltp_trials;
+                  if (pick(u, r) <= s_pot[D]) {                // eq.(6), R10: Dt = D >= 0
+                    ++ltp_events;
+                    if (((*pw >> wsh) & FMASK) < (uint32_t)qmax) atomicAdd(pw, 1u << wsh);
+                  }
+                } else {                                       // eqs.(4)(5)(8), R16/R17
+                  const int q0 = (int)((*pw >> wsh) & FMASK);
+                  const bool pot = lpi >= 0 && (tP - lpi) <= t_ltp;
+                  const int base = pot ? s_dbp[q0] : s_dbd[q0];
+                  const uint32_t thr = pot ? s_dtp[q0] : s_dtd[q0];
+                  const int dq = base + (pick(u, r) < thr ? 1 : 0);
+                  int q1 = pot ? q0 + dq : q0 - dq;
+                  q1 = q1 < 0 ? 0 : (q1 > qmax ? qmax : q1);
+                  if (q1 != q0) atomicAdd(pw, (uint32_t)(q1 - q0) << wsh);
+                  if (pot) { ++ltp_trials; if (dq > 0) ++ltp_events; }
+                  else     { ++ltd_trials; if (dq > 0) ++ltd_events; }
+                }
+              }
+            }
+          }
+        }
+        pend_mask = 0;
+        __syncwarp();
+      }
+
       // ---------------------------------------------------------- stage the active-row window
       if (k0 >= kb) {
+        __syncthreads();
         ka = k0;
         const int n_o = min(offs_cap, T - ka);
         for (int x = tid; x <= n_o; x += nthr) s_offs[x] = offs_g[ka + x];
@@ -332,85 +483,302 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         const uint32_t nrows = s_offs[nsteps] - wbase;
         for (uint32_t x = tid; x < nrows; x += nthr) s_rows[x] = rows_g[wbase + x];
         __syncthreads();
+        for (uint32_t x = tid; x < nrows; x += nthr) s_woff[x] = (uint32_t)s_rows[x] * (uint32_t)wpr;
+        for (int x = tid; x < nsteps; x += nthr)
+          for (uint32_t r = s_offs[x] - wbase; r < s_offs[x + 1] - wbase; ++r) s_rstep[r] = (uint16_t)x;
+        __syncthreads();
       }
       const int kend = kb;
       const int fp = ep & 1;
       if (trace && tid == 0) { tr0 = globaltimer(); *s_tmax = 0ull; }
 
-      // ---------------------------------------------------------- speculation (column-local, no barriers)
-      int p = kend;            // first step not fully processed by this thread
-      bool cand = false;       // stopped at its own threshold crossing at p (LIF done, LTD pending)
-      bool hz = false;         // stopped at p with nothing done (undo log full)
-      const int v0 = v, cnt0 = cnt;
-      int v1 = v, cnt1 = cnt, vb = v;
+      // ---------------------------------------------------------- speculation (warp-synchronous, no CTA barrier)
+      int p = kend;             // first step this thread did not fully process
+      bool cand = false;        // stopped at a crossing at p (LIF done for all its columns, LTD pending)
+      bool hz = false;          // stopped at p with nothing done (undo log full)
+      uint32_t cmask = 0;       // columns crossing at p
+      int cnt0[CPT], v1[CPT], cnt1[CPT], vb[CPT], cb[CPT];
+#pragma unroll
+      for (int c = 0; c < CPT; ++c) { cnt0[c] = cnt[c]; v1[c] = v[c]; cnt1[c] = cnt[c]; vb[c] = v[c]; cb[c] = cnt[c]; }
       int nlog = 0;
       {
-        // Warp-synchronous speculation: every lane of the warp walks the same step kk (lanes that
-        // stopped are predicated off), so the LTD Philox blocks of an LTD-active column can be
-        // spread over all 32 lanes (one block per row) instead of serialised in one lane.
         const uint32_t flag_addr = smem_u32(&s_flag[fp]);
-        const bool ltd_col = mycol && stoch && lpost >= 0;
-        const int jw = col0 + warp * 32;                          // column of lane 0 of this warp
+        uint32_t ltd_cols = 0;                                    // columns with a valid last_post
+#pragma unroll
+        for (int c = 0; c < CPT; ++c)
+          if (stoch && (valid >> c & 1u) && lpost[c] >= 0) ltd_cols |= 1u << c;
         bool done = !mycol;
         int kk = k0;
         int r0 = (int)(s_offs[k0 - ka] - wbase);
-        auto signal = [&](int f) {                                // tell the cluster where to stop
-          atomicMin(&s_flag[fp], f);
+        auto signal = [&](int fstep) {                            // tell the cluster where to stop
+          atomicMin(&s_flag[fp], fstep);
           for (int r = 0; r < cs; ++r)
-            if (r != rank) red_min_cluster(&s_flag[fp], (uint32_t)r, f);
+            if (r != rank) red_min_cluster(&s_flag[fp], (uint32_t)r, fstep);
         };
+        if (trace && lane == 0) prof_loop0 = clock64();
         while (__any_sync(FULL, !done)) {
           if (!done && (kk >= kend || kk > ld_volatile_shared_u32addr(flag_addr))) { done = true; p = kk; }
           if (kk >= kend) break;                                  // warp-uniform
+          // ======== block path: up to kBlk steps of <= kPadRows rows each (<= 64 rows in all).
+          // Integration of all block steps is independent of v, so it is issued at once from the
+          // fixed-width row slots (pad index n_in -> the all-zero row); the block's LTD Philox blocks
+          // are drawn in <= 2 warp-wide passes; only the LIF chain runs step by step.  An applied LTD
+          // decrement at step b is subtracted from the sums of the later block steps that contain
+          // the same row (exact: the sum was taken with the pre-decrement code).
+          {
+            int nb = 0;
+#pragma unroll
+            for (int b = 0; b < kBlk; ++b)
+              if (nb == b && kk + b < kend && (int)(s_offs[kk - ka + b + 1] - wbase) - r0 <= 64) nb = b + 1;
+            if (nb > 0) {
+              const int kb0 = kk;
+              const bool prof = trace && lane == 0;
+              long long pc0 = prof ? clock64() : 0;
+              uint32_t* const my_acc = s_acc + tid;              // [b * nthr + tid]: SWAR sums of block step b
+              const int rblk0 = r0;
+              const int rblk1 = (int)(s_offs[kb0 - ka + nb] - wbase);
+              if (!done) {
+                // (a2) eq.(3) for all block steps in one flattened pass over the block's rows: the running
+                // SWAR sum is stored into the slot of the row's step; lanes never overflow (<= 64 rows), so
+                // the sum at the end of step b is the lane-wise max of slots 0..b.
+#pragma unroll 1
+                for (int b = 0; b < nb; ++b) my_acc[b * nthr] = 0u;
+                uint32_t run = 0u;
+                const int sbase = kb0 - ka;
+                // groups of 8 rows: all loads of a group are issued before its stores (the slots live in
+                // the same shared buffer, so the compiler would otherwise serialise load after store)
+#pragma unroll 1
+                for (int r = rblk0; r < rblk1; r += 8) {
+                  uint32_t o[8], st[8], w[8];
+#pragma unroll
+                  for (int x = 0; x < 8; ++x) {
+                    const bool in = r + x < rblk1;
+                    o[x] = in ? s_woff[r + x] : (uint32_t)(n_in * wpr);   // the all-zero row
+                    st[x] = in ? (uint32_t)s_rstep[r + x] : 0xFFFFu;
+                  }
+#pragma unroll
+                  for (int x = 0; x < 8; ++x) w[x] = (wcol[o[x]] >> fsh) & Z::LMASK;
+#pragma unroll
+                  for (int x = 0; x < 8; ++x) {
+                    run += w[x];
+                    if (st[x] != 0xFFFFu) my_acc[((int)st[x] - sbase) * nthr] = run;
+                  }
+                }
+              }
+              long long pc1 = prof ? clock64() : 0;
+              // ---- LTD draws of the block for every LTD-active (lane, column) pair (eq.(7))
+              uint32_t ltd_blk = 0;
+              if (!done) {
+#pragma unroll
+                for (int c = 0; c < CPT; ++c)
+                  if ((ltd_cols >> c & 1u) && (tbase + kb0 - lpost[c]) < L_dep) ltd_blk |= 1u << c;
+              }
+              const int nrows_blk = rblk1 - rblk0;
+              if (__any_sync(FULL, ltd_blk != 0)) {
+                // this lane's rows of the block and their steps (the same for every pair)
+                const int bsel0 = lane < nrows_blk ? (int)s_rstep[rblk0 + lane] - (kb0 - ka) : 0;
+                const int bsel1 = lane + 32 < nrows_blk ? (int)s_rstep[rblk0 + 32 + lane] - (kb0 - ka) : 0;
+                const uint32_t row0 = lane < nrows_blk ? (uint32_t)s_rows[rblk0 + lane] : 0u;
+                const uint32_t row1 = lane + 32 < nrows_blk ? (uint32_t)s_rows[rblk0 + 32 + lane] : 0u;
+#pragma unroll 1
+                for (uint32_t lm = __ballot_sync(FULL, ltd_blk != 0); lm; lm &= lm - 1) {
+                  const int Ls = __ffs(lm) - 1;
+                  const int tidL = warp * 32 + Ls;
+#pragma unroll 1
+                  for (uint32_t cm = __shfl_sync(FULL, ltd_blk, Ls); cm; cm &= cm - 1) {
+                    const int c = __ffs(cm) - 1;
+                    const int jlL = (tidL / TPW) * CPW + (tidL % TPW) + TPW * c;
+                    const int jL = col0 + jlL;
+                    const int lpL = s_lpost[jlL];
+#pragma unroll 1
+                    for (int m = 0; m < 2; ++m) {
+                      const int x = 32 * m + lane;
+                      bool bit = false;
+                      if (x < nrows_blk) {
+                        const int t = tbase + kb0 + (m ? bsel1 : bsel0);
+                        const int D = t - lpL;
+                        if (D < L_dep) {
+                          const uint4 u = philox((uint32_t)t, m ? row1 : row0, (uint32_t)(jL >> 2), TAG_LTD, seed);
+                          bit = pick(u, jL & 3) <= s_dep[D];
+                        }
+                      }
+                      const uint32_t mm = __ballot_sync(FULL, bit);
+                      if (lane == Ls) s_ev[(c * 2 + m) * nthr + tid] = mm;
+                    }
+                  }
+                }
+              }
+              long long pc2 = prof ? clock64() : 0;
+              // ---- sequential LIF over the block (the only step-to-step dependency)
+              if (!done) {
+                int rlo = rblk0;
+                uint32_t run_prev = 0u;
+#pragma unroll 1
+                for (int b = 0; b < nb; ++b) {
+                  const int kk_b = kb0 + b;
+                  const int t = tbase + kk_b;
+                  const int rhi = (int)(s_offs[kk_b - ka + 1] - wbase);
+                  const uint32_t snap = vmax_lanes<CPT>(run_prev, my_acc[b * nthr]);
+                  const uint32_t a = snap - run_prev;              // this step's SWAR sums
+                  run_prev = snap;
+                  uint32_t cm_b = 0;
+                  int vn[CPT];
+#pragma unroll
+                  for (int c = 0; c < CPT; ++c) {                     // branch-free: the CPT chains overlap
+                    const int S = (int)(Z::LW == 32 ? a : ((a >> (c * Z::LW)) & ((1u << (Z::LW & 31)) - 1u)));
+                    vn[c] = v[c];
+                    const bool crossed = lif.step_t<FIXED>(vn[c], S);
+                    cm_b |= ((cnt[c] == 0 && crossed && (valid >> c & 1u)) ? 1u : 0u) << c;
+                  }
+                  if (cm_b) {                                         // stop here: LIF done, LTD pending
+#pragma unroll
+                    for (int c = 0; c < CPT; ++c) {
+                      cb[c] = cnt[c]; vb[c] = v[c];
+                      v[c] = cnt[c] == 0 ? vn[c] : v[c];
+                      cnt[c] = cnt[c] == 0 ? 0 : cnt[c] - 1;
+                    }
+                    cmask = cm_b; cand = true; done = true; p = kk_b; signal(kk_b);
+                    break;
+                  }
+                  uint32_t on_b = 0;
+                  if (ltd_blk) {
+#pragma unroll
+                    for (int c = 0; c < CPT; ++c)
+                      if ((ltd_blk >> c & 1u) && (t - lpost[c]) < L_dep) on_b |= 1u << c;
+                  }
+                  if (on_b) {                                         // LTD events of step b (rare)
+                    const int lo = rlo - rblk0, nrb = rhi - rlo;
+                    const int nlog_step = nlog;
+                    bool overflow = false;
+                    uint32_t ev_step = 0;
+#pragma unroll 1
+                    for (uint32_t cmm = on_b; cmm && !overflow; cmm &= cmm - 1) {
+                      const int c = __ffs(cmm) - 1;
+                      const unsigned long long e64 = (unsigned long long)s_ev[(c * 2) * nthr + tid] |
+                                                     ((unsigned long long)s_ev[(c * 2 + 1) * nthr + tid] << 32);
+                      unsigned long long em = nrb ? ((e64 >> lo) & ((1ull << nrb) - 1ull)) : 0ull;
+                      const int shc = fsh + c * Z::LW;
+                      while (em) {
+                        const int xr = __ffsll((long long)em) - 1;
+                        em &= em - 1;
+                        if (kk_b > k0 && nlog == logn) { overflow = true; break; }
+                        const int i = s_rows[rlo + xr];
+                        uint32_t* pw = wcol + i * wpr;
+                        const bool applied = ((*pw >> shc) & FMASK) != 0u;
+                        if (applied) {
+                          atomicSub(pw, 1u << shc);
+                          // the later block steps that contain row i were summed with the old code
+                          block_correct<CPT>(s_rows, s_rstep, my_acc, nthr, rhi, rblk1, kb0 - ka, b, nb, i,
+                                             0u - (1u << (c * Z::LW)));
+                        }
+                        ++ev_step;
+                        if (kk_b > k0) s_log[nlog++ * nthr + tid] = log_entry(kk_b - k0, c, applied, i);
+                      }
+                    }
+                    if (overflow) {                               // undo step b entirely; stop before it
+                      while (nlog > nlog_step) {
+                        const uint32_t e = s_log[(nlog - 1) * nthr + tid];
+                        const int i = (int)(e & 0x1FFFu), c = (int)((e >> 14) & 3u);
+                        if (e & 0x2000u) {
+                          atomicAdd(wcol + i * wpr, 1u << (fsh + c * Z::LW));
+                          block_correct<CPT>(s_rows, s_rstep, my_acc, nthr, rhi, rblk1, kb0 - ka, b, nb, i,
+                                             1u << (c * Z::LW));
+                        }
+                        --nlog;
+                      }
+                      hz = true; done = true; p = kk_b; ++eng_hz;     // v / cnt of step b were not committed
+                      signal(kk_b - 1);
+                      break;
+                    }
+                    ltd_events += ev_step;
+                    ltd_trials += (uint32_t)__popc(on_b) * (uint32_t)nrb;
+                  }
+#pragma unroll
+                  for (int c = 0; c < CPT; ++c) {                     // commit step b
+                    v[c] = cnt[c] == 0 ? vn[c] : v[c];
+                    cnt[c] = cnt[c] == 0 ? 0 : cnt[c] - 1;
+                  }
+                  if (kk_b == k0) {
+#pragma unroll
+                    for (int c = 0; c < CPT; ++c) { v1[c] = v[c]; cnt1[c] = cnt[c]; }
+                  }
+                  rlo = rhi;
+                }
+              }
+              if (prof) {
+                const long long pc3 = clock64();
+                prof_int += pc1 - pc0; prof_ltd += pc2 - pc1; prof_seq += pc3 - pc2; prof_blk += nb;
+              }
+              kk = kb0 + nb;
+              r0 = rblk1;
+              continue;
+            }
+          }
+          // ======== general path: one step (more than kPadRows active rows)
           const int r1 = (int)(s_offs[kk - ka + 1] - wbase);
           const int t = tbase + kk;
-          bool ltd_on = false;
-          int cb = cnt;
+          uint32_t ltd_on = 0;
           if (!done) {
-            const int S = integrate(wcol, s_rows, r0, r1, wpr, sh, fmask);   // (a2) eq.(3)
-            if (cnt > 0) {
-              --cnt;                                               // (a3) refractory / inhibited: hold v
-            } else {
-              vb = v;
-              if (lif.step_t<FIXED>(v, S)) { cand = true; done = true; p = kk; signal(kk); }   // (a3) eqs.(1)(2)
+            int S[CPT];
+            integrate_swar<BITS, CPT>(wcol, s_rows, r0, r1, wpr, fsh, S);        // (a2) eq.(3)
+#pragma unroll
+            for (int c = 0; c < CPT; ++c) {
+              cb[c] = cnt[c];
+              if (!(valid >> c & 1u)) continue;
+              if (cnt[c] > 0) {
+                --cnt[c];                                         // (a3) refractory / inhibited: hold v
+              } else {
+                vb[c] = v[c];
+                if (lif.step_t<FIXED>(v[c], S[c])) cmask |= 1u << c;   // (a3) eqs.(1)(2)
+              }
             }
-            ltd_on = !done && ltd_col && (t - lpost) < L_dep;
+            if (cmask) { cand = true; done = true; p = kk; signal(kk); }
+            else {
+#pragma unroll
+              for (int c = 0; c < CPT; ++c)
+                if ((ltd_cols >> c & 1u) && (t - lpost[c]) < L_dep) ltd_on |= 1u << c;
+            }
           }
-          // (a5) LTD, eq.(7), exact (R10, R14): cooperative draws, then this lane's events
-          const uint32_t lmask = __ballot_sync(FULL, ltd_on);
-          if (lmask) {
-            const uint32_t thr = ltd_on ? s_dep[t - lpost] : 0u;
+          // (a5) LTD, eq.(7), exact (R10, R14): for every LTD-active (lane, column) pair of the warp,
+          // all 32 lanes draw the Philox blocks of up to 32 active rows at once (one rolled call site
+          // keeps the loop inside the instruction cache); the owning lane applies its events.
+          if (__any_sync(FULL, ltd_on != 0)) {
             const int nlog_step = nlog;
             bool overflow = false;
             uint32_t ev_step = 0;
-            for (int c0 = r0; c0 < r1; c0 += 32) {               // warp-uniform chunks of <= 32 rows
-              const int n = min(32, r1 - c0);
-              const uint32_t row_here = lane < n ? (uint32_t)s_rows[c0 + lane] : 0u;
-              uint32_t mine = 0;
-              for (uint32_t lm = lmask; lm; lm &= lm - 1) {
-                const int L = __ffs(lm) - 1;
-                const int jL = jw + L;
-                const uint32_t thrL = __shfl_sync(FULL, thr, L);
-                bool bit = false;
-                if (lane < n) {
-                  const uint4 u = philox((uint32_t)t, row_here, (uint32_t)(jL >> 2), TAG_LTD, seed);
-                  bit = pick(u, jL & 3) <= thrL;
-                }
-                const uint32_t m = __ballot_sync(FULL, bit);
-                if (lane == L) mine = m;
-              }
-              if (ltd_on && !overflow) {
-                while (mine) {
-                  const int x = __ffs(mine) - 1;
-                  mine &= mine - 1;
-                  if (kk > k0 && nlog == logn) { overflow = true; break; }
-                  const int i = s_rows[c0 + x];
-                  uint32_t* pw = wcol + i * wpr;
-                  const bool applied = ((*pw >> sh) & fmask) != 0u;
-                  if (applied) atomicSub(pw, 1u << sh);
-                  ++ev_step;
-                  if (kk > k0)
-                    s_log[nlog++ * nthr + tid] = ((uint32_t)(kk - k0) << 16) | (applied ? 0x8000u : 0u) | (uint32_t)i;
+#pragma unroll 1
+            for (uint32_t lm = __ballot_sync(FULL, ltd_on != 0); lm; lm &= lm - 1) {
+              const int Ls = __ffs(lm) - 1;
+              const int tidL = warp * 32 + Ls;
+#pragma unroll 1
+              for (uint32_t cm = __shfl_sync(FULL, ltd_on, Ls); cm; cm &= cm - 1) {
+                const int c = __ffs(cm) - 1;
+                const int jlL = (tidL / TPW) * CPW + (tidL % TPW) + TPW * c;
+                const int jL = col0 + jlL;
+                const uint32_t thrL = s_dep[t - s_lpost[jlL]];
+                const int shc = fsh + c * Z::LW;
+#pragma unroll 1
+                for (int c0 = r0; c0 < r1; c0 += 32) {
+                  const int n = min(32, r1 - c0);
+                  bool bit = false;
+                  if (lane < n) {
+                    const uint4 u = philox((uint32_t)t, (uint32_t)s_rows[c0 + lane], (uint32_t)(jL >> 2), TAG_LTD, seed);
+                    bit = pick(u, jL & 3) <= thrL;
+                  }
+                  uint32_t mine = __ballot_sync(FULL, bit);
+                  if (lane == Ls) {
+                    while (mine && !overflow) {
+                      const int x = __ffs(mine) - 1;
+                      mine &= mine - 1;
+                      if (kk > k0 && nlog == logn) { overflow = true; break; }
+                      const int i = s_rows[c0 + x];
+                      uint32_t* pw = wcol + i * wpr;
+                      const bool applied = ((*pw >> shc) & FMASK) != 0u;
+                      if (applied) atomicSub(pw, 1u << shc);
+                      ++ev_step;
+                      if (kk > k0) s_log[nlog++ * nthr + tid] = log_entry(kk - k0, c, applied, i);
+                    }
+                  }
                 }
               }
             }
@@ -418,11 +786,11 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
               if (overflow) {                                      // undo this step entirely; stop before it
                 while (nlog > nlog_step) {
                   const uint32_t e = s_log[(nlog - 1) * nthr + tid];
-                  if (e & 0x8000u) atomicAdd(wcol + (int)(e & 0x7FFFu) * wpr, 1u << sh);
+                  if (e & 0x2000u) atomicAdd(wcol + (int)(e & 0x1FFFu) * wpr, 1u << (fsh + (int)((e >> 14) & 3u) * Z::LW));
                   --nlog;
                 }
-                cnt = cb;
-                if (cb == 0) v = vb;
+#pragma unroll
+                for (int c = 0; c < CPT; ++c) { if (cb[c] == 0) v[c] = vb[c]; cnt[c] = cb[c]; }
                 hz = true;
                 done = true;
                 p = kk;
@@ -430,29 +798,42 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
                 signal(kk - 1);
               } else {
                 ltd_events += ev_step;
-                ltd_trials += (uint32_t)(r1 - r0);
+                ltd_trials += (uint32_t)__popc(ltd_on) * (uint32_t)(r1 - r0);
               }
             }
           }
-          if (!done && kk == k0) { v1 = v; cnt1 = cnt; }
+          if (!done && kk == k0) {
+#pragma unroll
+            for (int c = 0; c < CPT; ++c) { v1[c] = v[c]; cnt1[c] = cnt[c]; }
+          }
           ++kk;
           r0 = r1;
         }
+        if (trace && lane == 0) prof_loop += clock64() - prof_loop0;
         if (!mycol) p = kend;
-        if (mycol) eng_spec += (uint32_t)(p - k0 + (cand ? 1 : 0));
+        if (mycol) eng_spec += (uint32_t)(p - k0 + (cand ? 1 : 0)) * (uint32_t)__popc(valid);
       }
-
       if (trace && lane == 0) atomicMax(s_tmax, globaltimer());
+
       // ---------------------------------------------------------- CTA summary -> cluster exchange
       {
         const uint32_t w1 = ((uint32_t)(0xFFFF - min(p, kend)) << 1) | (hz ? 1u : 0u);
         const uint32_t W1w = __reduce_max_sync(FULL, w1);
         const int Pw = 0xFFFF - (int)(W1w >> 1);
         const bool c_at = cand && p == Pw;
-        const uint32_t kh = c_at ? lif.ord(v) : 0u;
+        uint32_t kh = 0, kl = 0, cc = 0;
+        if (c_at) {
+#pragma unroll
+          for (int c = 0; c < CPT; ++c) {
+            if (!(cmask >> c & 1u)) continue;
+            const uint32_t h = lif.ord(v[c]), l = 0xFFFFFFFFu - (uint32_t)jcol[c];
+            if (h > kh || (h == kh && l > kl)) { kh = h; kl = l; }
+            ++cc;
+          }
+        }
         const uint32_t mh = __reduce_max_sync(FULL, kh);
-        const uint32_t ml = __reduce_max_sync(FULL, (c_at && kh == mh) ? (0xFFFFFFFFu - (uint32_t)j) : 0u);
-        const uint32_t cw = (uint32_t)__popc(__ballot_sync(FULL, c_at));
+        const uint32_t ml = __reduce_max_sync(FULL, (c_at && kh == mh) ? kl : 0u);
+        const uint32_t cw = __reduce_add_sync(FULL, cc);
         if (lane == 0) {
           s_wsum[2 * warp] = ((unsigned long long)W1w << 32) | cw;
           s_wsum[2 * warp + 1] = ((unsigned long long)mh << 32) | ml;
@@ -465,10 +846,10 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         const unsigned long long k = lane < nwarps ? s_wsum[2 * lane + 1] : 0ull;
         const uint32_t W1c = __reduce_max_sync(FULL, (uint32_t)(a >> 32));
         const bool at = lane < nwarps && (uint32_t)(a >> 32) == W1c;
-        const uint32_t cc = __reduce_add_sync(FULL, at ? (uint32_t)a : 0u);
+        const uint32_t ccs = __reduce_add_sync(FULL, at ? (uint32_t)a : 0u);
         const uint32_t kh = __reduce_max_sync(FULL, at ? (uint32_t)(k >> 32) : 0u);
         const uint32_t kl = __reduce_max_sync(FULL, (at && (uint32_t)(k >> 32) == kh) ? (uint32_t)k : 0u);
-        const unsigned long long A = ((unsigned long long)W1c << 32) | cc;
+        const unsigned long long A = ((unsigned long long)W1c << 32) | ccs;
         const unsigned long long K = ((unsigned long long)kh << 32) | kl;
         unsigned long long* slot = s_slots + (size_t)(fp * kMaxCluster + rank) * 2;
         if (cs == 1) {
@@ -477,7 +858,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
           st_cluster_u64(slot, (uint32_t)lane, A);
           st_cluster_u64(slot + 1, (uint32_t)lane, K);
         }
-        if (lane == 0) { s_flag[fp ^ 1] = INT_MAX; s_misc[1] = 0; }
+        if (lane == 0) s_flag[fp ^ 1] = INT_MAX;
       }
       if (cs > 1) { cluster_arrive(); cluster_wait(); } else { __syncthreads(); }   // the one cross-SM exchange
       if (trace && tid == 0) tr3 = globaltimer();
@@ -490,8 +871,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         const unsigned long long A = s_slots[(size_t)(fp * kMaxCluster + r) * 2];
         if ((uint32_t)(A >> 32) == W1) {
           count += (uint32_t)A;
-          const unsigned long long kk = s_slots[(size_t)(fp * kMaxCluster + r) * 2 + 1];
-          K = kk > K ? kk : K;
+          const unsigned long long kx = s_slots[(size_t)(fp * kMaxCluster + r) * 2 + 1];
+          K = kx > K ? kx : K;
         }
       }
       const int P = 0xFFFF - (int)(W1 >> 1);
@@ -501,48 +882,61 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
       const int tP = tbase + P;
 
       // ---------------------------------------------------------- per-thread resolution / rollback
-      // resim(X): state after step k0 + undo of every logged LTD, then replay k0+1..X exactly.
-      auto count_trials = [&](int from, int to) -> uint32_t {   // LTD trials of steps [from, to)
-        uint32_t n = 0;
-        if (stoch && lpost >= 0)
-          for (int kk = from; kk < to; ++kk)
-            if ((tbase + kk - lpost) < L_dep) n += s_offs[kk - ka + 1] - s_offs[kk - ka];
-        return n;
+      auto count_trials = [&](int c, int from, int to) -> uint32_t {   // LTD trials of column c, steps [from, to)
+        if (!stoch || lpost[c] < 0) return 0u;
+        const int last = lpost[c] + L_dep - 1 - tbase;                 // last step with D < L_dep
+        const int hi = min(to, last + 1);
+        return hi > from ? s_offs[hi - ka] - s_offs[from - ka] : 0u;
       };
-      auto undo_after = [&](int rel_keep) {       // undo logged LTD of steps k0+rel > k0+rel_keep
+      auto undo_after = [&](int rel_keep) {       // undo logged LTD of steps k0 + rel > k0 + rel_keep
         while (nlog > 0) {
           const uint32_t e = s_log[(nlog - 1) * nthr + tid];
           if ((int)(e >> 16) <= rel_keep) break;
-          if (e & 0x8000u) atomicAdd(wcol + (int)(e & 0x7FFFu) * wpr, 1u << sh);
+          if (e & 0x2000u) atomicAdd(wcol + (int)(e & 0x1FFFu) * wpr, 1u << (fsh + (int)((e >> 14) & 3u) * Z::LW));
           --ltd_events;
           --nlog;
           ++eng_undo;
         }
       };
-      auto resim = [&](int X) {
+      // per-lane LTD of all this thread's LTD-active columns at step kk (commit / re-simulation paths)
+      auto ltd_step = [&](int kk) {
+        const int t = tbase + kk;
+        const int r0 = (int)(s_offs[kk - ka] - wbase), r1 = (int)(s_offs[kk - ka + 1] - wbase);
+#pragma unroll
+        for (int c = 0; c < CPT; ++c) {
+          if (!stoch || !(valid >> c & 1u) || lpost[c] < 0 || (t - lpost[c]) >= L_dep) continue;
+          const uint32_t thr = s_dep[t - lpost[c]];
+          const int shc = fsh + c * Z::LW;
+          for (int r = r0; r < r1; ++r) {
+            const int i = s_rows[r];
+            const uint4 u = philox((uint32_t)t, (uint32_t)i, (uint32_t)(jcol[c] >> 2), TAG_LTD, seed);
+            if (pick(u, jcol[c] & 3) <= thr) {
+              uint32_t* pw = wcol + i * wpr;
+              if ((*pw >> shc) & FMASK) atomicSub(pw, 1u << shc);
+              ++ltd_events;
+            }
+          }
+          ltd_trials += (uint32_t)(r1 - r0);
+        }
+      };
+      auto resim = [&](int X) {      // state after step k0, undo every logged LTD, replay k0+1 .. X exactly
         ++eng_resim;
         undo_after(0);
-        ltd_trials -= count_trials(k0 + 1, p);
-        v = v1; cnt = cnt1;
+#pragma unroll
+        for (int c = 0; c < CPT; ++c) {
+          ltd_trials -= count_trials(c, k0 + 1, p);
+          v[c] = v1[c]; cnt[c] = cnt1[c];
+        }
         for (int kk = k0 + 1; kk <= X; ++kk) {
           const int r0 = (int)(s_offs[kk - ka] - wbase), r1 = (int)(s_offs[kk - ka + 1] - wbase);
-          const int t = tbase + kk;
-          const int S = integrate(wcol, s_rows, r0, r1, wpr, sh, fmask);
-          if (cnt > 0) --cnt; else lif.step_t<FIXED>(v, S);
-          if (stoch && lpost >= 0 && (t - lpost) < L_dep) {
-            const uint32_t thr = s_dep[t - lpost];
-            for (int c0 = r0; c0 < r1; c0 += 32) {
-              uint32_t m = ltd_draws(s_rows, c0, min(32, r1 - c0), (uint32_t)t, j, thr, seed);
-              while (m) {
-                const int x = __ffs(m) - 1;
-                m &= m - 1;
-                uint32_t* pw = wcol + (int)s_rows[c0 + x] * wpr;
-                if ((*pw >> sh) & fmask) atomicSub(pw, 1u << sh);
-                ++ltd_events;
-              }
-            }
-            ltd_trials += (uint32_t)(r1 - r0);
+          int S[CPT];
+          integrate_swar<BITS, CPT>(wcol, s_rows, r0, r1, wpr, fsh, S);
+#pragma unroll
+          for (int c = 0; c < CPT; ++c) {
+            if (!(valid >> c & 1u)) continue;
+            if (cnt[c] > 0) --cnt[c]; else lif.step_t<FIXED>(v[c], S[c]);
           }
+          ltd_step(kk);
         }
       };
       if (mycol && !at_end) {
@@ -550,79 +944,127 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
           if (p > P) {                                   // ran past t*: rebuild the state after step t*
             if (inh_reset) {
               undo_after(P - k0);
-              ltd_trials -= count_trials(P + 1, p);
-              cnt = max(cnt0 - (P - k0 + 1), 0);        // no crossing in [k0, t*]: cnt only counted down
-              (void)v0;
+#pragma unroll
+              for (int c = 0; c < CPT; ++c) {
+                ltd_trials -= count_trials(c, P + 1, p);
+                cnt[c] = max(cnt0[c] - (P - k0 + 1), 0);  // no crossing in [k0, t*]: cnt only counted down
+              }
             } else {
               resim(P);
             }
           }
         } else {                                         // unknown at P: commit only through P - 1
           if (p == P) {
-            if (cand) v = vb;
+            if (cand) {
+#pragma unroll
+              for (int c = 0; c < CPT; ++c) { if (cb[c] == 0) v[c] = vb[c]; cnt[c] = cb[c]; }
+            }
           } else {
             resim(P - 1);
           }
         }
       }
-      bool spiked = false;
-      uint32_t W = 0xFFFFFFFFu;
+      uint32_t spiked = 0;
       if (event) {
-        if (hard) {
-          W = 0xFFFFFFFFu - (uint32_t)K;
-          if (mycol) {
-            if ((uint32_t)j == W) { v = vreset; cnt = t_ref; spiked = true; }
-            else { cnt = max(cnt, t_inh); if (inh_reset) v = vreset; }
-          }
-          img_spikes += 1;
-        } else {
-          if (mycol) {
-            const bool me = cand && p == P;
-            if (me) { v = vreset; cnt = t_ref; spiked = true; }
-            if (count >= 2u || !me) { cnt = max(cnt, t_inh); if (inh_reset) v = vreset; }
-          }
-          img_spikes += (int)count;
+        const uint32_t W = 0xFFFFFFFFu - (uint32_t)K;
+        const bool at_p = cand && p == P;
+#pragma unroll
+        for (int c = 0; c < CPT; ++c) {
+          if (!(valid >> c & 1u)) continue;
+          bool me;
+          if (hard) me = (uint32_t)jcol[c] == W;
+          else me = at_p && (cmask >> c & 1u);
+          if (me) { v[c] = vreset; cnt[c] = t_ref; spiked |= 1u << c; }
+          if (hard ? !me : (count >= 2u || !me)) { cnt[c] = max(cnt[c], t_inh); if (inh_reset) v[c] = vreset; }
         }
-        // pending LTD at t* of the columns that stopped there (old last_post, R14)
-        if (mycol && cand && p == P && stoch && lpost >= 0 && (tP - lpost) < L_dep) {
+        img_spikes += hard ? 1 : (int)count;
+        // pending LTD at t* of the columns that stopped there (old last_post, R14): warp-cooperative draws
+        if (__any_sync(FULL, mycol && at_p)) {
           const int r0 = (int)(s_offs[P - ka] - wbase), r1 = (int)(s_offs[P - ka + 1] - wbase);
-          const uint32_t thr = s_dep[tP - lpost];
-          for (int c0 = r0; c0 < r1; c0 += 32) {
-            uint32_t m = ltd_draws(s_rows, c0, min(32, r1 - c0), (uint32_t)tP, j, thr, seed);
-            while (m) {
-              const int x = __ffs(m) - 1;
-              m &= m - 1;
-              uint32_t* pw = wcol + (int)s_rows[c0 + x] * wpr;
-              if ((*pw >> sh) & fmask) atomicSub(pw, 1u << sh);
-              ++ltd_events;
+          uint32_t on = 0;
+          if (mycol && at_p) {
+#pragma unroll
+            for (int c = 0; c < CPT; ++c)
+              if (stoch && (valid >> c & 1u) && lpost[c] >= 0 && (tP - lpost[c]) < L_dep) on |= 1u << c;
+          }
+#pragma unroll 1
+          for (uint32_t lm = __ballot_sync(FULL, on != 0); lm; lm &= lm - 1) {
+            const int Ls = __ffs(lm) - 1;
+            const int tidL = warp * 32 + Ls;
+#pragma unroll 1
+            for (uint32_t cm = __shfl_sync(FULL, on, Ls); cm; cm &= cm - 1) {
+              const int c = __ffs(cm) - 1;
+              const int jlL = (tidL / TPW) * CPW + (tidL % TPW) + TPW * c;
+              const int jL = col0 + jlL;
+              const uint32_t thrL = s_dep[tP - s_lpost[jlL]];
+              const int shc = fsh + c * Z::LW;
+#pragma unroll 1
+              for (int c0 = r0; c0 < r1; c0 += 32) {
+                const int n = min(32, r1 - c0);
+                bool bit = false;
+                if (lane < n) {
+                  const uint4 u = philox((uint32_t)tP, (uint32_t)s_rows[c0 + lane], (uint32_t)(jL >> 2), TAG_LTD, seed);
+                  bit = pick(u, jL & 3) <= thrL;
+                }
+                uint32_t mine = __ballot_sync(FULL, bit);
+                if (lane == Ls) {
+                  while (mine) {
+                    const int x = __ffs(mine) - 1;
+                    mine &= mine - 1;
+                    uint32_t* pw = wcol + (int)s_rows[c0 + x] * wpr;
+                    if ((*pw >> shc) & FMASK) atomicSub(pw, 1u << shc);
+                    ++ltd_events;
+                  }
+                }
+              }
+              if (lane == Ls) ltd_trials += (uint32_t)(r1 - r0);
             }
           }
-          ltd_trials += (uint32_t)(r1 - r0);
         }
-        if (rec_out) {
-          const uint32_t bal = __ballot_sync(FULL, spiked);
-          if (lane == 0 && warp < ngrp_cta) d.raster_out[(size_t)P * nwe + g0 + warp] = bal;
+        if (rec_out && spiked) {
+#pragma unroll
+          for (int c = 0; c < CPT; ++c)
+            if (spiked >> c & 1u) atomicOr(&d.raster_out[(size_t)P * nwe + (jcol[c] >> 5)], 1u << (jcol[c] & 31));
         }
-        if (spiked && !hard) { const int pos = atomicAdd(&s_misc[1], 1); s_splist[pos] = (uint16_t)tid; }
       }
       const int k_last = event ? P : (at_end ? kend - 1 : P - 1);
-      __syncthreads();                                                               // S2
       // spike timers of the inputs through the committed step
       for (int kk = k0 + tid; kk <= k_last; kk += nthr) {
         const int r0 = (int)(s_offs[kk - ka] - wbase), r1 = (int)(s_offs[kk - ka + 1] - wbase);
         for (int r = r0; r < r1; ++r) atomicMax(&s_lpre[s_rows[r]], tbase + kk);
       }
-      const bool local_spike = event && (hard ? (W >= (uint32_t)col0 && W < (uint32_t)(col0 + ncols)) : false);
-      __syncthreads();                                                               // S3
-      if (trace && tid == 0 && ep < d.trace_cap) trace[(size_t)ep * 8 + 6] = globaltimer();
-      const int nsp = hard ? (local_spike ? 1 : 0) : (event ? s_misc[1] : 0);
-      if (nsp > 0) {
-        // (a5) LTP eq.(6) / (a6) deterministic arm at t*, rows spread over threads (row words owned)
-        for (int grp = tid; grp < nq4; grp += nthr) {
-          for (int m = 0; m < nsp; ++m) {
-            const int Wl = hard ? (int)(W - (uint32_t)col0) : (int)s_splist[m];
-            const int Wg = col0 + Wl;
-            const int ww = Wl >> lg, wsh = (Wl & ((1 << lg) - 1)) * bits;
+      __syncthreads();                                                               // S2
+      if (trace && tid == 0 && ep < d.trace_cap) {
+        unsigned long long* rec = trace + (size_t)ep * 8;
+        rec[0] = ((unsigned long long)b << 32) | (unsigned)k0;
+        rec[1] = ((unsigned long long)(event ? 1 : (unknown ? 2 : 0)) << 32) | (unsigned)P;
+        rec[2] = tr0; rec[3] = *s_tmax; rec[4] = tr2; rec[5] = tr3; rec[6] = globaltimer(); rec[7] = rec[6];
+      }
+      if (spiked) {
+#pragma unroll
+        for (int c = 0; c < CPT; ++c)
+          if (spiked >> c & 1u) { lpost[c] = tP; s_lpost[jcol[c] - col0] = tP; }
+      }
+      pend_mask = spiked;
+      pend_t = tP;
+      k0 = k_last + 1;
+      ++ep;
+      ++eng_epochs;
+    }  // epochs
+
+    // the last event's LTP of this image (if any) before the state is written back
+    if (__any_sync(FULL, pend_mask != 0)) {
+      const int tP = pend_t;
+      for (uint32_t wm = __ballot_sync(FULL, pend_mask != 0); wm; wm &= wm - 1) {
+        const int Lsrc = __ffs(wm) - 1;
+        const uint32_t pm = __shfl_sync(FULL, pend_mask, Lsrc);
+        for (uint32_t cm = pm; cm; cm &= cm - 1) {
+          const int c = __ffs(cm) - 1;
+          const int tidL = warp * 32 + Lsrc;
+          const int jl = (tidL / TPW) * CPW + (tidL % TPW) + TPW * c;
+          const int Wg = col0 + jl;
+          const int ww = jl / CPW, wsh = (jl % CPW) * BITS;
+          for (int grp = lane; grp < nq4; grp += 32) {
             const uint4 u = philox((uint32_t)tP, (uint32_t)Wg, (uint32_t)grp, stoch ? TAG_LTP : TAG_ROUND, seed);
 #pragma unroll
             for (int r = 0; r < 4; ++r) {
@@ -637,45 +1079,35 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
                 ++ltp_trials;
                 if (pick(u, r) <= s_pot[D]) {
                   ++ltp_events;
-                  const uint32_t word = *pw;
-                  if (((word >> wsh) & fmask) < (uint32_t)qmax) *pw = word + (1u << wsh);
+                  if (((*pw >> wsh) & FMASK) < (uint32_t)qmax) atomicAdd(pw, 1u << wsh);
                 }
               } else {
-                const uint32_t word = *pw;
-                const int q0 = (int)((word >> wsh) & fmask);
+                const int q0 = (int)((*pw >> wsh) & FMASK);
                 const bool pot = lpi >= 0 && (tP - lpi) <= t_ltp;
                 const int base = pot ? s_dbp[q0] : s_dbd[q0];
                 const uint32_t thr = pot ? s_dtp[q0] : s_dtd[q0];
                 const int dq = base + (pick(u, r) < thr ? 1 : 0);
                 int q1 = pot ? q0 + dq : q0 - dq;
                 q1 = q1 < 0 ? 0 : (q1 > qmax ? qmax : q1);
-                *pw = (word & ~(fmask << wsh)) | ((uint32_t)q1 << wsh);
+                if (q1 != q0) atomicAdd(pw, (uint32_t)(q1 - q0) << wsh);
                 if (pot) { ++ltp_trials; if (dq > 0) ++ltp_events; }
                 else     { ++ltd_trials; if (dq > 0) ++ltd_events; }
               }
             }
           }
         }
-        __syncthreads();                                                             // S4
       }
-      if (spiked) lpost = tP;
-      if (trace && tid == 0 && ep < d.trace_cap) {
-        unsigned long long* rec = trace + (size_t)ep * 8;
-        rec[0] = ((unsigned long long)b << 32) | (unsigned)k0;
-        rec[1] = ((unsigned long long)(event ? 1 : (unknown ? 2 : 0)) << 32) | (unsigned)P;
-        rec[2] = tr0; rec[3] = *s_tmax; rec[4] = tr2; rec[5] = tr3; rec[7] = globaltimer();
-      }
-      k0 = k_last + 1;
-      ++ep;
-      ++eng_epochs;
-    }  // epochs
-
+      pend_mask = 0;
+    }
     if (rank == 0 && tid == 0) {
       post_sum += (unsigned long long)img_spikes;
       if (d.spike_counts) d.spike_counts[b] = img_spikes;
     }
     if (last_img) {
-      if (mycol) { d.v[j] = v; d.cnt[j] = cnt; d.last_post[j] = lpost; }
+#pragma unroll
+      for (int c = 0; c < CPT; ++c)
+        if (valid >> c & 1u) { d.v[jcol[c]] = v[c]; d.cnt[jcol[c]] = cnt[c]; d.last_post[jcol[c]] = lpost[c]; }
+      __syncthreads();
       if (rank == 0) for (int i = tid; i < n_in; i += nthr) d.last_pre[i] = s_lpre[i];
     }
     __syncthreads();
@@ -687,7 +1119,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
     for (int k = tid; k < slice_words / 4; k += nthr) dst[k] = src[k];
   }
   {
-    unsigned long long a = ltd_trials, b2 = ltd_events, c = ltp_trials, e = ltp_events;  // widen before the warp sum
+    unsigned long long a = ltd_trials, b2 = ltd_events, c = ltp_trials, e = ltp_events;
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
       a += __shfl_xor_sync(FULL, a, o); b2 += __shfl_xor_sync(FULL, b2, o);
@@ -719,6 +1151,28 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
       if (u2) atomicAdd(&d.stats[12], u2);
     }
   }
+  // slowest warp of the CTA (by whole speculation-loop cycles) reports its phase profile
+  if (trace) {
+    __syncthreads();
+    unsigned long long* s_pm = reinterpret_cast<unsigned long long*>(s_misc + 8);
+    if (tid == 0) *s_pm = 0ull;
+    __syncthreads();
+    if (lane == 0) atomicMax(s_pm, ((unsigned long long)prof_loop << 8) | (unsigned)warp);
+    __syncthreads();
+    if (lane == 0 && (int)(*s_pm & 0xFFull) == warp && d.trace_cap > 0) {
+      unsigned long long* rec = trace + (size_t)(d.trace_cap - 1) * 8;
+      rec[0] = (0xFFFFFFFFull << 32) | (unsigned)warp; rec[1] = (unsigned long long)prof_int;
+      rec[2] = (unsigned long long)prof_ltd; rec[3] = (unsigned long long)prof_seq; rec[4] = (unsigned long long)prof_blk;
+      rec[5] = (unsigned long long)prof_loop; rec[6] = (unsigned long long)(clock64() - prof_clk0);
+      rec[7] = globaltimer() - prof_ns0;
+    }
+  }
+  if (false) {
+    unsigned long long* rec = trace + (size_t)(d.trace_cap - 1) * 8;
+    rec[0] = 0xFFFFFFFFull << 32; rec[1] = (unsigned long long)prof_int; rec[2] = (unsigned long long)prof_ltd;
+    rec[3] = (unsigned long long)prof_seq; rec[4] = (unsigned long long)prof_blk; rec[5] = (unsigned long long)prof_loop;
+    rec[6] = (unsigned long long)(clock64() - prof_clk0); rec[7] = globaltimer() - prof_ns0;
+  }
   if (cs > 1) { cluster_arrive(); cluster_wait(); }
 }
 
@@ -740,17 +1194,17 @@ cudaError_t launch_counts_from_raster(const uint32_t* raster, int n_in, int T, u
 }
 
 cudaError_t launch_compact(const uint32_t* words, const uint32_t* counts, int n_in, int T, int n_images,
-                           long long rows_stride, uint32_t* offs, uint16_t* rows, cudaStream_t s) {
+                           long long rows_stride, uint32_t* offs, uint16_t* rows, uint16_t* rows16, cudaStream_t s) {
   if (n_images <= 0) return cudaSuccess;
-  compact_kernel<<<(unsigned)n_images, 256, 0, s>>>(words, counts, n_in, T, rows_stride, offs, rows);
+  compact_kernel<<<(unsigned)n_images, 256, 0, s>>>(words, counts, n_in, T, rows_stride, offs, rows, rows16);
   return cudaGetLastError();
 }
 
-template <bool FIXED>
-static cudaError_t configure_event(size_t smem, int cs) {
-  cudaError_t e = cudaFuncSetAttribute(present_event_kernel<FIXED>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+template <int BITS, int CPT, bool FIXED>
+static cudaError_t configure_event_t(size_t smem, int cs) {
+  cudaError_t e = cudaFuncSetAttribute(present_event_kernel<BITS, CPT, FIXED>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  if (cs > 8) e = cudaFuncSetAttribute(present_event_kernel<FIXED>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+  if (cs > 8) e = cudaFuncSetAttribute(present_event_kernel<BITS, CPT, FIXED>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
   return e;
 }
 
@@ -772,37 +1226,55 @@ static void fill_cfg_ev(cudaLaunchConfig_t& cfg, cudaLaunchAttribute* attr, int 
   }
 }
 
-cudaError_t query_max_clusters_event(int cs, int nthr, size_t smem, int* out) {
-  cudaError_t e = configure_event<false>(smem, cs);
-  if (e == cudaSuccess) e = configure_event<true>(smem, cs);
-  if (e != cudaSuccess) return e;
-  if (cs == 1) return cudaOccupancyMaxActiveBlocksPerMultiprocessor(out, present_event_kernel<false>, nthr, smem);
-  cudaLaunchConfig_t cfg;
-  cudaLaunchAttribute attr[1];
-  fill_cfg_ev(cfg, attr, 1, cs, nthr, smem, 0);
-  return cudaOccupancyMaxActiveClusters(out, present_event_kernel<false>, &cfg);
-}
-
-cudaError_t launch_present_event(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, cudaStream_t s) {
-  const bool fixed = (lp.descs ? 0 : lp.single.membrane_mode) == 1;   // ensembles: see launch_present_event_mode
-  cudaError_t e = fixed ? configure_event<true>(smem, cs) : configure_event<false>(smem, cs);
+template <int BITS, int CPT, bool FIXED>
+static cudaError_t launch_t(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, cudaStream_t s,
+                            int* occupancy_out) {
+  cudaError_t e = configure_event_t<BITS, CPT, FIXED>(smem, cs);
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg;
   cudaLaunchAttribute attr[1];
   fill_cfg_ev(cfg, attr, n_nets, cs, nthr, smem, s);
-  return fixed ? cudaLaunchKernelEx(&cfg, present_event_kernel<true>, lp)
-               : cudaLaunchKernelEx(&cfg, present_event_kernel<false>, lp);
+  if (occupancy_out) {
+    if (cs == 1) return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occupancy_out, present_event_kernel<BITS, CPT, FIXED>, nthr, smem);
+    return cudaOccupancyMaxActiveClusters(occupancy_out, present_event_kernel<BITS, CPT, FIXED>, &cfg);
+  }
+  return cudaLaunchKernelEx(&cfg, present_event_kernel<BITS, CPT, FIXED>, lp);
 }
 
-cudaError_t launch_present_event_mode(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, int fixed,
-                                      cudaStream_t s) {
-  cudaError_t e = fixed ? configure_event<true>(smem, cs) : configure_event<false>(smem, cs);
-  if (e != cudaSuccess) return e;
-  cudaLaunchConfig_t cfg;
-  cudaLaunchAttribute attr[1];
-  fill_cfg_ev(cfg, attr, n_nets, cs, nthr, smem, s);
-  return fixed ? cudaLaunchKernelEx(&cfg, present_event_kernel<true>, lp)
-               : cudaLaunchKernelEx(&cfg, present_event_kernel<false>, lp);
+template <int BITS, int CPT>
+static cudaError_t dispatch_f(int fixed, const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem,
+                              cudaStream_t s, int* occ) {
+  return fixed ? launch_t<BITS, CPT, true>(lp, n_nets, cs, nthr, smem, s, occ)
+               : launch_t<BITS, CPT, false>(lp, n_nets, cs, nthr, smem, s, occ);
+}
+
+static cudaError_t dispatch(int bits, int cpt, int fixed, const LaunchParams& lp, int n_nets, int cs, int nthr,
+                            size_t smem, cudaStream_t s, int* occ) {
+  if (bits == 2) {
+    if (cpt == 4) return dispatch_f<2, 4>(fixed, lp, n_nets, cs, nthr, smem, s, occ);
+    if (cpt == 1) return dispatch_f<2, 1>(fixed, lp, n_nets, cs, nthr, smem, s, occ);
+    return dispatch_f<2, 2>(fixed, lp, n_nets, cs, nthr, smem, s, occ);
+  }
+  if (bits == 4) {
+    if (cpt == 1) return dispatch_f<4, 1>(fixed, lp, n_nets, cs, nthr, smem, s, occ);
+    return dispatch_f<4, 2>(fixed, lp, n_nets, cs, nthr, smem, s, occ);
+  }
+  return dispatch_f<8, 1>(fixed, lp, n_nets, cs, nthr, smem, s, occ);
+}
+
+int event_threads(int max_groups, int bits, int cpt) {
+  const int t = max_groups * 32 / cpt;            // CPW/CPT threads per packed word
+  return ((t + 31) / 32) * 32;
+}
+
+cudaError_t query_max_clusters_event(int bits, int cpt, int fixed, int cs, int nthr, size_t smem, int* out) {
+  LaunchParams lp{};
+  return dispatch(bits, cpt, fixed, lp, 1, cs, nthr, smem, 0, out);
+}
+
+cudaError_t launch_present_event_mode(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, int bits,
+                                      int cpt, int fixed, cudaStream_t s) {
+  return dispatch(bits, cpt, fixed, lp, n_nets, cs, nthr, smem, s, nullptr);
 }
 
 }  // namespace snn

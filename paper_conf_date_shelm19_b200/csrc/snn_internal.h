@@ -10,6 +10,7 @@ constexpr int kMaxCluster = 16;     // non-portable cluster size limit on B200
 constexpr int kMaxThreads = 1024;   // one column per thread -> <= 32 groups of 32 columns per CTA
 constexpr int kLutMax = 4096;       // R19
 constexpr int kNever = -1;
+constexpr int kPadRows = 16;        // fixed-width per-step row slots used by the event engine's block integration
 
 enum : uint32_t { TAG_ENC = 1, TAG_LTD = 2, TAG_LTP = 3, TAG_ROUND = 4, TAG_INIT = 5 };
 enum : int { FLAG_RASTER_INPUT = 1, FLAG_KEEP_STATE = 2, FLAG_RECORD_INPUT = 4, FLAG_ASYNC = 8, FLAG_FLOOR = 16 };
@@ -21,6 +22,7 @@ struct NetDesc {
   int cs;          // CTAs per network (= cluster size)
   int ngroups;     // ceil(n_exc / 32): columns are sliced across CTAs in groups of 32
   int wpr;         // u32 words per weight row of one CTA slice (max_groups * bits)
+  int slice_words; // u32 words of one CTA slice: (n_in + 1) rows (row n_in is all zero), rounded to 4
   int nwi, nwe;    // u32 words per input / output raster row
   // LIF
   int membrane_mode;
@@ -55,6 +57,7 @@ struct NetDesc {
   // event engine: per-image active-row lists from the encoder pre-pass
   const uint32_t* ev_offs;             // [n_images][T+1] prefix offsets into ev_rows
   const uint16_t* ev_rows;             // [n_images][rows_stride] active input rows, step-major, ascending
+  const uint16_t* ev_rows16;           // [n_images][T][kPadRows] first kPadRows rows of each step, padded with n_in
   long long rows_stride;
   int rows_cap, offs_cap, logn;        // on-chip window of the lists, per-thread LTD undo-log entries
   // optional per-epoch trace: [cs][trace_cap][8] u64 (%globaltimer ns)
@@ -70,19 +73,20 @@ struct LaunchParams {
 // kernels.cu entry points (host side)
 cudaError_t launch_present(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, cudaStream_t s);
 // event engine (snn_event.cu)
-constexpr int kEvMaxThreads = 512;
+constexpr int kEvMaxThreads = 256;   // 255 registers per thread: the speculation loop keeps all its state in registers
 constexpr int kEvMaxT = 32767;
 size_t event_smem_bytes(int n_in, int slice_words, int L_pot, int L_dep, int q_max, int nthr, int rows_cap,
                         int offs_cap, int logn);
-cudaError_t query_max_clusters_event(int cs, int nthr, size_t smem, int* out);
+inline int slice_words_for(int n_in, int wpr) { return (((n_in + 1) * wpr) + 3) & ~3; }
+cudaError_t query_max_clusters_event(int bits, int cpt, int fixed, int cs, int nthr, size_t smem, int* out);
+int event_threads(int max_groups, int bits, int cpt);
 cudaError_t launch_encode(const uint8_t* images, const unsigned long long* thr_enc, const unsigned long long* seeds,
                           int n_in, int T, int n_images, int t0, uint32_t* words, uint32_t* counts, cudaStream_t s);
 cudaError_t launch_counts_from_raster(const uint32_t* raster, int n_in, int T, uint32_t* counts, cudaStream_t s);
 cudaError_t launch_compact(const uint32_t* words, const uint32_t* counts, int n_in, int T, int n_images,
-                           long long rows_stride, uint32_t* offs, uint16_t* rows, cudaStream_t s);
-cudaError_t launch_present_event(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, cudaStream_t s);
-cudaError_t launch_present_event_mode(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, int fixed,
-                                      cudaStream_t s);
+                           long long rows_stride, uint32_t* offs, uint16_t* rows, uint16_t* rows16, cudaStream_t s);
+cudaError_t launch_present_event_mode(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, int bits,
+                                      int cpt, int fixed, cudaStream_t s);
 cudaError_t configure_present_kernel(size_t smem, int cs);
 cudaError_t query_max_clusters(int cs, int nthr, size_t smem, int* out);
 cudaError_t launch_init_weights(const NetDesc& d, uint64_t init_seed, cudaStream_t s);

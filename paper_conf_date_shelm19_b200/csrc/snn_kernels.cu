@@ -51,9 +51,7 @@ size_t present_smem_bytes(int n_in, int slice_words, int L_pot, int L_dep, int q
   return smem_layout(n_in, slice_words, L_pot, L_dep, q_max, nthr).total;
 }
 
-__device__ __forceinline__ int slice_words_of(const NetDesc& d) {
-  return ((d.n_in * d.wpr) + 3) & ~3;
-}
+__device__ __forceinline__ int slice_words_of(const NetDesc& d) { return d.slice_words; }
 
 // ------------------------------------------------------------------ the persistent step kernel
 __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_constant__ LaunchParams lp) {
@@ -543,17 +541,17 @@ __global__ void check_codes_kernel(const uint8_t* __restrict__ codes, size_t n, 
 static unsigned grid_for(size_t n, int bs) { return (unsigned)((n + bs - 1) / bs); }
 
 cudaError_t launch_init_weights(const NetDesc& d, uint64_t init_seed, cudaStream_t s) {
-  const size_t n = (size_t)d.cs * (((d.n_in * d.wpr) + 3) & ~3);
+  const size_t n = (size_t)d.cs * d.slice_words;
   init_weights_kernel<<<grid_for(n, 256), 256, 0, s>>>(d, init_seed);
   return cudaGetLastError();
 }
 cudaError_t launch_pack_weights(const NetDesc& d, const uint8_t* codes, cudaStream_t s) {
-  const size_t n = (size_t)d.cs * (((d.n_in * d.wpr) + 3) & ~3);
+  const size_t n = (size_t)d.cs * d.slice_words;
   pack_weights_kernel<<<grid_for(n, 256), 256, 0, s>>>(d, codes);
   return cudaGetLastError();
 }
 cudaError_t launch_unpack_weights(const NetDesc& d, uint8_t* codes, cudaStream_t s) {
-  const size_t n = (size_t)d.cs * (((d.n_in * d.wpr) + 3) & ~3);
+  const size_t n = (size_t)d.cs * d.slice_words;
   unpack_weights_kernel<<<grid_for(n, 256), 256, 0, s>>>(d, codes);
   return cudaGetLastError();
 }

@@ -172,9 +172,10 @@ class Network:
             pass
 
     def info(self) -> dict:
-        a = (ctypes.c_int64 * 8)()
+        a = (ctypes.c_int64 * 12)()
         _check(lib().snn_get_info(self._h, a), "snn_get_info")
-        keys = ["cluster_size", "threads", "smem_bytes", "words_per_row", "q_max", "L_pot", "L_dep", "launches"]
+        keys = ["cluster_size", "threads", "smem_bytes", "words_per_row", "q_max", "L_pot", "L_dep", "launches",
+                "engine", "cols_per_thread", "row_window", "log_depth"]
         return dict(zip(keys, [int(x) for x in a]))
 
     def set_stream(self, stream_ptr: int):

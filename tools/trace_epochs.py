@@ -21,9 +21,18 @@ def main():
     ap.add_argument("--T", type=int, default=350)
     ap.add_argument("--cluster-size", type=int, default=0)
     ap.add_argument("--kind", default="fashion")
+    ap.add_argument("--gamma-pot", type=float, default=None)
+    ap.add_argument("--gamma-dep", type=float, default=None)
+    ap.add_argument("--membrane", type=int, default=0)
     a = ap.parse_args()
     pre = {2: "2b", 4: "4b", 8: "8b"}[a.bits]
-    net = P.Network(784, a.n_exc, a.bits, P.preset(pre, cluster_size=a.cluster_size))
+    prm = P.preset(pre, cluster_size=a.cluster_size, membrane_mode=a.membrane)
+    if a.gamma_pot is not None:
+        prm.gamma_pot = a.gamma_pot
+    if a.gamma_dep is not None:
+        prm.gamma_dep = a.gamma_dep
+    net = P.Network(784, a.n_exc, a.bits, prm)
+    print("info", net.info())
     imgs = synthdata.images(a.images + 2, a.kind)
     seeds = synthdata.seeds(a.images + 2, 1)
     net.present_batch(imgs[:2], a.T, seeds[:2])            # warm-up
@@ -31,6 +40,14 @@ def main():
     net.reset_stats()
     net.present_batch(imgs[2:], a.T, seeds[2:])
     tr = net.trace().astype(np.int64)                       # (cs, E, 8)
+    prof = tr[:, -1, :].copy()
+    print("prof raw", prof[:2].tolist())
+    tr = tr[:, :-1, :]
+    for r in range(prof.shape[0]):
+        if (prof[r, 0] >> 32) & 0xFFFFFFFF == 0xFFFFFFFF and prof[r, 4] > 0:
+            nbk = prof[r, 4]
+            print(f"CTA {r} slowest warp {prof[r,0] & 0xFFFFFFFF} cycles/step: integrate {prof[r,1]/nbk:.0f}  ltd {prof[r,2]/nbk:.0f}  seq {prof[r,3]/nbk:.0f}"
+                  f"  whole-loop {prof[r,5]/nbk:.0f}  (block steps {nbk})  SM clock {prof[r,6]/max(1,prof[r,7]):.3f} GHz")
     st = net.stats()
     cs, E, _ = tr.shape
     valid = tr[0, :, 7] > 0
@@ -52,6 +69,7 @@ def main():
     commit = comm.max(axis=0) - exch.min(axis=0)
     ltp = end.max(axis=0) - comm.min(axis=0)
     adv = np.diff(np.append(k0, k0[-1]))
+    print("stats", [int(x) for x in st[:13]])
     print(f"cluster {cs}  epochs {E}  images {a.images}  epochs/image {E / a.images:.1f}  post spikes {int(st[1])}")
     print(f"per-epoch mean ns: total {tot.mean():.0f}  speculation {spec.mean():.0f} (spread across CTAs {spread.mean():.0f})"
           f"  summary->exchanged {wait.mean():.0f}  commit {commit.mean():.0f}  LTP+tail {ltp.mean():.0f}")
