@@ -160,12 +160,19 @@ def main():
     import paper_conf_date_shelm19_b200 as P
 
     ws, rank, local = _dist_env()
-    torch.cuda.set_device(local)
+    ndev = torch.cuda.device_count()
+    local_dev = local % max(1, ndev)
+    torch.cuda.set_device(local_dev)
     dist = None
+    coll_dev = torch.device("cuda", local_dev)
     if ws > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    dev = torch.device("cuda", local)
+        if ndev >= ws:      # one process per GPU (the driver's layout): NCCL
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_dev))
+        else:               # functional check with ranks sharing a GPU: gloo on CPU tensors
+            dist.init_process_group("gloo")
+            coll_dev = torch.device("cpu")
+    dev = torch.device("cuda", local_dev)
     # a dedicated (non-default) stream: the handle launches on it and the CUDA events are recorded on it
     stream = torch.cuda.Stream(dev)
     torch.cuda.set_stream(stream)
@@ -221,10 +228,10 @@ def main():
     events = int(stats[0]) * N_EXC
     # max over ranks of the device time
     if dist:
-        t = torch.tensor([dev_s], device=dev, dtype=torch.float64)
+        t = torch.tensor([dev_s], device=coll_dev, dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         dev_s = float(t.item())
-        tot = torch.tensor([images, events], device=dev, dtype=torch.float64)
+        tot = torch.tensor([images, events], device=coll_dev, dtype=torch.float64)
         dist.all_reduce(tot, op=dist.ReduceOp.SUM)
         images, events = int(tot[0].item()), int(tot[1].item())
     value = images / dev_s
@@ -265,7 +272,7 @@ def main():
     torch.cuda.synchronize()
     e2e_s = time.perf_counter() - t0
     if dist:
-        t = torch.tensor([e2e_s], device=dev, dtype=torch.float64)
+        t = torch.tensor([e2e_s], device=coll_dev, dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_s = float(t.item())
     e2e = {"value": images / e2e_s, "unit": "images/s", "h2d_bytes_per_step": B * (N_IN + 8),
