@@ -214,7 +214,6 @@ template <int CPT>
 __device__ __forceinline__ void block_correct(const uint16_t* __restrict__ rows, const uint16_t* __restrict__ rstep,
                                               uint32_t* my_acc, int nthr, int rlo, int rhi, int sbase, int b, int nb,
                                               int i, uint32_t delta) {
-  // first later step containing row i (one pass, 8 independent loads per group)
   int first = nb;
   for (int r = rlo; r < rhi && first == nb; r += 8) {
     uint32_t rv[8];
@@ -222,7 +221,7 @@ __device__ __forceinline__ void block_correct(const uint16_t* __restrict__ rows,
     for (int x = 0; x < 8; ++x) rv[x] = r + x < rhi ? (uint32_t)rows[r + x] : 0xFFFFFFFFu;
 #pragma unroll
     for (int x = 0; x < 8; ++x)
-      if (rv[x] == (uint32_t)i && first == nb) first = (int)rstep[r + x] - sbase;
+      if (rv[x] == (uint32_t)i && first == nb) first = (int)(rstep[r + x] & 0x7FFFu) - sbase;
   }
   if (first >= nb) return;
   // each occurrence of i at step s2 lowers the running sums of every step >= s2: walk the later rows once
@@ -230,7 +229,7 @@ __device__ __forceinline__ void block_correct(const uint16_t* __restrict__ rows,
   int rr = rlo;
   for (int b2 = b + 1; b2 < nb; ++b2) {
     bool nonempty = false;
-    while (rr < rhi && (int)rstep[rr] - sbase == b2) {
+    while (rr < rhi && (int)(rstep[rr] & 0x7FFFu) - sbase == b2) {
       if ((uint32_t)rows[rr] == (uint32_t)i) cum += delta;
       nonempty = true;
       ++rr;
@@ -250,7 +249,7 @@ __host__ __device__ inline EvLayout ev_layout(int n_in, int slice_words, int L_p
   L.slots = o;  o = align16(o + 2 * kMaxCluster * 2 * 8);   // [parity][rank][2] u64
   L.wsum = o;   o = align16(o + 32 * 2 * 8);                // per warp: summary, key
   L.flags = o;  o = align16(o + 4 * 4);                     // early-stop flag per epoch parity
-  L.misc = o;   o = align16(o + 16 * 8);
+  L.misc = o;   o = align16(o + 16 * 8 + (size_t)nthr * 4 * 4);   // header + local spiker list
   L.w = o;      o = align16(o + (size_t)slice_words * 4);
   L.pot = o;    o = align16(o + (size_t)(L_pot > 0 ? L_pot : 1) * 4);
   L.dep = o;    o = align16(o + (size_t)(L_dep > 0 ? L_dep : 1) * 4);
@@ -388,8 +387,6 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
   const long long prof_clk0 = clock64();
   const unsigned long long prof_ns0 = globaltimer();
   // pending LTP of the previous epoch (owner warps run it while the others start speculating)
-  int pend_t = -1;
-  uint32_t pend_mask = 0;                                      // bit c: this thread's column c spiked
 
   for (int b = 0; b < n_images; ++b) {
     const unsigned long long seed = d.seeds[b];
@@ -413,58 +410,6 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
     __syncthreads();
 
     while (k0 < T) {
-      // ---------------------------------------------------------- (a5)/(a6) pending LTP of the last event
-      // Run by the warps that own a spiking column; the other warps go straight to speculation.
-      // Updates are atomic (other columns' LTD shares the words), and column W's own thread is in
-      // this warp, so it cannot speculate on W before W's potentiation is complete.
-      if (__any_sync(FULL, pend_mask != 0)) {
-        const int tP = pend_t;
-        for (uint32_t wm = __ballot_sync(FULL, pend_mask != 0); wm; wm &= wm - 1) {
-          const int Lsrc = __ffs(wm) - 1;
-          const uint32_t pm = __shfl_sync(FULL, pend_mask, Lsrc);
-          for (uint32_t cm = pm; cm; cm &= cm - 1) {
-            const int c = __ffs(cm) - 1;
-            const int tidL = warp * 32 + Lsrc;
-            const int jl = (tidL / TPW) * CPW + (tidL % TPW) + TPW * c;
-            const int Wg = col0 + jl;
-            const int ww = jl / CPW, wsh = (jl % CPW) * BITS;
-            for (int grp = lane; grp < nq4; grp += 32) {
-              const uint4 u = philox((uint32_t)tP, (uint32_t)Wg, (uint32_t)grp, stoch ? TAG_LTP : TAG_ROUND, seed);
-#pragma unroll
-              for (int r = 0; r < 4; ++r) {
-                const int i = 4 * grp + r;
-                if (i >= n_in) break;
-                const int lpi = s_lpre[i];
-                uint32_t* pw = s_w + i * wpr + ww;
-                if (stoch) {
-                  if (lpi < 0) continue;
-                  const int D = tP - lpi;
-                  if (D >= L_pot) continue;
-                  ++ltp_trials;
-                  if (pick(u, r) <= s_pot[D]) {                // eq.(6), R10: Dt = D >= 0
-                    ++ltp_events;
-                    if (((*pw >> wsh) & FMASK) < (uint32_t)qmax) atomicAdd(pw, 1u << wsh);
-                  }
-                } else {                                       // eqs.(4)(5)(8), R16/R17
-                  const int q0 = (int)((*pw >> wsh) & FMASK);
-                  const bool pot = lpi >= 0 && (tP - lpi) <= t_ltp;
-                  const int base = pot ? s_dbp[q0] : s_dbd[q0];
-                  const uint32_t thr = pot ? s_dtp[q0] : s_dtd[q0];
-                  const int dq = base + (pick(u, r) < thr ? 1 : 0);
-                  int q1 = pot ? q0 + dq : q0 - dq;
-                  q1 = q1 < 0 ? 0 : (q1 > qmax ? qmax : q1);
-                  if (q1 != q0) atomicAdd(pw, (uint32_t)(q1 - q0) << wsh);
-                  if (pot) { ++ltp_trials; if (dq > 0) ++ltp_events; }
-                  else     { ++ltd_trials; if (dq > 0) ++ltd_events; }
-                }
-              }
-            }
-          }
-        }
-        pend_mask = 0;
-        __syncwarp();
-      }
-
       // ---------------------------------------------------------- stage the active-row window
       if (k0 >= kb) {
         __syncthreads();
@@ -487,10 +432,20 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         for (int x = tid; x < nsteps; x += nthr)
           for (uint32_t r = s_offs[x] - wbase; r < s_offs[x + 1] - wbase; ++r) s_rstep[r] = (uint16_t)x;
         __syncthreads();
+        // bit 15 of s_rstep[r]: the same input occurs again within the next 64 rows (a block holds <= 64
+        // rows, so an LTD decrement of row r can only need corrections of later block steps if set)
+        for (uint32_t x = tid; x < nrows; x += nthr) {
+          const uint16_t id = s_rows[x];
+          bool dup = false;
+          const uint32_t lim = min(nrows, x + 65u);
+          for (uint32_t y = x + 1; y < lim && !dup; ++y) dup = s_rows[y] == id;
+          if (dup) s_rstep[x] = (uint16_t)(s_rstep[x] | 0x8000u);
+        }
+        __syncthreads();
       }
       const int kend = kb;
       const int fp = ep & 1;
-      if (trace && tid == 0) { tr0 = globaltimer(); *s_tmax = 0ull; }
+      if (trace && tid == 0) { tr0 = globaltimer(); *s_tmax = 0ull; s_misc[3] = 0; }
 
       // ---------------------------------------------------------- speculation (warp-synchronous, no CTA barrier)
       int p = kend;             // first step this thread did not fully process
@@ -554,7 +509,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
                   for (int x = 0; x < 8; ++x) {
                     const bool in = r + x < rblk1;
                     o[x] = in ? s_woff[r + x] : (uint32_t)(n_in * wpr);   // the all-zero row
-                    st[x] = in ? (uint32_t)s_rstep[r + x] : 0xFFFFu;
+                    st[x] = in ? (uint32_t)(s_rstep[r + x] & 0x7FFFu) : 0xFFFFu;
                   }
 #pragma unroll
                   for (int x = 0; x < 8; ++x) w[x] = (wcol[o[x]] >> fsh) & Z::LMASK;
@@ -576,8 +531,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
               const int nrows_blk = rblk1 - rblk0;
               if (__any_sync(FULL, ltd_blk != 0)) {
                 // this lane's rows of the block and their steps (the same for every pair)
-                const int bsel0 = lane < nrows_blk ? (int)s_rstep[rblk0 + lane] - (kb0 - ka) : 0;
-                const int bsel1 = lane + 32 < nrows_blk ? (int)s_rstep[rblk0 + 32 + lane] - (kb0 - ka) : 0;
+                const int bsel0 = lane < nrows_blk ? (int)(s_rstep[rblk0 + lane] & 0x7FFFu) - (kb0 - ka) : 0;
+                const int bsel1 = lane + 32 < nrows_blk ? (int)(s_rstep[rblk0 + 32 + lane] & 0x7FFFu) - (kb0 - ka) : 0;
                 const uint32_t row0 = lane < nrows_blk ? (uint32_t)s_rows[rblk0 + lane] : 0u;
                 const uint32_t row1 = lane + 32 < nrows_blk ? (uint32_t)s_rows[rblk0 + 32 + lane] : 0u;
 #pragma unroll 1
@@ -616,6 +571,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
 #pragma unroll 1
                 for (int b = 0; b < nb; ++b) {
                   const int kk_b = kb0 + b;
+                  // a crossing before kk_b exists in the cluster: stop here (state is that after kk_b - 1)
+                  if (b > 0 && kk_b > ld_volatile_shared_u32addr(flag_addr)) { done = true; p = kk_b; break; }
                   const int t = tbase + kk_b;
                   const int rhi = (int)(s_offs[kk_b - ka + 1] - wbase);
                   const uint32_t snap = vmax_lanes<CPT>(run_prev, my_acc[b * nthr]);
@@ -668,7 +625,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
                         if (applied) {
                           atomicSub(pw, 1u << shc);
                           // the later block steps that contain row i were summed with the old code
-                          block_correct<CPT>(s_rows, s_rstep, my_acc, nthr, rhi, rblk1, kb0 - ka, b, nb, i,
+                          if (s_rstep[rlo + xr] & 0x8000u) block_correct<CPT>(s_rows, s_rstep, my_acc, nthr, rhi, rblk1, kb0 - ka, b, nb, i,
                                              0u - (1u << (c * Z::LW)));
                         }
                         ++ev_step;
@@ -814,6 +771,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         if (mycol) eng_spec += (uint32_t)(p - k0 + (cand ? 1 : 0)) * (uint32_t)__popc(valid);
       }
       if (trace && lane == 0) atomicMax(s_tmax, globaltimer());
+      if (trace && mycol) atomicMax(&s_misc[3], p - k0);       // deepest speculation of the CTA
 
       // ---------------------------------------------------------- CTA summary -> cluster exchange
       {
@@ -858,7 +816,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
           st_cluster_u64(slot, (uint32_t)lane, A);
           st_cluster_u64(slot + 1, (uint32_t)lane, K);
         }
-        if (lane == 0) s_flag[fp ^ 1] = INT_MAX;
+        if (lane == 0) { s_flag[fp ^ 1] = INT_MAX; s_misc[1] = 0; }
       }
       if (cs > 1) { cluster_arrive(); cluster_wait(); } else { __syncthreads(); }   // the one cross-SM exchange
       if (trace && tid == 0) tr3 = globaltimer();
@@ -1027,6 +985,11 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
             if (spiked >> c & 1u) atomicOr(&d.raster_out[(size_t)P * nwe + (jcol[c] >> 5)], 1u << (jcol[c] & 31));
         }
       }
+      if (event && spiked) {                               // this CTA's spikers (local column index)
+#pragma unroll
+        for (int c = 0; c < CPT; ++c)
+          if (spiked >> c & 1u) { const int pos = atomicAdd(&s_misc[1], 1); s_misc[16 + pos] = jcol[c] - col0; }
+      }
       const int k_last = event ? P : (at_end ? kend - 1 : P - 1);
       // spike timers of the inputs through the committed step
       for (int kk = k0 + tid; kk <= k_last; kk += nthr) {
@@ -1038,67 +1001,60 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         unsigned long long* rec = trace + (size_t)ep * 8;
         rec[0] = ((unsigned long long)b << 32) | (unsigned)k0;
         rec[1] = ((unsigned long long)(event ? 1 : (unknown ? 2 : 0)) << 32) | (unsigned)P;
-        rec[2] = tr0; rec[3] = *s_tmax; rec[4] = tr2; rec[5] = tr3; rec[6] = globaltimer(); rec[7] = rec[6];
+        rec[2] = tr0; rec[3] = *s_tmax; rec[4] = tr2; rec[5] = tr3; rec[6] = (unsigned long long)s_misc[3];
+        rec[7] = globaltimer();
       }
       if (spiked) {
 #pragma unroll
         for (int c = 0; c < CPT; ++c)
           if (spiked >> c & 1u) { lpost[c] = tP; s_lpost[jcol[c] - col0] = tP; }
       }
-      pend_mask = spiked;
-      pend_t = tP;
+      // (a5) LTP eq.(6) / (a6) deterministic arm eqs.(4)(5)(8) at t* for this CTA's spikers: every thread
+      // takes (spiker, group of 4 rows) pairs; updates are atomic (two spikers may share a row word)
+      const int nsp = event ? s_misc[1] : 0;
+      if (nsp > 0) {
+        for (int item = tid; item < nsp * nq4; item += nthr) {
+          const int m = item / nq4, grp = item - m * nq4;
+          const int jl = s_misc[16 + m];
+          const int Wg = col0 + jl;
+          const int ww = jl / CPW, wsh = (jl % CPW) * BITS;
+          const uint4 u = philox((uint32_t)tP, (uint32_t)Wg, (uint32_t)grp, stoch ? TAG_LTP : TAG_ROUND, seed);
+#pragma unroll
+          for (int r = 0; r < 4; ++r) {
+            const int i = 4 * grp + r;
+            if (i >= n_in) break;
+            const int lpi = s_lpre[i];
+            uint32_t* pw = s_w + i * wpr + ww;
+            if (stoch) {
+              if (lpi < 0) continue;
+              const int D = tP - lpi;
+              if (D >= L_pot) continue;
+              ++ltp_trials;
+              if (pick(u, r) <= s_pot[D]) {                    // eq.(6), R10: Dt = D >= 0
+                ++ltp_events;
+                if (((*pw >> wsh) & FMASK) < (uint32_t)qmax) atomicAdd(pw, 1u << wsh);
+              }
+            } else {                                           // eqs.(4)(5)(8), R16/R17
+              const int q0 = (int)((*pw >> wsh) & FMASK);
+              const bool pot = lpi >= 0 && (tP - lpi) <= t_ltp;
+              const int base = pot ? s_dbp[q0] : s_dbd[q0];
+              const uint32_t thr = pot ? s_dtp[q0] : s_dtd[q0];
+              const int dq = base + (pick(u, r) < thr ? 1 : 0);
+              int q1 = pot ? q0 + dq : q0 - dq;
+              q1 = q1 < 0 ? 0 : (q1 > qmax ? qmax : q1);
+              if (q1 != q0) atomicAdd(pw, (uint32_t)(q1 - q0) << wsh);
+              if (pot) { ++ltp_trials; if (dq > 0) ++ltp_events; }
+              else     { ++ltd_trials; if (dq > 0) ++ltd_events; }
+            }
+          }
+        }
+        __syncthreads();                                                             // S4
+      }
       k0 = k_last + 1;
       ++ep;
       ++eng_epochs;
     }  // epochs
 
-    // the last event's LTP of this image (if any) before the state is written back
-    if (__any_sync(FULL, pend_mask != 0)) {
-      const int tP = pend_t;
-      for (uint32_t wm = __ballot_sync(FULL, pend_mask != 0); wm; wm &= wm - 1) {
-        const int Lsrc = __ffs(wm) - 1;
-        const uint32_t pm = __shfl_sync(FULL, pend_mask, Lsrc);
-        for (uint32_t cm = pm; cm; cm &= cm - 1) {
-          const int c = __ffs(cm) - 1;
-          const int tidL = warp * 32 + Lsrc;
-          const int jl = (tidL / TPW) * CPW + (tidL % TPW) + TPW * c;
-          const int Wg = col0 + jl;
-          const int ww = jl / CPW, wsh = (jl % CPW) * BITS;
-          for (int grp = lane; grp < nq4; grp += 32) {
-            const uint4 u = philox((uint32_t)tP, (uint32_t)Wg, (uint32_t)grp, stoch ? TAG_LTP : TAG_ROUND, seed);
-#pragma unroll
-            for (int r = 0; r < 4; ++r) {
-              const int i = 4 * grp + r;
-              if (i >= n_in) break;
-              const int lpi = s_lpre[i];
-              uint32_t* pw = s_w + i * wpr + ww;
-              if (stoch) {
-                if (lpi < 0) continue;
-                const int D = tP - lpi;
-                if (D >= L_pot) continue;
-                ++ltp_trials;
-                if (pick(u, r) <= s_pot[D]) {
-                  ++ltp_events;
-                  if (((*pw >> wsh) & FMASK) < (uint32_t)qmax) atomicAdd(pw, 1u << wsh);
-                }
-              } else {
-                const int q0 = (int)((*pw >> wsh) & FMASK);
-                const bool pot = lpi >= 0 && (tP - lpi) <= t_ltp;
-                const int base = pot ? s_dbp[q0] : s_dbd[q0];
-                const uint32_t thr = pot ? s_dtp[q0] : s_dtd[q0];
-                const int dq = base + (pick(u, r) < thr ? 1 : 0);
-                int q1 = pot ? q0 + dq : q0 - dq;
-                q1 = q1 < 0 ? 0 : (q1 > qmax ? qmax : q1);
-                if (q1 != q0) atomicAdd(pw, (uint32_t)(q1 - q0) << wsh);
-                if (pot) { ++ltp_trials; if (dq > 0) ++ltp_events; }
-                else     { ++ltd_trials; if (dq > 0) ++ltd_events; }
-              }
-            }
-          }
-        }
-      }
-      pend_mask = 0;
-    }
     if (rank == 0 && tid == 0) {
       post_sum += (unsigned long long)img_spikes;
       if (d.spike_counts) d.spike_counts[b] = img_spikes;

@@ -60,7 +60,8 @@ def main():
     spec_end = tr[:, :, 3]
     summ = tr[:, :, 4]
     exch = tr[:, :, 5]
-    comm = tr[:, :, 6]
+    depth = tr[:, :, 6]
+    comm = tr[:, :, 7]
     end = tr[:, :, 7]
     tot = end.max(axis=0) - start
     spec = spec_end.max(axis=0) - start
@@ -81,6 +82,10 @@ def main():
     print(f"per-CTA speculation ns: mean {own.mean():.0f}  max-over-CTAs mean {own.max(axis=0).mean():.0f}  "
           f"-> {own.max(axis=0).sum() / steps.sum():.0f} ns/step (max CTA)  {own.mean(axis=0).sum() / steps.sum():.0f} ns/step (mean CTA)")
     print(f"start skew ns: mean {skew.mean():.0f}  max {skew.max(axis=0).mean():.0f}")
+    rate = own / np.maximum(1, depth)                       # ns per speculated step, per CTA per epoch
+    crit = own.argmax(axis=0)
+    print(f"critical CTA: ns/step {np.mean([rate[crit[e], e] for e in range(E)]):.0f} at depth "
+          f"{np.mean([depth[crit[e], e] for e in range(E)]):.1f};  other CTAs ns/step {np.median(rate):.0f} at depth {np.median(depth):.1f}")
     print("first 12 epochs: k0 P kind | spec(ns) spread wait commit ltp")
     for e in range(min(12, E)):
         print(f"{k0[e]:4d} {Pst[e]:5d} {kind[e]} | {spec[e]:7d} {spread[e]:6d} {wait[e]:6d} {commit[e]:6d} {ltp[e]:6d}")
