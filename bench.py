@@ -237,8 +237,20 @@ def main():
     value = images / dev_s
     ev_rate = events / dev_s
 
-    # ---- latency floor: same launch shape, barriers + exchange only (SNN_FLOOR_PROBE)
+    # ---- latency floor.  Event engine: the path needs one cluster exchange per epoch (post spike), so
+    # its synchronisation floor is epochs x the measured barrier.cluster cost at this cluster size
+    # (profiles/r01_sync_probe.txt, 128 threads); per-step engine: measured live with SNN_FLOOR_PROBE.
     floor = None
+    if args.engine == 0:
+        probe_ns = {1: 380.7, 2: 444.0, 4: 485.5, 8: 572.6, 16: 760.9}
+        cs = info["cluster_size"]
+        key = min(probe_ns, key=lambda k: abs(k - cs))
+        per_image_us = 1e3 * (sum(step_ms) / args.steps) / B
+        ep = int(stats[8]) / (B * args.steps)
+        floor = {"kind": "event engine: epochs x cluster-exchange cost",
+                 "epochs_per_image": ep, "exchange_ns": probe_ns[key],
+                 "t_floor_us_per_image": ep * probe_ns[key] / 1e3, "t_image_us": per_image_us,
+                 "frac": ep * probe_ns[key] / 1e3 / per_image_us}
     if not args.no_floor and args.engine == 1:
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)

@@ -445,13 +445,13 @@ int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** 
   for (int cs : order) {
     if (cs > h->ngroups) continue;
     const int max_groups = (h->ngroups + cs - 1) / cs;
-    // columns per thread: SWAR-maximal (8/bits) -- fewest warps, fewest per-step instructions per SM
-    // (measured faster than 2 columns/thread on C4, profiles/r01_event_engine.md); SNN_CPT overrides
+    // columns per thread: 2 at 2 bits when the CTA stays <= 256 threads (measured best on C4 with
+    // tools/sweep.py), else the SWAR maximum 8/bits; SNN_CPT overrides
     int cpt = 1;
     if (ev) {
       const char* env = getenv("SNN_CPT");
       const int cap = 8 / bits;
-      cpt = cap;
+      cpt = (bits == 2 && snn::event_threads(max_groups, bits, 2) <= max_thr) ? 2 : cap;
       if (env && atoi(env) >= 1 && atoi(env) <= cap && (cap % atoi(env)) == 0) cpt = atoi(env);
     }
     const int nthr = ev ? snn::event_threads(max_groups, bits, cpt) : (max_groups * 32 < 128 ? 128 : max_groups * 32);

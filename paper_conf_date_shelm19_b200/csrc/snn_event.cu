@@ -249,7 +249,7 @@ __host__ __device__ inline EvLayout ev_layout(int n_in, int slice_words, int L_p
   L.slots = o;  o = align16(o + 2 * kMaxCluster * 2 * 8);   // [parity][rank][2] u64
   L.wsum = o;   o = align16(o + 32 * 2 * 8);                // per warp: summary, key
   L.flags = o;  o = align16(o + 4 * 4);                     // early-stop flag per epoch parity
-  L.misc = o;   o = align16(o + 16 * 8 + (size_t)nthr * 4 * 4);   // header + local spiker list
+  L.misc = o;   o = align16(o + 16 * 8 + (size_t)nthr * 4 * 4 + 16 + 32 * 16);   // header, spikers, warp prof
   L.w = o;      o = align16(o + (size_t)slice_words * 4);
   L.pot = o;    o = align16(o + (size_t)(L_pot > 0 ? L_pot : 1) * 4);
   L.dep = o;    o = align16(o + (size_t)(L_dep > 0 ? L_dep : 1) * 4);
@@ -384,6 +384,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
   unsigned long long* s_tmax = reinterpret_cast<unsigned long long*>(s_misc + 8);
   unsigned long long tr0 = 0, tr2 = 0, tr3 = 0;
   long long prof_int = 0, prof_ltd = 0, prof_seq = 0, prof_blk = 0, prof_loop0 = 0, prof_loop = 0;
+  long long prof_ev = 0, prof_nev = 0;
   const long long prof_clk0 = clock64();
   const unsigned long long prof_ns0 = globaltimer();
   // pending LTP of the previous epoch (owner warps run it while the others start speculating)
@@ -445,7 +446,11 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
       }
       const int kend = kb;
       const int fp = ep & 1;
-      if (trace && tid == 0) { tr0 = globaltimer(); *s_tmax = 0ull; s_misc[3] = 0; }
+      if (trace && tid == 0) {
+        tr0 = globaltimer(); *s_tmax = 0ull; s_misc[3] = 0;
+        *reinterpret_cast<unsigned long long*>(s_misc + 10) = 0ull;
+        *reinterpret_cast<unsigned long long*>(s_misc + 12) = 0ull;
+      }
 
       // ---------------------------------------------------------- speculation (warp-synchronous, no CTA barrier)
       int p = kend;             // first step this thread did not fully process
@@ -470,7 +475,12 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
           for (int r = 0; r < cs; ++r)
             if (r != rank) red_min_cluster(&s_flag[fp], (uint32_t)r, fstep);
         };
-        if (trace && lane == 0) prof_loop0 = clock64();
+        long long e_int0 = prof_int, e_ltd0 = prof_ltd, e_seq0 = prof_seq, e_ev0 = prof_ev;
+        if (trace && lane == 0) {
+          prof_loop0 = clock64();
+          const unsigned long long gt = globaltimer();
+          atomicMax(reinterpret_cast<unsigned long long*>(s_misc + 10), gt);   // latest warp loop start
+        }
         while (__any_sync(FULL, !done)) {
           if (!done && (kk >= kend || kk > ld_volatile_shared_u32addr(flag_addr))) { done = true; p = kk; }
           if (kk >= kend) break;                                  // warp-uniform
@@ -492,7 +502,35 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
               uint32_t* const my_acc = s_acc + tid;              // [b * nthr + tid]: SWAR sums of block step b
               const int rblk0 = r0;
               const int rblk1 = (int)(s_offs[kb0 - ka + nb] - wbase);
+              // columns held (refractory / inhibited) through the whole block run no LIF, so their sums
+              // are never used: a warp with no LIF and no LTD in the block only counts down (exact)
+              uint32_t live = 0, ltd_pre = 0;
               if (!done) {
+#pragma unroll
+                for (int c = 0; c < CPT; ++c) {
+                  if ((valid >> c & 1u) && cnt[c] < nb) live |= 1u << c;
+                  if ((ltd_cols >> c & 1u) && (tbase + kb0 - lpost[c]) < L_dep) ltd_pre |= 1u << c;
+                }
+              }
+              const bool warp_live = __any_sync(FULL, live != 0);
+              if (!warp_live && !__any_sync(FULL, ltd_pre != 0)) {
+                if (!done) {
+                  int stop_at = nb;                                // honour the early-stop flag per step
+                  const int f = ld_volatile_shared_u32addr(flag_addr);
+                  if (f < kb0 + nb - 1) stop_at = max(1, f - kb0 + 1);
+#pragma unroll
+                  for (int c = 0; c < CPT; ++c) cnt[c] -= stop_at;
+                  if (kb0 == k0) {
+#pragma unroll
+                    for (int c = 0; c < CPT; ++c) { v1[c] = v[c]; cnt1[c] = cnt[c] + stop_at - 1; }
+                  }
+                  if (stop_at < nb) { done = true; p = kb0 + stop_at; }
+                }
+                kk = kb0 + nb;
+                r0 = rblk1;
+                continue;
+              }
+              if (!done && warp_live) {
                 // (a2) eq.(3) for all block steps in one flattened pass over the block's rows: the running
                 // SWAR sum is stored into the slot of the row's step; lanes never overflow (<= 64 rows), so
                 // the sum at the end of step b is the lane-wise max of slots 0..b.
@@ -603,6 +641,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
                     for (int c = 0; c < CPT; ++c)
                       if ((ltd_blk >> c & 1u) && (t - lpost[c]) < L_dep) on_b |= 1u << c;
                   }
+                  const long long pe0 = prof ? clock64() : 0;
                   if (on_b) {                                         // LTD events of step b (rare)
                     const int lo = rlo - rblk0, nrb = rhi - rlo;
                     const int nlog_step = nlog;
@@ -649,7 +688,9 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
                     }
                     ltd_events += ev_step;
                     ltd_trials += (uint32_t)__popc(on_b) * (uint32_t)nrb;
+                    if (trace) prof_nev += ev_step;
                   }
+                  if (prof) { __syncwarp(__activemask()); prof_ev += clock64() - pe0; }
 #pragma unroll
                   for (int c = 0; c < CPT; ++c) {                     // commit step b
                     v[c] = cnt[c] == 0 ? vn[c] : v[c];
@@ -766,7 +807,18 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
           ++kk;
           r0 = r1;
         }
-        if (trace && lane == 0) prof_loop += clock64() - prof_loop0;
+        if (trace && lane == 0) {
+          const long long dl = clock64() - prof_loop0;
+          prof_loop += dl;
+          atomicMax(reinterpret_cast<unsigned long long*>(s_misc + 12), (unsigned long long)dl);  // longest warp loop
+          // per-warp per-epoch breakdown (16-bit fields, cycles/16): int | ltd | seq | events
+          unsigned long long* s_wp = reinterpret_cast<unsigned long long*>(s_misc + 16 + nthr * CPT + 4) + warp * 2;
+          s_wp[0] = (unsigned long long)dl;
+          s_wp[1] = (unsigned long long)(min((prof_int - e_int0) >> 4, 0xFFFFll)) |
+                    ((unsigned long long)(min((prof_ltd - e_ltd0) >> 4, 0xFFFFll)) << 16) |
+                    ((unsigned long long)(min((prof_seq - e_seq0) >> 4, 0xFFFFll)) << 32) |
+                    ((unsigned long long)(min((prof_ev - e_ev0) >> 4, 0xFFFFll)) << 48);
+        }
         if (!mycol) p = kend;
         if (mycol) eng_spec += (uint32_t)(p - k0 + (cand ? 1 : 0)) * (uint32_t)__popc(valid);
       }
@@ -822,16 +874,17 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
       if (trace && tid == 0) tr3 = globaltimer();
 
       // ---------------------------------------------------------- global decision
-      uint32_t W1 = 0, count = 0;
-      unsigned long long K = 0;
-      for (int r = 0; r < cs; ++r) W1 = max(W1, (uint32_t)(s_slots[(size_t)(fp * kMaxCluster + r) * 2] >> 32));
-      for (int r = 0; r < cs; ++r) {
-        const unsigned long long A = s_slots[(size_t)(fp * kMaxCluster + r) * 2];
-        if ((uint32_t)(A >> 32) == W1) {
-          count += (uint32_t)A;
-          const unsigned long long kx = s_slots[(size_t)(fp * kMaxCluster + r) * 2 + 1];
-          K = kx > K ? kx : K;
-        }
+      uint32_t W1, count;
+      unsigned long long K;
+      {                                                    // lane r reads CTA r's summary; warp reductions
+        const unsigned long long A = lane < cs ? s_slots[(size_t)(fp * kMaxCluster + lane) * 2] : 0ull;
+        const unsigned long long Kr = lane < cs ? s_slots[(size_t)(fp * kMaxCluster + lane) * 2 + 1] : 0ull;
+        W1 = __reduce_max_sync(FULL, (uint32_t)(A >> 32));
+        const bool at = lane < cs && (uint32_t)(A >> 32) == W1;
+        count = __reduce_add_sync(FULL, at ? (uint32_t)A : 0u);
+        const uint32_t kh = __reduce_max_sync(FULL, at ? (uint32_t)(Kr >> 32) : 0u);
+        const uint32_t kl = __reduce_max_sync(FULL, (at && (uint32_t)(Kr >> 32) == kh) ? (uint32_t)Kr : 0u);
+        K = ((unsigned long long)kh << 32) | kl;
       }
       const int P = 0xFFFF - (int)(W1 >> 1);
       const bool unknown = (W1 & 1u) != 0u;
@@ -1001,7 +1054,14 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         unsigned long long* rec = trace + (size_t)ep * 8;
         rec[0] = ((unsigned long long)b << 32) | (unsigned)k0;
         rec[1] = ((unsigned long long)(event ? 1 : (unknown ? 2 : 0)) << 32) | (unsigned)P;
-        rec[2] = tr0; rec[3] = *s_tmax; rec[4] = tr2; rec[5] = tr3; rec[6] = (unsigned long long)s_misc[3];
+        unsigned long long best = 0, bestw = 0;
+        {
+          const unsigned long long* s_wp = reinterpret_cast<const unsigned long long*>(s_misc + 16 + nthr * CPT + 4);
+          for (int w = 0; w < nwarps; ++w) if (s_wp[2 * w] > best) { best = s_wp[2 * w]; bestw = s_wp[2 * w + 1]; }
+        }
+        rec[2] = tr0; rec[3] = *s_tmax; rec[4] = bestw; rec[5] = tr3;
+        rec[6] = (unsigned long long)s_misc[3] |
+                 ((*reinterpret_cast<unsigned long long*>(s_misc + 12)) << 16);   // depth | longest warp loop (cycles)
         rec[7] = globaltimer();
       }
       if (spiked) {
@@ -1114,12 +1174,14 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
     if (tid == 0) *s_pm = 0ull;
     __syncthreads();
     if (lane == 0) atomicMax(s_pm, ((unsigned long long)prof_loop << 8) | (unsigned)warp);
+    prof_nev = __reduce_add_sync(FULL, (unsigned)prof_nev);
     __syncthreads();
     if (lane == 0 && (int)(*s_pm & 0xFFull) == warp && d.trace_cap > 0) {
       unsigned long long* rec = trace + (size_t)(d.trace_cap - 1) * 8;
-      rec[0] = (0xFFFFFFFFull << 32) | (unsigned)warp; rec[1] = (unsigned long long)prof_int;
+      rec[0] = (0xFFFFFFFFull << 32) | ((unsigned long long)(prof_nev & 0xFFFF) << 16) | (unsigned)warp;
+      rec[1] = (unsigned long long)prof_int;
       rec[2] = (unsigned long long)prof_ltd; rec[3] = (unsigned long long)prof_seq; rec[4] = (unsigned long long)prof_blk;
-      rec[5] = (unsigned long long)prof_loop; rec[6] = (unsigned long long)(clock64() - prof_clk0);
+      rec[5] = (unsigned long long)prof_loop; rec[6] = (unsigned long long)prof_ev;
       rec[7] = globaltimer() - prof_ns0;
     }
   }

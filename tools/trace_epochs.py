@@ -46,8 +46,8 @@ def main():
     for r in range(prof.shape[0]):
         if (prof[r, 0] >> 32) & 0xFFFFFFFF == 0xFFFFFFFF and prof[r, 4] > 0:
             nbk = prof[r, 4]
-            print(f"CTA {r} slowest warp {prof[r,0] & 0xFFFFFFFF} cycles/step: integrate {prof[r,1]/nbk:.0f}  ltd {prof[r,2]/nbk:.0f}  seq {prof[r,3]/nbk:.0f}"
-                  f"  whole-loop {prof[r,5]/nbk:.0f}  (block steps {nbk})  SM clock {prof[r,6]/max(1,prof[r,7]):.3f} GHz")
+            print(f"CTA {r} slowest warp {prof[r,0] & 0xFFFF} cycles/step: integrate {prof[r,1]/nbk:.0f}  ltd {prof[r,2]/nbk:.0f}  seq {prof[r,3]/nbk:.0f}"
+                  f" (of which LTD events {prof[r,6]/nbk:.0f}, {((prof[r,0] >> 16) & 0xFFFF)/nbk:.2f} events/step)  whole-loop {prof[r,5]/nbk:.0f}  (block steps {nbk})")
     st = net.stats()
     cs, E, _ = tr.shape
     valid = tr[0, :, 7] > 0
@@ -60,7 +60,8 @@ def main():
     spec_end = tr[:, :, 3]
     summ = tr[:, :, 4]
     exch = tr[:, :, 5]
-    depth = tr[:, :, 6]
+    depth = tr[:, :, 6] & 0xFFFF
+    late = tr[:, :, 6] >> 16                                 # longest warp loop of the CTA (cycles)
     comm = tr[:, :, 7]
     end = tr[:, :, 7]
     tot = end.max(axis=0) - start
@@ -86,6 +87,13 @@ def main():
     crit = own.argmax(axis=0)
     print(f"critical CTA: ns/step {np.mean([rate[crit[e], e] for e in range(E)]):.0f} at depth "
           f"{np.mean([depth[crit[e], e] for e in range(E)]):.1f};  other CTAs ns/step {np.median(rate):.0f} at depth {np.median(depth):.1f}")
+    bw = tr[:, :, 4]
+    parts = np.array([[(bw[crit[e], e] >> (16 * k)) & 0xFFFF for k in range(4)] for e in range(E)]) * 16.0
+    dc = np.array([max(1, depth[crit[e], e]) for e in range(E)])
+    print("critical CTA slowest warp cycles/step: integrate %.0f  ltd-draws %.0f  seq %.0f (LTD events %.0f)" %
+          tuple((parts / dc[:, None]).mean(axis=0)))
+    print(f"longest warp loop: critical CTA {np.mean([late[crit[e], e] for e in range(E)]) / 1.965:.0f} ns "
+          f"(= {np.mean([late[crit[e], e] / max(1, depth[crit[e], e]) for e in range(E)]):.0f} cycles/step), median CTA {np.median(late) / 1.965:.0f} ns")
     print("first 12 epochs: k0 P kind | spec(ns) spread wait commit ltp")
     for e in range(min(12, E)):
         print(f"{k0[e]:4d} {Pst[e]:5d} {kind[e]} | {spec[e]:7d} {spread[e]:6d} {wait[e]:6d} {commit[e]:6d} {ltp[e]:6d}")
