@@ -133,7 +133,8 @@ int snn_present_ex(snn_handle* h, const void* input, int T, uint64_t seed, int f
 int snn_present_raster(snn_handle* h, const uint32_t* raster, int T, uint64_t seed);
 
 /* Ensemble: n independent handles (equal n_in, n_exc, cluster size; bits and parameters may
- * differ) each present n_images images in ONE launch.  images[k]: n_images x n_in bytes and
+ * differ) each present n_images images in ONE launch (linked shards of one world: all of them,
+ * see snn_shard_link).  images[k]: n_images x n_in bytes and
  * seeds[k]: n_images seeds for handle k (arrays of host pointers to host or device buffers). */
 int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images, int n_images, int T,
                      const uint64_t* const* seeds);
@@ -160,8 +161,9 @@ int snn_get_stats(snn_handle* h, uint64_t stats[SNN_NSTATS]);
 int snn_reset_stats(snn_handle* h);
 /* Introspection: [0] cluster size, [1] threads per CTA, [2] dynamic smem bytes per CTA,
  * [3] words per weight row in a CTA slice, [4] q_max, [5] L_pot, [6] L_dep, [7] kernel launches so far,
- * [8] engine, [9] columns per thread (event engine), [10] on-chip row window, [11] LTD undo-log depth. */
-#define SNN_NINFO 12
+ * [8] engine, [9] columns per thread (event engine), [10] on-chip row window, [11] LTD undo-log depth,
+ * [12] first global column (col_base), [13] columns of the whole network, [14] world, [15] shard. */
+#define SNN_NINFO 16
 int snn_get_info(const snn_handle* h, int64_t info[SNN_NINFO]);
 
 /* Tracing: with max_epochs > 0 the event engine records, per CTA and epoch,
@@ -171,6 +173,35 @@ int snn_get_info(const snn_handle* h, int64_t info[SNN_NINFO]);
  * values of the last presentation call.  0 disables tracing. */
 int snn_set_trace(snn_handle* h, int max_epochs);
 int snn_get_trace(snn_handle* h, uint64_t* out, size_t cap);
+
+/* ---- Column sharding of ONE network across ranks.
+ * The n_exc_total post-synaptic columns are split into `world` contiguous slices on 32-column
+ * boundaries: shard r owns columns [32*floor(r*G/world), 32*floor((r+1)*G/world)) with
+ * G = ceil(n_exc_total/32) (G >= world required).  A shard handle is a network of its own columns
+ * whose random draws (R13: init, LTD, LTP, rounding) and WTA keys (R7) use GLOBAL column indices, so
+ * the union of the shards reproduces the unsharded network bit for bit.  The encoder and the input
+ * spike timers are replicated (every shard draws the same inputs from the same seeds).  Per epoch of
+ * the event engine each shard publishes a 16-byte summary (earliest crossing step,
+ * crossing count, best WTA key) into every shard's mailbox in device memory (peer stores over NVLink)
+ * and every shard applies the same reduction: the exchange step of P:88 §III-B's lateral inhibition
+ * across GPUs.  Event engine only.  All shards of a world must run the same presentation calls
+ * (inputs, seeds, T, flags) in the same order; a rank that stops answering makes the others trap
+ * after 20 s instead of hanging.
+ * Readouts (weights, spikes, state) of a shard cover its own columns: n_in x n_exc_local codes, a
+ * T x ceil(n_exc_local/32) raster, state with n_exc = n_exc_local.  Stats [2..5] count the shard's own
+ * trials/events; [0], [1], [6], [7] are the network's (identical on every shard). */
+#define SNN_IPC_HANDLE_BYTES 64
+int snn_create_shard(int n_in, int n_exc_total, int bits, const snn_params* p, int shard, int world,
+                     snn_handle** out);
+/* Multi-process (one rank per GPU): export this shard's mailbox as a CUDA IPC handle
+ * (SNN_IPC_HANDLE_BYTES bytes into out), gather all ranks' handles (e.g. torch.distributed
+ * all_gather), then connect with the world's handles in rank order (world x SNN_IPC_HANDLE_BYTES). */
+int snn_shard_ipc_handle(snn_handle* h, void* out, size_t cap);
+int snn_shard_connect(snn_handle* h, const void* handles, size_t n_bytes);
+/* Single process: link shards 0..world-1 directly (hs[r] is shard r).  Shards on one device must be
+ * presented together with snn_present_many (one launch keeps every shard co-resident); shards on
+ * distinct peer-capable devices may be presented from one thread each. */
+int snn_shard_link(snn_handle* const* hs, int world);
 
 const char* snn_last_error(void);
 

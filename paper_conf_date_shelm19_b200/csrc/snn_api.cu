@@ -106,6 +106,15 @@ struct snn_handle {
   uint16_t* d_rows = nullptr;    size_t rows_buf_cap = 0;
   uint16_t* d_rows16 = nullptr;  size_t rows16_cap = 0;
   unsigned long long* d_trace = nullptr; int trace_epochs = 0;
+  int max_clusters = 0;          // co-resident clusters of this launch shape
+  // column sharding
+  int col_base = 0, n_exc_total = 0, world = 1, shard = 0;
+  snn::Mailbox* d_mbox = nullptr;
+  snn::Mailbox** d_peers = nullptr;
+  std::vector<void*> ipc_opened;       // peer mailboxes opened with cudaIpcOpenMemHandle
+  std::vector<snn_handle*> linked;     // in-process shards (snn_shard_link), rank order
+  bool connected = false;
+  unsigned long long shard_launches = 0;
 };
 
 namespace {
@@ -170,13 +179,30 @@ void fill_static(const snn_handle* h, NetDesc& d) {
   d.stats = h->d_stats;
   d.rows_cap = h->rows_cap; d.offs_cap = h->offs_cap; d.logn = h->logn;
   d.trace = h->d_trace; d.trace_cap = h->trace_epochs;
+  d.col_base = h->col_base; d.n_exc_total = h->n_exc_total; d.world = 1; d.shard = h->shard;
+}
+
+// Sharded launch fields: mailbox, peers and a launch-unique sequence base (all shards count the
+// same presentation calls, so the base agrees across ranks); this rank's early-stop flags are
+// cleared before the launch.
+int shard_arm(snn_handle* h, NetDesc& d) {
+  if (h->world <= 1) return SNN_OK;
+  if (!h->connected) return fail(SNN_EINVAL, "shard %d of %d is not connected (snn_shard_connect / snn_shard_link)",
+                                 h->shard, h->world);
+  d.world = h->world; d.shard = h->shard; d.mbox = h->d_mbox; d.peers = h->d_peers;
+  d.seq_base = (++h->shard_launches) << 32;
+  CUDA_TRY(cudaMemsetAsync(&h->d_mbox->flag[0], 0x7F, 2 * sizeof(int), h->stream));
+  return SNN_OK;
 }
 
 void free_all(snn_handle* h) {
+  for (void* q : h->ipc_opened) if (q) cudaIpcCloseMemHandle(q);
+  h->ipc_opened.clear();
   void* ptrs[] = {h->d_w, h->d_enc, h->d_pot, h->d_dep, h->d_dbp, h->d_dbd, h->d_dtp, h->d_dtd,
                   h->d_v, h->d_cnt, h->d_lpost, h->d_lpre, h->d_stats, h->d_raster, h->d_inrec,
                   h->d_img, h->d_rin, h->d_seeds, h->d_counts, h->d_codes, h->d_bad,
-                  h->d_words, h->d_ecnt, h->d_offs, h->d_rows, h->d_rows16, h->d_trace};
+                  h->d_words, h->d_ecnt, h->d_offs, h->d_rows, h->d_rows16, h->d_trace,
+                  h->d_mbox, h->d_peers};
   for (void* q : ptrs) if (q) cudaFree(q);
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
 }
@@ -275,6 +301,9 @@ int present_impl(snn_handle* h, const void* input, int n_images, int T, const ui
     return SNN_OK;
   }
   if (!input || !seeds) return fail(SNN_EINVAL, "input / seeds is NULL");
+  for (snn_handle* o : h->linked)
+    if (o != h && o->dev == h->dev)
+      return fail(SNN_EINVAL, "shards linked on one device must be presented together (snn_present_many)");
   DevGuard g(h->dev);
   NetDesc d;
   fill_static(h, d);
@@ -316,6 +345,7 @@ int present_impl(snn_handle* h, const void* input, int n_images, int T, const ui
   if (ev) {
     rc = event_prepass(h, d, img, rin, n_images, T, (flags & SNN_KEEP_STATE) ? t0 : 0, sd);
     if (rc) return rc;
+    if ((rc = shard_arm(h, d))) return rc;
     lp.single = d;
     CUDA_TRY(snn::launch_present_event_mode(lp, 1, h->cs, h->nthr, h->smem, h->bits, h->cpt, h->p.membrane_mode,
                                             h->stream));
@@ -366,15 +396,22 @@ int snn_params_preset(snn_params* p, int preset) {
   return SNN_OK;
 }
 
-int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** out) {
-  if (!out) return fail(SNN_EINVAL, "out is NULL");
-  *out = nullptr;
-  int rc = validate(n_in, n_exc, bits, p);
-  if (rc) return rc;
+}  // extern "C"
+
+namespace {
+// A network of columns [col_base, col_base + n_exc) of an n_exc_total-column network (col_base = 0,
+// n_exc_total = n_exc: an unsharded network).
+// Shards choose their launch shape from the largest shard's column groups (layout_groups) with at most
+// as many CTAs as the smallest shard has groups (cs_cap), so every shard of a world has the same
+// cluster size, CTA shape and shared-memory plan (one snn_present_many launch can hold them all).
+int create_impl(int n_in, int n_exc, int bits, const snn_params* p, int col_base, int n_exc_total, int shard,
+                int world, int layout_groups, int cs_cap, snn_handle** out) {
   snn_handle* h = new (std::nothrow) snn_handle();
   if (!h) return fail(SNN_ENOMEM, "host allocation failed");
+  int rc;
   h->p = *p;
   h->n_in = n_in; h->n_exc = n_exc; h->bits = bits;
+  h->col_base = col_base; h->n_exc_total = n_exc_total; h->shard = shard; h->world = world;
   h->frac_bits = p->frac_bits > 0 ? p->frac_bits : bits;
   h->q_max = (1 << bits) - 1;
   if (h->frac_bits != bits) {
@@ -443,8 +480,8 @@ int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** 
   for (int cs = cs_lo; cs <= cs_hi; ++cs) order.push_back(cs);
   if (ev && p->cluster_size == 0) std::reverse(order.begin(), order.end());
   for (int cs : order) {
-    if (cs > h->ngroups) continue;
-    const int max_groups = (h->ngroups + cs - 1) / cs;
+    if (cs > cs_cap) continue;
+    const int max_groups = (layout_groups + cs - 1) / cs;
     // columns per thread: 2 at 2 bits when the CTA stays <= 256 threads (measured best on C4 with
     // tools/sweep.py), else the SWAR maximum 8/bits; SNN_CPT overrides
     int cpt = 1;
@@ -493,6 +530,12 @@ int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** 
     return fail(SNN_ECOOP, "cluster of %d CTAs x %zu B smem cannot be co-resident (%s)", h->cs, h->smem,
                 cudaGetErrorString(ce));
   }
+  if (h->cs == 1) {                    // the query returned CTAs per SM
+    int sms = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->dev);
+    nclusters *= sms;
+  }
+  h->max_clusters = nclusters;
 
 #define ALLOC(ptr, n)                                                            \
   do {                                                                           \
@@ -518,6 +561,10 @@ int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** 
   ALLOC(h->d_stats, SNN_NSTATS);
   ALLOC(h->d_codes, (size_t)n_in * n_exc);
   ALLOC(h->d_bad, 1);
+  if (world > 1) {
+    ALLOC(h->d_mbox, 1);
+    ALLOC(h->d_peers, (size_t)world);
+  }
 #undef ALLOC
   if (cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking) != cudaSuccess) {
     free_all(h);
@@ -545,6 +592,7 @@ int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** 
   if (e == cudaSuccess) e = up(h->d_lpost, m1.data(), (size_t)n_exc * 4);
   if (e == cudaSuccess) e = up(h->d_lpre, m1.data(), (size_t)n_in * 4);
   if (e == cudaSuccess) e = cudaMemsetAsync(h->d_stats, 0, SNN_NSTATS * sizeof(unsigned long long), h->stream);
+  if (e == cudaSuccess && h->d_mbox) e = cudaMemsetAsync(h->d_mbox, 0, sizeof(snn::Mailbox), h->stream);
   NetDesc d;
   fill_static(h, d);
   if (e == cudaSuccess) e = snn::launch_init_weights(d, p->init_seed, h->stream);   // R4
@@ -558,11 +606,116 @@ int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** 
   *out = h;
   return SNN_OK;
 }
+}  // namespace
+
+extern "C" {
+
+int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** out) {
+  if (!out) return fail(SNN_EINVAL, "out is NULL");
+  *out = nullptr;
+  int rc = validate(n_in, n_exc, bits, p);
+  if (rc) return rc;
+  const int G = (n_exc + 31) / 32;
+  return create_impl(n_in, n_exc, bits, p, 0, n_exc, 0, 1, G, G, out);
+}
+
+int snn_create_shard(int n_in, int n_exc_total, int bits, const snn_params* p, int shard, int world,
+                     snn_handle** out) {
+  if (!out) return fail(SNN_EINVAL, "out is NULL");
+  *out = nullptr;
+  int rc = validate(n_in, n_exc_total, bits, p);
+  if (rc) return rc;
+  if (world < 1 || world > snn::kMaxWorld) return fail(SNN_EINVAL, "world=%d outside [1, %d]", world, snn::kMaxWorld);
+  if (shard < 0 || shard >= world) return fail(SNN_EINVAL, "shard=%d outside [0, %d)", shard, world);
+  if (p->engine != SNN_ENGINE_EVENT) return fail(SNN_EINVAL, "column sharding needs the event engine");
+  const int G = (n_exc_total + 31) / 32;
+  if (G < world) return fail(SNN_EINVAL, "%d column groups of 32 cannot feed %d shards", G, world);
+  const int lo = 32 * (int)(((long long)shard * G) / world);
+  const int hi = std::min(n_exc_total, 32 * (int)(((long long)(shard + 1) * G) / world));
+  return create_impl(n_in, hi - lo, bits, p, lo, n_exc_total, shard, world, (G + world - 1) / world, G / world, out);
+}
+
+int snn_shard_ipc_handle(snn_handle* h, void* out, size_t cap) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  if (h->world <= 1 || !h->d_mbox) return fail(SNN_EINVAL, "not a shard of a world > 1");
+  if (!out || cap < SNN_IPC_HANDLE_BYTES) return fail(SNN_ESIZE, "need %d bytes", SNN_IPC_HANDLE_BYTES);
+  static_assert(sizeof(cudaIpcMemHandle_t) == SNN_IPC_HANDLE_BYTES, "IPC handle size");
+  DevGuard g(h->dev);
+  cudaIpcMemHandle_t ih;
+  CUDA_TRY(cudaIpcGetMemHandle(&ih, h->d_mbox));
+  std::memcpy(out, &ih, sizeof(ih));
+  return SNN_OK;
+}
+
+int snn_shard_connect(snn_handle* h, const void* handles, size_t n_bytes) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  if (h->world <= 1 || !h->d_mbox) return fail(SNN_EINVAL, "not a shard of a world > 1");
+  if (h->connected) return fail(SNN_EINVAL, "shard already connected");
+  if (!handles || n_bytes < (size_t)h->world * SNN_IPC_HANDLE_BYTES)
+    return fail(SNN_ESIZE, "need world x %d handle bytes", SNN_IPC_HANDLE_BYTES);
+  DevGuard g(h->dev);
+  std::vector<snn::Mailbox*> peers(h->world, nullptr);
+  for (int r = 0; r < h->world; ++r) {
+    if (r == h->shard) { peers[r] = h->d_mbox; continue; }
+    cudaIpcMemHandle_t ih;
+    std::memcpy(&ih, static_cast<const char*>(handles) + (size_t)r * SNN_IPC_HANDLE_BYTES, sizeof(ih));
+    void* ptr = nullptr;
+    const cudaError_t e = cudaIpcOpenMemHandle(&ptr, ih, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      for (void* q : h->ipc_opened) cudaIpcCloseMemHandle(q);
+      h->ipc_opened.clear();
+      return fail(SNN_ECUDA, "opening the mailbox of shard %d: %s", r, cudaGetErrorString(e));
+    }
+    h->ipc_opened.push_back(ptr);
+    peers[r] = static_cast<snn::Mailbox*>(ptr);
+  }
+  CUDA_TRY(cudaMemcpy(h->d_peers, peers.data(), sizeof(void*) * h->world, cudaMemcpyHostToDevice));
+  h->connected = true;
+  return SNN_OK;
+}
+
+int snn_shard_link(snn_handle* const* hs, int world) {
+  if (!hs || world < 2) return fail(SNN_EINVAL, "need >= 2 shard handles");
+  for (int r = 0; r < world; ++r) {
+    const snn_handle* h = hs[r];
+    if (!h) return fail(SNN_EINVAL, "handle %d is NULL", r);
+    if (h->world != world || h->shard != r) return fail(SNN_EINVAL, "hs[%d] is not shard %d of %d", r, r, world);
+    if (h->connected) return fail(SNN_EINVAL, "shard %d already connected", r);
+    if (h->n_in != hs[0]->n_in || h->n_exc_total != hs[0]->n_exc_total || h->bits != hs[0]->bits)
+      return fail(SNN_EINVAL, "shards of one network must share n_in, n_exc_total, bits");
+  }
+  std::vector<snn::Mailbox*> peers(world);
+  for (int r = 0; r < world; ++r) peers[r] = hs[r]->d_mbox;
+  for (int r = 0; r < world; ++r) {
+    snn_handle* h = hs[r];
+    DevGuard g(h->dev);
+    for (int o = 0; o < world; ++o) {
+      if (hs[o]->dev == h->dev) continue;
+      int ok = 0;
+      CUDA_TRY(cudaDeviceCanAccessPeer(&ok, h->dev, hs[o]->dev));
+      if (!ok) return fail(SNN_ECUDA, "device %d cannot access device %d", h->dev, hs[o]->dev);
+      const cudaError_t e = cudaDeviceEnablePeerAccess(hs[o]->dev, 0);
+      if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) return fail(SNN_ECUDA, "%s", cudaGetErrorString(e));
+      cudaGetLastError();
+    }
+    CUDA_TRY(cudaMemcpy(h->d_peers, peers.data(), sizeof(void*) * world, cudaMemcpyHostToDevice));
+  }
+  for (int r = 0; r < world; ++r) {
+    hs[r]->linked.assign(hs, hs + world);
+    hs[r]->connected = true;
+  }
+  return SNN_OK;
+}
 
 int snn_destroy(snn_handle* h) {
   if (!h) return SNN_OK;
   DevGuard g(h->dev);
   if (h->stream) cudaStreamSynchronize(h->stream);
+  for (snn_handle* o : h->linked)      // the rest of its world can no longer run
+    if (o != h) { o->linked.clear(); o->connected = false; }
   free_all(h);
   delete h;
   return SNN_OK;
@@ -626,6 +779,17 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
       return fail(SNN_EINVAL, "ensemble handles must share n_in, cluster size, CTA shape, engine, membrane mode, device");
     for (int m = 0; m < k; ++m)
       if (hs[m] == hs[k]) return fail(SNN_EINVAL, "handle %d appears twice", k);
+    if (hs[k]->world > 1) {        // every shard of its world must be in this launch (they wait on each other)
+      if (hs[k]->linked.empty()) return fail(SNN_EINVAL, "shard handle %d is not linked in this process", k);
+      for (snn_handle* o : hs[k]->linked)
+        if (std::find(hs, hs + n, o) == hs + n) return fail(SNN_EINVAL, "handle %d: its world is incomplete", k);
+    }
+  }
+  {
+    int nsh = 0;
+    for (int k = 0; k < n; ++k) nsh += hs[k]->world > 1 ? 1 : 0;
+    if (nsh > 0 && n > hs[0]->max_clusters)
+      return fail(SNN_ECOOP, "%d networks cannot be co-resident (%d clusters fit)", n, hs[0]->max_clusters);
   }
   const bool ev = hs[0]->engine == SNN_ENGINE_EVENT;
   if (ev && T > snn::kEvMaxT) return fail(SNN_EINVAL, "T=%d exceeds %d for the event engine", T, snn::kEvMaxT);
@@ -650,6 +814,7 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
     if (!rc) {
       d.images = img; d.seeds = sd; d.raster_out = h->d_raster;
       if (ev) rc = event_prepass(h, d, img, nullptr, n_images, T, 0, sd);
+      if (!rc && ev) rc = shard_arm(h, d);
     }
     h->stream = own;
     if (rc) return rc;
@@ -885,6 +1050,7 @@ int snn_get_info(const snn_handle* h, int64_t info[SNN_NINFO]) {
   info[0] = h->cs; info[1] = h->nthr; info[2] = (int64_t)h->smem; info[3] = h->wpr;
   info[4] = h->q_max; info[5] = h->L_pot; info[6] = h->L_dep; info[7] = h->launches;
   info[8] = h->engine; info[9] = h->cpt; info[10] = h->rows_cap; info[11] = h->logn;
+  info[12] = h->col_base; info[13] = h->n_exc_total; info[14] = h->world; info[15] = h->shard;
   return SNN_OK;
 }
 

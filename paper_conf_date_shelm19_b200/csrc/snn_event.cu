@@ -324,6 +324,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwarps = nthr >> 5;
   const int g0 = (rank * d.ngroups) / cs, g1 = ((rank + 1) * d.ngroups) / cs;
   const int col0 = g0 * 32;
+  const int cbase = d.col_base;                              // global index of local column 0 (shards)
   const int ncols = min(g1 * 32, n_exc) - col0;
   // this thread's word and columns
   const int wj = tid / TPW, f = tid % TPW;
@@ -350,6 +351,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
   const bool inh_reset = d.inh_mode == 0;
   const bool keep = (flags & FLAG_KEEP_STATE) != 0;
   const int tbase = keep ? d.t0 : 0;
+  const int world = d.world;
+  const bool sharded = world > 1;
 
   // ---- one-time staging
   for (int k = tid; k < L_pot; k += nthr) s_pot[k] = d.pot_m1[k];
@@ -470,11 +473,18 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         bool done = !mycol;
         int kk = k0;
         int r0 = (int)(s_offs[k0 - ka] - wbase);
-        auto signal = [&](int fstep) {                            // tell the cluster where to stop
+        auto signal = [&](int fstep) {                            // tell the cluster (and the other shards) where to stop
           atomicMin(&s_flag[fp], fstep);
           for (int r = 0; r < cs; ++r)
             if (r != rank) red_min_cluster(&s_flag[fp], (uint32_t)r, fstep);
+          if (sharded)
+            for (int r = 0; r < world; ++r)
+              if (r != d.shard) red_min_sys(&d.peers[r]->flag[fp], fstep);
         };
+        // other shards' early-stop flag: lane 0 folds the value loaded one iteration earlier into the
+        // CTA's flag and issues the next load (its latency overlaps the iteration)
+        int gflag_next = INT_MAX;
+        if (sharded && lane == 0) gflag_next = ld_relaxed_sys_s32(&d.mbox->flag[fp]);
         long long e_int0 = prof_int, e_ltd0 = prof_ltd, e_seq0 = prof_seq, e_ev0 = prof_ev;
         if (trace && lane == 0) {
           prof_loop0 = clock64();
@@ -482,6 +492,11 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
           atomicMax(reinterpret_cast<unsigned long long*>(s_misc + 10), gt);   // latest warp loop start
         }
         while (__any_sync(FULL, !done)) {
+          if (sharded && lane == 0) {
+            if (gflag_next < INT_MAX) atomicMin(&s_flag[fp], gflag_next);
+            gflag_next = ld_relaxed_sys_s32(&d.mbox->flag[fp]);
+          }
+          __syncwarp();
           if (!done && (kk >= kend || kk > ld_volatile_shared_u32addr(flag_addr))) { done = true; p = kk; }
           if (kk >= kend) break;                                  // warp-uniform
           // ======== block path: up to kBlk steps of <= kPadRows rows each (<= 64 rows in all).
@@ -581,7 +596,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
                   for (uint32_t cm = __shfl_sync(FULL, ltd_blk, Ls); cm; cm &= cm - 1) {
                     const int c = __ffs(cm) - 1;
                     const int jlL = (tidL / TPW) * CPW + (tidL % TPW) + TPW * c;
-                    const int jL = col0 + jlL;
+                    const int jL = cbase + col0 + jlL;
                     const int lpL = s_lpost[jlL];
 #pragma unroll 1
                     for (int m = 0; m < 2; ++m) {
@@ -752,7 +767,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
               for (uint32_t cm = __shfl_sync(FULL, ltd_on, Ls); cm; cm &= cm - 1) {
                 const int c = __ffs(cm) - 1;
                 const int jlL = (tidL / TPW) * CPW + (tidL % TPW) + TPW * c;
-                const int jL = col0 + jlL;
+                const int jL = cbase + col0 + jlL;
                 const uint32_t thrL = s_dep[t - s_lpost[jlL]];
                 const int shc = fsh + c * Z::LW;
 #pragma unroll 1
@@ -836,7 +851,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
 #pragma unroll
           for (int c = 0; c < CPT; ++c) {
             if (!(cmask >> c & 1u)) continue;
-            const uint32_t h = lif.ord(v[c]), l = 0xFFFFFFFFu - (uint32_t)jcol[c];
+            const uint32_t h = lif.ord(v[c]), l = 0xFFFFFFFFu - (uint32_t)(jcol[c] + cbase);
             if (h > kh || (h == kh && l > kl)) { kh = h; kl = l; }
             ++cc;
           }
@@ -886,6 +901,39 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         const uint32_t kl = __reduce_max_sync(FULL, (at && (uint32_t)(Kr >> 32) == kh) ? (uint32_t)Kr : 0u);
         K = ((unsigned long long)kh << 32) | kl;
       }
+      if (sharded) {
+        // (e) column sharding: the cluster's summary {A, K} goes to slot [fp][shard] of every rank's
+        // mailbox (NVLink peer stores, data then a release-ordered sequence number); every warp then
+        // reads the world summaries from its own mailbox and applies the same reduction
+        const unsigned long long seq = d.seq_base + (unsigned long long)ep + 1ull;
+        if (rank == 0 && warp == 0 && lane == 0) {
+          const unsigned long long A = ((unsigned long long)W1 << 32) | count;
+          st_relaxed_sys_s32(&d.mbox->flag[fp ^ 1], INT_MAX);     // next epoch's flag (peers write it after our seq)
+          for (int r = 0; r < world; ++r) {
+            unsigned long long* sl = d.peers[r]->slot[fp][d.shard];
+            st_relaxed_sys_u64(sl, A);
+            st_relaxed_sys_u64(sl + 1, K);
+          }
+          __threadfence_system();
+          for (int r = 0; r < world; ++r) st_release_sys_u64(d.peers[r]->slot[fp][d.shard] + 2, seq);
+        }
+        unsigned long long A = 0ull, Kr = 0ull;
+        if (lane < world) {
+          const unsigned long long* sl = d.mbox->slot[fp][lane];
+          const unsigned long long t_start = globaltimer();
+          while (ld_acquire_sys_u64(sl + 2) != seq) {
+            if (globaltimer() - t_start > kShardTimeoutNs) __trap();   // a rank is gone: fail, never hang
+          }
+          A = ld_relaxed_sys_u64(sl);
+          Kr = ld_relaxed_sys_u64(sl + 1);
+        }
+        W1 = __reduce_max_sync(FULL, (uint32_t)(A >> 32));
+        const bool at = lane < world && (uint32_t)(A >> 32) == W1;
+        count = __reduce_add_sync(FULL, at ? (uint32_t)A : 0u);
+        const uint32_t kh = __reduce_max_sync(FULL, at ? (uint32_t)(Kr >> 32) : 0u);
+        const uint32_t kl = __reduce_max_sync(FULL, (at && (uint32_t)(Kr >> 32) == kh) ? (uint32_t)Kr : 0u);
+        K = ((unsigned long long)kh << 32) | kl;
+      }
       const int P = 0xFFFF - (int)(W1 >> 1);
       const bool unknown = (W1 & 1u) != 0u;
       const bool at_end = P >= kend;
@@ -920,8 +968,9 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
           const int shc = fsh + c * Z::LW;
           for (int r = r0; r < r1; ++r) {
             const int i = s_rows[r];
-            const uint4 u = philox((uint32_t)t, (uint32_t)i, (uint32_t)(jcol[c] >> 2), TAG_LTD, seed);
-            if (pick(u, jcol[c] & 3) <= thr) {
+            const int jg = jcol[c] + cbase;
+            const uint4 u = philox((uint32_t)t, (uint32_t)i, (uint32_t)(jg >> 2), TAG_LTD, seed);
+            if (pick(u, jg & 3) <= thr) {
               uint32_t* pw = wcol + i * wpr;
               if ((*pw >> shc) & FMASK) atomicSub(pw, 1u << shc);
               ++ltd_events;
@@ -983,7 +1032,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         for (int c = 0; c < CPT; ++c) {
           if (!(valid >> c & 1u)) continue;
           bool me;
-          if (hard) me = (uint32_t)jcol[c] == W;
+          if (hard) me = (uint32_t)(jcol[c] + cbase) == W;
           else me = at_p && (cmask >> c & 1u);
           if (me) { v[c] = vreset; cnt[c] = t_ref; spiked |= 1u << c; }
           if (hard ? !me : (count >= 2u || !me)) { cnt[c] = max(cnt[c], t_inh); if (inh_reset) v[c] = vreset; }
@@ -1006,7 +1055,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
             for (uint32_t cm = __shfl_sync(FULL, on, Ls); cm; cm &= cm - 1) {
               const int c = __ffs(cm) - 1;
               const int jlL = (tidL / TPW) * CPW + (tidL % TPW) + TPW * c;
-              const int jL = col0 + jlL;
+              const int jL = cbase + col0 + jlL;
               const uint32_t thrL = s_dep[tP - s_lpost[jlL]];
               const int shc = fsh + c * Z::LW;
 #pragma unroll 1
@@ -1076,7 +1125,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         for (int item = tid; item < nsp * nq4; item += nthr) {
           const int m = item / nq4, grp = item - m * nq4;
           const int jl = s_misc[16 + m];
-          const int Wg = col0 + jl;
+          const int Wg = cbase + col0 + jl;
           const int ww = jl / CPW, wsh = (jl % CPW) * BITS;
           const uint4 u = philox((uint32_t)tP, (uint32_t)Wg, (uint32_t)grp, stoch ? TAG_LTP : TAG_ROUND, seed);
 #pragma unroll

@@ -16,6 +16,8 @@ enum : uint32_t { TAG_ENC = 1, TAG_LTD = 2, TAG_LTP = 3, TAG_ROUND = 4, TAG_INIT
 enum : int { FLAG_RASTER_INPUT = 1, FLAG_KEEP_STATE = 2, FLAG_RECORD_INPUT = 4, FLAG_ASYNC = 8, FLAG_FLOOR = 16 };
 
 // Everything one network needs inside the persistent kernel.  Built per launch on the host.
+struct Mailbox;
+
 struct NetDesc {
   // geometry
   int n_in, n_exc, bits, q_max;
@@ -63,6 +65,21 @@ struct NetDesc {
   // optional per-epoch trace: [cs][trace_cap][8] u64 (%globaltimer ns)
   unsigned long long* trace;
   int trace_cap;
+  // column sharding across ranks: this network is columns [col_base, col_base + n_exc)
+  // of a network of n_exc_total; per epoch the rank summaries meet in every rank's mailbox
+  int col_base, n_exc_total, world, shard;
+  Mailbox* mbox;                  // this rank's mailbox
+  Mailbox* const* peers;          // device array [world] of every rank's mailbox (own, peer or IPC pointers)
+  unsigned long long seq_base;           // launch-unique epoch sequence base (identical on all ranks)
+};
+
+// One rank's mailbox of the column-sharded exchange: per epoch parity and source
+// rank the rank summary {A, K} and its sequence number; the early-stop flag of each parity.
+constexpr int kMaxWorld = 32;
+struct Mailbox {
+  unsigned long long slot[2][kMaxWorld][4];   // {A, K, seq, pad}
+  int flag[2];
+  int pad[30];
 };
 
 struct LaunchParams {
@@ -75,6 +92,7 @@ cudaError_t launch_present(const LaunchParams& lp, int n_nets, int cs, int nthr,
 // event engine (snn_event.cu)
 constexpr int kEvMaxThreads = 256;   // 255 registers per thread: the speculation loop keeps all its state in registers
 constexpr int kEvMaxT = 32767;
+constexpr unsigned long long kShardTimeoutNs = 20000000000ull;   // a missing rank traps after 20 s
 size_t event_smem_bytes(int n_in, int slice_words, int L_pot, int L_dep, int q_max, int nthr, int rows_cap,
                         int offs_cap, int logn);
 inline int slice_words_for(int n_in, int wpr) { return (((n_in + 1) * wpr) + 3) & ~3; }

@@ -492,7 +492,7 @@ __global__ void init_weights_kernel(const NetDesc d, unsigned long long init_see
   for (int c4 = 0; c4 < cpw; c4 += 4) {
     const int jl = w * cpw + c4;
     if (jl >= ncols) break;
-    const int jg = col0 + jl;
+    const int jg = d.col_base + col0 + jl;                  // global column (a shard starts at col_base)
     const uint4 u = philox((uint32_t)i, (uint32_t)(jg >> 2), 0u, TAG_INIT, init_seed);   // R4
 #pragma unroll
     for (int l = 0; l < 4; ++l) {

@@ -23,7 +23,10 @@ EXPORTS = [
     "snn_get_weights", "snn_set_weights", "snn_get_spikes", "snn_get_input_raster",
     "snn_state_bytes", "snn_get_state", "snn_set_state", "snn_get_stats", "snn_reset_stats",
     "snn_get_info", "snn_set_trace", "snn_get_trace", "snn_last_error",
+    "snn_create_shard", "snn_shard_ipc_handle", "snn_shard_connect", "snn_shard_link",
 ]
+SNN_IPC_HANDLE_BYTES = 64
+NINFO = 16
 
 
 class SnnParams(ctypes.Structure):
@@ -87,6 +90,10 @@ def lib():
             "snn_set_trace": ([vp, i32], i32),
             "snn_get_trace": ([vp, vp, sz], i32),
             "snn_last_error": ([], ctypes.c_char_p),
+            "snn_create_shard": ([i32, i32, i32, pp, i32, i32, ctypes.POINTER(vp)], i32),
+            "snn_shard_ipc_handle": ([vp, vp, sz], i32),
+            "snn_shard_connect": ([vp, vp, sz], i32),
+            "snn_shard_link": ([vp, i32], i32),
         }
         for name, (args, res) in sig.items():
             f = getattr(L, name)
@@ -147,13 +154,26 @@ def _ptr(x) -> ctypes.c_void_p:
 class Network:
     """One snn_handle: n_in -> n_exc network with `bits`-bit conductance codes on the GPU."""
 
-    def __init__(self, n_in: int, n_exc: int, bits: int, params: Optional[SnnParams] = None, **overrides):
+    def __init__(self, n_in: int, n_exc: int, bits: int, params: Optional[SnnParams] = None,
+                 shard: Optional[tuple] = None, **overrides):
+        """shard=(rank, world): this object is shard `rank` of an n_exc-column network split over
+        `world` ranks (include/snn.h snn_create_shard); self.n_exc becomes the shard's own columns."""
         self.n_in, self.n_exc, self.bits = n_in, n_exc, bits
         self.params = params if params is not None else preset({2: "2b", 4: "4b", 8: "8b"}[bits])
         for k, v in overrides.items():
             setattr(self.params, k, v)
         self._h = ctypes.c_void_p()
-        _check(lib().snn_create(n_in, n_exc, bits, ctypes.byref(self.params), ctypes.byref(self._h)), "snn_create")
+        if shard is None:
+            _check(lib().snn_create(n_in, n_exc, bits, ctypes.byref(self.params), ctypes.byref(self._h)), "snn_create")
+            self.col_base, self.n_exc_total = 0, n_exc
+        else:
+            rank, world = shard
+            _check(lib().snn_create_shard(n_in, n_exc, bits, ctypes.byref(self.params), rank, world,
+                                          ctypes.byref(self._h)), "snn_create_shard")
+            inf = self.info()
+            self.col_base, self.n_exc_total = inf["col_base"], inf["n_exc_total"]
+            self.n_exc = (min(self.n_exc_total, 32 * (((rank + 1) * ((n_exc + 31) // 32)) // world))
+                          - self.col_base)
         self.last_T = 0
 
     @property
@@ -172,10 +192,10 @@ class Network:
             pass
 
     def info(self) -> dict:
-        a = (ctypes.c_int64 * 12)()
+        a = (ctypes.c_int64 * NINFO)()
         _check(lib().snn_get_info(self._h, a), "snn_get_info")
         keys = ["cluster_size", "threads", "smem_bytes", "words_per_row", "q_max", "L_pot", "L_dep", "launches",
-                "engine", "cols_per_thread", "row_window", "log_depth"]
+                "engine", "cols_per_thread", "row_window", "log_depth", "col_base", "n_exc_total", "world", "shard"]
         return dict(zip(keys, [int(x) for x in a]))
 
     def set_stream(self, stream_ptr: int):
@@ -251,6 +271,23 @@ class Network:
 
     def reset_stats(self):
         _check(lib().snn_reset_stats(self._h), "snn_reset_stats")
+
+    # ---- column sharding (include/snn.h)
+    def ipc_handle(self) -> bytes:
+        buf = ctypes.create_string_buffer(SNN_IPC_HANDLE_BYTES)
+        _check(lib().snn_shard_ipc_handle(self._h, buf, SNN_IPC_HANDLE_BYTES), "snn_shard_ipc_handle")
+        return buf.raw
+
+    def connect(self, handles: Sequence[bytes]):
+        """Open every rank's mailbox (handles in rank order, this rank's own included)."""
+        blob = b"".join(handles)
+        _check(lib().snn_shard_connect(self._h, ctypes.c_char_p(blob), len(blob)), "snn_shard_connect")
+
+
+def link_shards(shards: Sequence[Network]):
+    """Single process: link shards 0..world-1 of one network (include/snn.h snn_shard_link)."""
+    hs = (ctypes.c_void_p * len(shards))(*[x.handle.value for x in shards])
+    _check(lib().snn_shard_link(hs, len(shards)), "snn_shard_link")
 
 
 def present_many(nets: Sequence[Network], images: Sequence, T: int, seeds: Sequence):
