@@ -8,8 +8,13 @@ membranes.  A "step" = one snn_present_batch launch presenting B images back to 
 learning: the images of a step are sequential by construction).  value = training images/s with
 inputs resident in HBM; secondary = synaptic events/s (sum_t act(t) * n_exc).
 
-Multi-GPU (torchrun, N > 1): one independent network per GPU (replicas, "scaling": "weak"); no
-data-path collective -- one network's steps are strictly sequential.
+Multi-GPU (torchrun, N > 1), --mode:
+  replicas (default): one independent network per GPU, no data-path collective ("scaling": "weak");
+  shard: ONE network whose 6400 columns are split over the N GPUs (include/snn.h snn_create_shard):
+         per post-spike epoch the shards exchange 16-byte summaries through CUDA-IPC mailboxes over
+         NVLink ("scaling": "strong": every rank presents the same images).
+--local-shards K (N = 1): the one network split into K shards on this GPU, presented in one launch
+(K clusters exchanging through L2 mailboxes) -- more SMs per network.
 
 --impl reference: the CPU oracle (oracle/) as it stands, single-threaded, timed on the host.
 """
@@ -150,6 +155,8 @@ def main():
     ap.add_argument("--cpu-images", type=int, default=10, help="oracle images for cpu_baseline (0 = skip)")
     ap.add_argument("--no-floor", action="store_true")
     ap.add_argument("--engine", type=int, default=0, help="0 event-driven epochs, 1 per-step exchange")
+    ap.add_argument("--mode", default="replicas", choices=["replicas", "shard"], help="N > 1 layout")
+    ap.add_argument("--local-shards", type=int, default=1, help="shards of the network on this GPU (N = 1)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -178,16 +185,45 @@ def main():
     torch.cuda.set_stream(stream)
 
     B = args.images_per_step
-    params = P.preset("2b", membrane_mode=args.membrane, init_seed=1 + rank, cluster_size=args.cluster_size,
-                      engine=args.engine)
-    net = P.Network(N_IN, N_EXC, BITS, params)
-    net.set_stream(stream.cuda_stream)
+    sharded = ws > 1 and args.mode == "shard"
+    K = args.local_shards if ws == 1 else 1
+    net_rank = 0 if sharded else rank           # shards of one network share seeds and images
+
+    def make_runner():
+        """-> (present(imgs, seeds, counts, flags), stats(), nets) for the configured layout."""
+        params = P.preset("2b", membrane_mode=args.membrane, init_seed=1 + net_rank,
+                          cluster_size=args.cluster_size, engine=args.engine)
+        if sharded:
+            n = P.Network(N_IN, N_EXC, BITS, params, shard=(rank, ws))
+            n.set_stream(stream.cuda_stream)
+            hs = [None] * ws
+            dist.all_gather_object(hs, n.ipc_handle())
+            n.connect(hs)
+            nets = [n]
+        elif K > 1:
+            nets = [P.Network(N_IN, N_EXC, BITS, params, shard=(r, K)) for r in range(K)]
+            P.link_shards(nets)
+            for n in nets:
+                n.set_stream(stream.cuda_stream)
+        else:
+            nets = [P.Network(N_IN, N_EXC, BITS, params)]
+            nets[0].set_stream(stream.cuda_stream)
+        if K > 1:
+            def present(imgs, seeds, counts, flags=0):
+                P.present_many(nets, [imgs] * K, T_STEPS, [seeds] * K)
+        else:
+            def present(imgs, seeds, counts, flags=0):
+                nets[0].present_batch(imgs, T_STEPS, seeds, counts, flags=flags)
+        return present, nets
+
+    present, nets = make_runner()
+    net = nets[0]
     info = net.info()
 
     n_steps_total = args.warmup + args.steps
     pool_n = B * n_steps_total
-    imgs_h = synthdata.images(pool_n, "fashion", start=rank * 100000)
-    seeds_h = synthdata.seeds(pool_n, base_seed=1 + rank)
+    imgs_h = synthdata.images(pool_n, "fashion", start=net_rank * 100000)
+    seeds_h = synthdata.seeds(pool_n, base_seed=1 + net_rank)
     imgs_d = torch.from_numpy(imgs_h).to(dev)
     seeds_d = torch.from_numpy(seeds_h.view(np.int64)).to(dev)
     counts_d = torch.zeros(pool_n, dtype=torch.int32, device=dev)
@@ -195,13 +231,14 @@ def main():
 
     def step(k, flags=0):
         sl = slice(k * B, (k + 1) * B)
-        net.present_batch(imgs_d[sl], T_STEPS, seeds_d[sl], counts_d[sl], flags=flags | P.SNN_ASYNC)
+        present(imgs_d[sl], seeds_d[sl], counts_d[sl], flags | P.SNN_ASYNC)
 
     for k in range(args.warmup):
         step(k)
     torch.cuda.synchronize()
-    net.reset_stats()
-    launches0 = net.info()["launches"]
+    for n in nets:
+        n.reset_stats()
+    launches0 = sum(n.info()["launches"] for n in nets)
 
     # ---- timed region: device time per step (CUDA events on the launching stream), L2 flushed between steps
     sampler = ClockSampler(local)
@@ -223,7 +260,9 @@ def main():
     step_ms = [a.elapsed_time(b) for a, b in ev]
     dev_s = sum(step_ms) / 1e3
     stats = net.stats()
-    launches = net.info()["launches"] - launches0
+    for n in nets[1:]:                 # per-shard trial / event counters add up; [0], [1], [6..8] are network-wide
+        stats[2:6] += n.stats()[2:6]
+    launches = sum(n.info()["launches"] for n in nets) - launches0
     images = B * args.steps
     events = int(stats[0]) * N_EXC
     # max over ranks of the device time
@@ -231,9 +270,10 @@ def main():
         t = torch.tensor([dev_s], device=coll_dev, dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         dev_s = float(t.item())
-        tot = torch.tensor([images, events], device=coll_dev, dtype=torch.float64)
-        dist.all_reduce(tot, op=dist.ReduceOp.SUM)
-        images, events = int(tot[0].item()), int(tot[1].item())
+        if not sharded:                # replicas: every rank trained its own network on its own images
+            tot = torch.tensor([images, events], device=coll_dev, dtype=torch.float64)
+            dist.all_reduce(tot, op=dist.ReduceOp.SUM)
+            images, events = int(tot[0].item()), int(tot[1].item())
     value = images / dev_s
     ev_rate = events / dev_s
 
@@ -266,13 +306,15 @@ def main():
     imgs_pin = torch.from_numpy(imgs_h).pin_memory()
     seeds_pin = torch.from_numpy(seeds_h.view(np.int64)).pin_memory()
     counts_pin = torch.zeros(pool_n, dtype=torch.int32).pin_memory()
-    net2_params = P.preset("2b", membrane_mode=args.membrane, init_seed=1 + rank, cluster_size=args.cluster_size,
-                      engine=args.engine)
-    net2 = P.Network(N_IN, N_EXC, BITS, net2_params)
-    net2.set_stream(stream.cuda_stream)
+    present2, nets2 = make_runner()
+    d2h = B * 4 if K == 1 else 16 * 8
+
+    def step2(sl):
+        present2(imgs_pin[sl], seeds_pin[sl], counts_pin[sl])
+        if K > 1:                      # synchronous present_many: read the post-spike counter back
+            nets2[0].stats()
     for k in range(args.warmup):
-        sl = slice(k * B, (k + 1) * B)
-        net2.present_batch(imgs_pin[sl], T_STEPS, seeds_pin[sl], counts_pin[sl])
+        step2(slice(k * B, (k + 1) * B))
     if dist:
         dist.barrier()
     torch.cuda.synchronize()
@@ -280,15 +322,15 @@ def main():
     for i in range(args.steps):
         k = args.warmup + i
         sl = slice(k * B, (k + 1) * B)
-        net2.present_batch(imgs_pin[sl], T_STEPS, seeds_pin[sl], counts_pin[sl])   # synchronous: result on host
+        step2(sl)                      # synchronous: result on host
     torch.cuda.synchronize()
     e2e_s = time.perf_counter() - t0
     if dist:
         t = torch.tensor([e2e_s], device=coll_dev, dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_s = float(t.item())
-    e2e = {"value": images / e2e_s, "unit": "images/s", "h2d_bytes_per_step": B * (N_IN + 8),
-           "d2h_bytes_per_step": B * 4, "timing": "host wall clock around synchronous snn_present_batch calls"}
+    e2e = {"value": images / e2e_s, "unit": "images/s", "h2d_bytes_per_step": B * (N_IN + 8) * K,
+           "d2h_bytes_per_step": d2h, "timing": "host wall clock around synchronous presentation calls"}
 
     # ---- roofline of the dominant kernel (present_kernel; one launch per step)
     bits_b = BITS / 8.0
@@ -309,9 +351,12 @@ def main():
     line = {
         "metric": METRIC, "value": value, "unit": "images/s", "n_gpus": ws, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": 1e3 * dev_s / args.steps, "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "f32/u2", "data": "synthetic",
+        "scaling": "strong" if sharded else "weak", "vs_baseline": None, "dtype": "f32/u2", "data": "synthetic",
         "config": {"workload": WORKLOAD, "n_in": N_IN, "n_exc": N_EXC, "bits": BITS, "T": T_STEPS,
-                   "images_per_step": B, "parallelism": f"replicas x{ws}" if ws > 1 else "1 network / 1 GPU",
+                   "images_per_step": B,
+                   "parallelism": (f"1 network column-sharded over {ws} GPUs" if sharded else
+                                   f"replicas x{ws}" if ws > 1 else
+                                   f"1 network in {K} shards on 1 GPU" if K > 1 else "1 network / 1 GPU"),
                    "cluster_size": info["cluster_size"], "threads_per_cta": info["threads"],
                    "smem_bytes_per_cta": info["smem_bytes"],
                    "l2": "flushed between timed steps (256 MiB write)", "membrane": "fp32" if args.membrane == 0 else "Q15.16"},

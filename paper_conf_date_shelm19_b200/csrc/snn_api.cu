@@ -114,7 +114,6 @@ struct snn_handle {
   std::vector<void*> ipc_opened;       // peer mailboxes opened with cudaIpcOpenMemHandle
   std::vector<snn_handle*> linked;     // in-process shards (snn_shard_link), rank order
   bool connected = false;
-  unsigned long long shard_launches = 0;
 };
 
 namespace {
@@ -182,16 +181,12 @@ void fill_static(const snn_handle* h, NetDesc& d) {
   d.col_base = h->col_base; d.n_exc_total = h->n_exc_total; d.world = 1; d.shard = h->shard;
 }
 
-// Sharded launch fields: mailbox, peers and a launch-unique sequence base (all shards count the
-// same presentation calls, so the base agrees across ranks); this rank's early-stop flags are
-// cleared before the launch.
+// Sharded launch fields: this rank's mailbox and every rank's.
 int shard_arm(snn_handle* h, NetDesc& d) {
   if (h->world <= 1) return SNN_OK;
   if (!h->connected) return fail(SNN_EINVAL, "shard %d of %d is not connected (snn_shard_connect / snn_shard_link)",
                                  h->shard, h->world);
   d.world = h->world; d.shard = h->shard; d.mbox = h->d_mbox; d.peers = h->d_peers;
-  d.seq_base = (++h->shard_launches) << 32;
-  CUDA_TRY(cudaMemsetAsync(&h->d_mbox->flag[0], 0x7F, 2 * sizeof(int), h->stream));
   return SNN_OK;
 }
 

@@ -353,6 +353,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
   const int tbase = keep ? d.t0 : 0;
   const int world = d.world;
   const bool sharded = world > 1;
+  // epoch numbering of the shard exchange: continues the previous launch's count
+  const uint32_t seq0 = sharded ? (uint32_t)ld_relaxed_sys_s32(reinterpret_cast<const int*>(&d.mbox->seq)) : 0u;
 
   // ---- one-time staging
   for (int k = tid; k < L_pot; k += nthr) s_pot[k] = d.pot_m1[k];
@@ -449,6 +451,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
       }
       const int kend = kb;
       const int fp = ep & 1;
+      const uint32_t cur = seq0 + (uint32_t)ep + 1u;        // shard-exchange epoch number (never 0 in use)
       if (trace && tid == 0) {
         tr0 = globaltimer(); *s_tmax = 0ull; s_misc[3] = 0;
         *reinterpret_cast<unsigned long long*>(s_misc + 10) = 0ull;
@@ -477,14 +480,16 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
           atomicMin(&s_flag[fp], fstep);
           for (int r = 0; r < cs; ++r)
             if (r != rank) red_min_cluster(&s_flag[fp], (uint32_t)r, fstep);
-          if (sharded)
+          if (sharded) {
+            const unsigned long long fv = ((unsigned long long)cur << 32) | (0xFFFFFFFFu - (uint32_t)fstep);
             for (int r = 0; r < world; ++r)
-              if (r != d.shard) red_min_sys(&d.peers[r]->flag[fp], fstep);
+              if (r != d.shard) red_max_sys_u64(&d.peers[r]->flag, fv);
+          }
         };
         // other shards' early-stop flag: lane 0 folds the value loaded one iteration earlier into the
         // CTA's flag and issues the next load (its latency overlaps the iteration)
-        int gflag_next = INT_MAX;
-        if (sharded && lane == 0) gflag_next = ld_relaxed_sys_s32(&d.mbox->flag[fp]);
+        unsigned long long gflag_next = 0ull;
+        if (sharded && lane == 0) gflag_next = ld_relaxed_sys_u64(&d.mbox->flag);
         long long e_int0 = prof_int, e_ltd0 = prof_ltd, e_seq0 = prof_seq, e_ev0 = prof_ev;
         if (trace && lane == 0) {
           prof_loop0 = clock64();
@@ -493,8 +498,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         }
         while (__any_sync(FULL, !done)) {
           if (sharded && lane == 0) {
-            if (gflag_next < INT_MAX) atomicMin(&s_flag[fp], gflag_next);
-            gflag_next = ld_relaxed_sys_s32(&d.mbox->flag[fp]);
+            if ((uint32_t)(gflag_next >> 32) == cur) atomicMin(&s_flag[fp], (int)(0xFFFFFFFFu - (uint32_t)gflag_next));
+            gflag_next = ld_relaxed_sys_u64(&d.mbox->flag);
           }
           __syncwarp();
           if (!done && (kk >= kend || kk > ld_volatile_shared_u32addr(flag_addr))) { done = true; p = kk; }
@@ -902,37 +907,49 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         K = ((unsigned long long)kh << 32) | kl;
       }
       if (sharded) {
-        // (e) column sharding: the cluster's summary {A, K} goes to slot [fp][shard] of every rank's
-        // mailbox (NVLink peer stores, data then a release-ordered sequence number); every warp then
-        // reads the world summaries from its own mailbox and applies the same reduction
-        const unsigned long long seq = d.seq_base + (unsigned long long)ep + 1ull;
-        if (rank == 0 && warp == 0 && lane == 0) {
-          const unsigned long long A = ((unsigned long long)W1 << 32) | count;
-          st_relaxed_sys_s32(&d.mbox->flag[fp ^ 1], INT_MAX);     // next epoch's flag (peers write it after our seq)
-          for (int r = 0; r < world; ++r) {
-            unsigned long long* sl = d.peers[r]->slot[fp][d.shard];
-            st_relaxed_sys_u64(sl, A);
-            st_relaxed_sys_u64(sl + 1, K);
-          }
-          __threadfence_system();
-          for (int r = 0; r < world; ++r) st_release_sys_u64(d.peers[r]->slot[fp][d.shard] + 2, seq);
+        // (e) column sharding: the cluster's summary {A, K} goes to slot [cur & 1][shard] of every rank's
+        // mailbox as four LL words (NVLink peer stores); warp 0 of every CTA reads the world's summaries
+        // from its own mailbox and applies the same reduction as the cluster exchange
+        const int mp = (int)(cur & 1u);
+        const unsigned long long tag = (unsigned long long)cur << 32;
+        if (rank == 0 && warp == 0 && lane < world) {           // lane r -> rank r: four LL words, no fence
+          unsigned long long* sl = d.peers[lane]->slot[mp][d.shard];
+          st_relaxed_sys_u64(sl, tag | W1);
+          st_relaxed_sys_u64(sl + 1, tag | count);
+          st_relaxed_sys_u64(sl + 2, tag | (uint32_t)(K >> 32));
+          st_relaxed_sys_u64(sl + 3, tag | (uint32_t)K);
         }
-        unsigned long long A = 0ull, Kr = 0ull;
-        if (lane < world) {
-          const unsigned long long* sl = d.mbox->slot[fp][lane];
-          const unsigned long long t_start = globaltimer();
-          while (ld_acquire_sys_u64(sl + 2) != seq) {
-            if (globaltimer() - t_start > kShardTimeoutNs) __trap();   // a rank is gone: fail, never hang
+        if (warp == 0) {                                           // warp 0 polls; the CTA reads its result
+          unsigned long long A = 0ull, Kr = 0ull;
+          if (lane < world) {
+            const unsigned long long* sl = d.mbox->slot[mp][lane];
+            const unsigned long long t_start = globaltimer();
+            unsigned long long w0, w1, w2, w3;
+            while (true) {
+              w0 = ld_relaxed_sys_u64(sl); w1 = ld_relaxed_sys_u64(sl + 1);
+              w2 = ld_relaxed_sys_u64(sl + 2); w3 = ld_relaxed_sys_u64(sl + 3);
+              if ((uint32_t)(w0 >> 32) == cur && (uint32_t)(w1 >> 32) == cur && (uint32_t)(w2 >> 32) == cur &&
+                  (uint32_t)(w3 >> 32) == cur) break;
+              if (globaltimer() - t_start > kShardTimeoutNs) __trap();   // a rank is gone: fail, never hang
+            }
+            A = ((unsigned long long)(uint32_t)w0 << 32) | (uint32_t)w1;
+            Kr = ((unsigned long long)(uint32_t)w2 << 32) | (uint32_t)w3;
           }
-          A = ld_relaxed_sys_u64(sl);
-          Kr = ld_relaxed_sys_u64(sl + 1);
+          const uint32_t W1g = __reduce_max_sync(FULL, (uint32_t)(A >> 32));
+          const bool at = lane < world && (uint32_t)(A >> 32) == W1g;
+          const uint32_t cg = __reduce_add_sync(FULL, at ? (uint32_t)A : 0u);
+          const uint32_t kh = __reduce_max_sync(FULL, at ? (uint32_t)(Kr >> 32) : 0u);
+          const uint32_t kl = __reduce_max_sync(FULL, (at && (uint32_t)(Kr >> 32) == kh) ? (uint32_t)Kr : 0u);
+          if (lane == 0) {     // s_wsum is free here: the CTA summary was consumed before the cluster exchange
+            s_wsum[0] = ((unsigned long long)W1g << 32) | cg;
+            s_wsum[1] = ((unsigned long long)kh << 32) | kl;
+          }
         }
-        W1 = __reduce_max_sync(FULL, (uint32_t)(A >> 32));
-        const bool at = lane < world && (uint32_t)(A >> 32) == W1;
-        count = __reduce_add_sync(FULL, at ? (uint32_t)A : 0u);
-        const uint32_t kh = __reduce_max_sync(FULL, at ? (uint32_t)(Kr >> 32) : 0u);
-        const uint32_t kl = __reduce_max_sync(FULL, (at && (uint32_t)(Kr >> 32) == kh) ? (uint32_t)Kr : 0u);
-        K = ((unsigned long long)kh << 32) | kl;
+        __syncthreads();
+        W1 = (uint32_t)(s_wsum[0] >> 32);
+        count = (uint32_t)s_wsum[0];
+        K = s_wsum[1];
+        if (trace && tid == 0) tr3 = globaltimer();            // sharded: "exchanged" = after the world exchange
       }
       const int P = 0xFFFF - (int)(W1 >> 1);
       const bool unknown = (W1 & 1u) != 0u;
@@ -1241,6 +1258,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
     rec[6] = (unsigned long long)(clock64() - prof_clk0); rec[7] = globaltimer() - prof_ns0;
   }
   if (cs > 1) { cluster_arrive(); cluster_wait(); }
+  else if (sharded) __syncthreads();
+  if (sharded && rank == 0 && tid == 0) d.mbox->seq = seq0 + (uint32_t)ep;   // every CTA read seq0 long ago
 }
 
 // ====================================================================== host launchers

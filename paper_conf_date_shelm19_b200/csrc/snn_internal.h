@@ -70,16 +70,21 @@ struct NetDesc {
   int col_base, n_exc_total, world, shard;
   Mailbox* mbox;                  // this rank's mailbox
   Mailbox* const* peers;          // device array [world] of every rank's mailbox (own, peer or IPC pointers)
-  unsigned long long seq_base;           // launch-unique epoch sequence base (identical on all ranks)
 };
 
-// One rank's mailbox of the column-sharded exchange: per epoch parity and source
-// rank the rank summary {A, K} and its sequence number; the early-stop flag of each parity.
+// One rank's mailbox of the column-sharded exchange.  Epochs are numbered by a
+// per-shard counter that persists across launches (`seq`, identical on every shard because the
+// epoch sequence is).  slot[seq & 1][r] holds rank r's summary of epoch seq as four LL words
+// {data32 | seq32 << 32} (W1, count, key hi, key lo): a reader spins until all four carry seq, so
+// no fence is needed and a stale word can never pass (slots are rewritten every second epoch).
+// flag = max over signals of (seq << 32 | ~step): the earliest crossing step reported for epoch
+// seq by another shard (values of older epochs lose the max and are ignored).
 constexpr int kMaxWorld = 32;
 struct Mailbox {
-  unsigned long long slot[2][kMaxWorld][4];   // {A, K, seq, pad}
-  int flag[2];
-  int pad[30];
+  unsigned long long slot[2][kMaxWorld][4];
+  unsigned long long flag;
+  unsigned int seq;               // epochs completed by this shard (written at the end of each launch)
+  unsigned int pad[29];
 };
 
 struct LaunchParams {
