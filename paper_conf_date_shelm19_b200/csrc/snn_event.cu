@@ -206,35 +206,21 @@ __device__ __forceinline__ uint32_t vmax_lanes(uint32_t a, uint32_t b) {
 }
 
 
-// After an applied LTD decrement of row i at block step b (or its undo), add `delta` (one LSB of the
-// column's SWAR lane, two's complement for -1) to the running-sum slot of every later block step at
-// or after the first later step whose rows contain i, and to every later non-empty slot after it.
-// Rows r in [rlo, rhi) belong to steps > b (ascending).  Slots of empty steps stay 0.
-template <int CPT>
-__device__ __forceinline__ void block_correct(const uint16_t* __restrict__ rows, const uint16_t* __restrict__ rstep,
-                                              uint32_t* my_acc, int nthr, int rlo, int rhi, int sbase, int b, int nb,
-                                              int i, uint32_t delta) {
-  int first = nb;
-  for (int r = rlo; r < rhi && first == nb; r += 8) {
-    uint32_t rv[8];
-#pragma unroll
-    for (int x = 0; x < 8; ++x) rv[x] = r + x < rhi ? (uint32_t)rows[r + x] : 0xFFFFFFFFu;
-#pragma unroll
-    for (int x = 0; x < 8; ++x)
-      if (rv[x] == (uint32_t)i && first == nb) first = (int)(rstep[r + x] & 0x7FFFu) - sbase;
-  }
-  if (first >= nb) return;
-  // each occurrence of i at step s2 lowers the running sums of every step >= s2: walk the later rows once
-  uint32_t cum = 0u;
-  int rr = rlo;
-  for (int b2 = b + 1; b2 < nb; ++b2) {
-    bool nonempty = false;
-    while (rr < rhi && (int)(rstep[rr] & 0x7FFFu) - sbase == b2) {
-      if ((uint32_t)rows[rr] == (uint32_t)i) cum += delta;
-      nonempty = true;
-      ++rr;
-    }
-    if (nonempty && cum) my_acc[b2 * nthr] += cum;
+// LTD decrement of the row at window position r (step b of the block): the later block steps that
+// contain the same input were summed with the old code, so every later occurrence q (followed through
+// the next-occurrence links in bits 9..15 of rstep) lowers the running sums of every non-empty block
+// step >= step(q) by delta.  Slots of empty steps stay 0 (the LIF chain reads them through vmax).
+__device__ __forceinline__ void block_correct(const uint16_t* __restrict__ rstep, uint32_t* my_acc, int nthr, int r,
+                                              int rblk1, int sbase, uint32_t nonempty, uint32_t delta) {
+  uint32_t lk = (uint32_t)rstep[r] >> 9;
+  int q = r + (int)lk;
+  while (lk != 0u && q < rblk1) {
+    const uint32_t rs = rstep[q];
+    const int s2 = (int)(rs & 0x1FFu) - sbase;
+#pragma unroll 1
+    for (uint32_t m = nonempty & (0xFFFFFFFFu << s2); m; m &= m - 1u) my_acc[(__ffs(m) - 1) * nthr] += delta;
+    lk = rs >> 9;
+    q += (int)lk;
   }
 }
 
@@ -438,14 +424,14 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         for (int x = tid; x < nsteps; x += nthr)
           for (uint32_t r = s_offs[x] - wbase; r < s_offs[x + 1] - wbase; ++r) s_rstep[r] = (uint16_t)x;
         __syncthreads();
-        // bit 15 of s_rstep[r]: the same input occurs again within the next 64 rows (a block holds <= 64
-        // rows, so an LTD decrement of row r can only need corrections of later block steps if set)
+        // bits 9..15 of s_rstep[r]: distance to the next occurrence of the same input within the next 64
+        // rows, 0 if none (a block holds <= 64 rows; LTD corrections follow these links, block_correct)
         for (uint32_t x = tid; x < nrows; x += nthr) {
           const uint16_t id = s_rows[x];
-          bool dup = false;
+          uint32_t link = 0;
           const uint32_t lim = min(nrows, x + 65u);
-          for (uint32_t y = x + 1; y < lim && !dup; ++y) dup = s_rows[y] == id;
-          if (dup) s_rstep[x] = (uint16_t)(s_rstep[x] | 0x8000u);
+          for (uint32_t y = x + 1; y < lim && !link; ++y) if (s_rows[y] == id) link = y - x;
+          if (link) s_rstep[x] = (uint16_t)(s_rstep[x] | (link << 9));
         }
         __syncthreads();
       }
@@ -512,9 +498,21 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
           // the same row (exact: the sum was taken with the pre-decrement code).
           {
             int nb = 0;
+            uint32_t nonempty = 0u;                            // block steps with >= 1 active row
+            {
+              int prev = r0;
 #pragma unroll
-            for (int b = 0; b < kBlk; ++b)
-              if (nb == b && kk + b < kend && (int)(s_offs[kk - ka + b + 1] - wbase) - r0 <= 64) nb = b + 1;
+              for (int b = 0; b < kBlk; ++b) {
+                if (nb == b && kk + b < kend) {
+                  const int o = (int)(s_offs[kk - ka + b + 1] - wbase);
+                  if (o - r0 <= 64) {
+                    nb = b + 1;
+                    if (o != prev) nonempty |= 1u << b;
+                    prev = o;
+                  }
+                }
+              }
+            }
             if (nb > 0) {
               const int kb0 = kk;
               const bool prof = trace && lane == 0;
@@ -567,7 +565,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
                   for (int x = 0; x < 8; ++x) {
                     const bool in = r + x < rblk1;
                     o[x] = in ? s_woff[r + x] : (uint32_t)(n_in * wpr);   // the all-zero row
-                    st[x] = in ? (uint32_t)(s_rstep[r + x] & 0x7FFFu) : 0xFFFFu;
+                    st[x] = in ? (uint32_t)(s_rstep[r + x] & 0x1FFu) : 0xFFFFu;
                   }
 #pragma unroll
                   for (int x = 0; x < 8; ++x) w[x] = (wcol[o[x]] >> fsh) & Z::LMASK;
@@ -589,8 +587,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
               const int nrows_blk = rblk1 - rblk0;
               if (__any_sync(FULL, ltd_blk != 0)) {
                 // this lane's rows of the block and their steps (the same for every pair)
-                const int bsel0 = lane < nrows_blk ? (int)(s_rstep[rblk0 + lane] & 0x7FFFu) - (kb0 - ka) : 0;
-                const int bsel1 = lane + 32 < nrows_blk ? (int)(s_rstep[rblk0 + 32 + lane] & 0x7FFFu) - (kb0 - ka) : 0;
+                const int bsel0 = lane < nrows_blk ? (int)(s_rstep[rblk0 + lane] & 0x1FFu) - (kb0 - ka) : 0;
+                const int bsel1 = lane + 32 < nrows_blk ? (int)(s_rstep[rblk0 + 32 + lane] & 0x1FFu) - (kb0 - ka) : 0;
                 const uint32_t row0 = lane < nrows_blk ? (uint32_t)s_rows[rblk0 + lane] : 0u;
                 const uint32_t row1 = lane + 32 < nrows_blk ? (uint32_t)s_rows[rblk0 + 32 + lane] : 0u;
 #pragma unroll 1
@@ -684,8 +682,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
                         if (applied) {
                           atomicSub(pw, 1u << shc);
                           // the later block steps that contain row i were summed with the old code
-                          if (s_rstep[rlo + xr] & 0x8000u) block_correct<CPT>(s_rows, s_rstep, my_acc, nthr, rhi, rblk1, kb0 - ka, b, nb, i,
-                                             0u - (1u << (c * Z::LW)));
+                          if (s_rstep[rlo + xr] >> 9)
+                            block_correct(s_rstep, my_acc, nthr, rlo + xr, rblk1, kb0 - ka, nonempty, 0u - (1u << (c * Z::LW)));
                         }
                         ++ev_step;
                         if (kk_b > k0) s_log[nlog++ * nthr + tid] = log_entry(kk_b - k0, c, applied, i);
@@ -697,8 +695,9 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
                         const int i = (int)(e & 0x1FFFu), c = (int)((e >> 14) & 3u);
                         if (e & 0x2000u) {
                           atomicAdd(wcol + i * wpr, 1u << (fsh + c * Z::LW));
-                          block_correct<CPT>(s_rows, s_rstep, my_acc, nthr, rhi, rblk1, kb0 - ka, b, nb, i,
-                                             1u << (c * Z::LW));
+                          int rpos = rlo;                             // the event's row position in step b
+                          while (rpos < rhi - 1 && (int)s_rows[rpos] != i) ++rpos;
+                          block_correct(s_rstep, my_acc, nthr, rpos, rblk1, kb0 - ka, nonempty, 1u << (c * Z::LW));
                         }
                         --nlog;
                       }
