@@ -22,6 +22,11 @@
 #include <climits>
 #include <cstdint>
 
+// ablation switch for timing experiments only (tools/ablate.sh); 0 in every shipped build
+#ifndef SNN_EXP
+#define SNN_EXP 0
+#endif
+
 namespace snn {
 
 // ====================================================================== pre-pass 1: encoder (a1)
@@ -206,26 +211,33 @@ __device__ __forceinline__ uint32_t vmax_lanes(uint32_t a, uint32_t b) {
 }
 
 
+// Window row metadata (one u32 per active row): word offset row*wpr (bits 0..15; the slice holds
+// < 2^16 words), step within the window (bits 16..24), distance to the next occurrence of the same
+// input within the next 64 rows (bits 25..31, 0 = none).
+__device__ __forceinline__ uint32_t meta_woff(uint32_t m) { return m & 0xFFFFu; }
+__device__ __forceinline__ int meta_step(uint32_t m) { return (int)((m >> 16) & 0x1FFu); }
+__device__ __forceinline__ uint32_t meta_link(uint32_t m) { return m >> 25; }
+
 // LTD decrement of the row at window position r (step b of the block): the later block steps that
 // contain the same input were summed with the old code, so every later occurrence q (followed through
-// the next-occurrence links in bits 9..15 of rstep) lowers the running sums of every non-empty block
-// step >= step(q) by delta.  Slots of empty steps stay 0 (the LIF chain reads them through vmax).
-__device__ __forceinline__ void block_correct(const uint16_t* __restrict__ rstep, uint32_t* my_acc, int nthr, int r,
+// the next-occurrence links) lowers the running sums of every non-empty block step >= step(q) by
+// delta (the LIF chain reads only the slots of non-empty steps).
+__device__ __forceinline__ void block_correct(const uint32_t* __restrict__ meta, uint32_t* my_acc, int nthr, int r,
                                               int rblk1, int sbase, uint32_t nonempty, uint32_t delta) {
-  uint32_t lk = (uint32_t)rstep[r] >> 9;
+  uint32_t lk = meta_link(meta[r]);
   int q = r + (int)lk;
   while (lk != 0u && q < rblk1) {
-    const uint32_t rs = rstep[q];
-    const int s2 = (int)(rs & 0x1FFu) - sbase;
+    const uint32_t rs = meta[q];
+    const int s2 = meta_step(rs) - sbase;
 #pragma unroll 1
     for (uint32_t m = nonempty & (0xFFFFFFFFu << s2); m; m &= m - 1u) my_acc[(__ffs(m) - 1) * nthr] += delta;
-    lk = rs >> 9;
+    lk = meta_link(rs);
     q += (int)lk;
   }
 }
 
 struct EvLayout {
-  size_t slots, wsum, flags, misc, w, pot, dep, dbp, dbd, dtp, dtd, lpre, lpost, offs, rows, rows16, rstep, ev, acc, log, total;
+  size_t slots, wsum, flags, misc, w, pot, dep, dbp, dbd, dtp, dtd, lpre, lpost, offs, binfo, rows, meta, ev, acc, log, total;
 };
 
 __host__ __device__ inline EvLayout ev_layout(int n_in, int slice_words, int L_pot, int L_dep, int q_max, int nthr,
@@ -246,11 +258,11 @@ __host__ __device__ inline EvLayout ev_layout(int n_in, int slice_words, int L_p
   L.lpre = o;   o = align16(o + (size_t)n_in * 4);
   L.lpost = o;  o = align16(o + (size_t)nthr * 4 * 4);        // last_post of the CTA's local columns
   L.offs = o;   o = align16(o + (size_t)(offs_cap + 1) * 4);
-  L.rows = o;   o = align16(o + (size_t)rows_cap * 2);
-  L.rows16 = o; o = align16(o + (size_t)rows_cap * 4);               // word offset (row * wpr) of every window row
-  L.rstep = o;  o = align16(o + (size_t)rows_cap * 2);               // step (relative to the window) of every row
+  L.binfo = o;  o = align16(o + (size_t)offs_cap * 4);               // block shape from every window step
+  L.rows = o;   o = align16(o + (size_t)(rows_cap + 2) * 2);         // input id of every window row (+ pad)
+  L.meta = o;   o = align16(o + (size_t)(rows_cap + 8) * 4);         // row metadata (+ 8 zero-row pads)
   L.ev = o;     o = align16(o + (size_t)8 * nthr * 4);               // block LTD event masks [c][2][thread]
-  L.acc = o;    o = align16(o + (size_t)kBlk * nthr * 4);            // block SWAR sums [b][thread]
+  L.acc = o;    o = align16(o + (size_t)(kBlk + 1) * nthr * 4);      // block SWAR sums [b][thread] + spill slot
   L.log = o;    o = align16(o + (size_t)logn * nthr * 4);
   L.total = o;
   return L;
@@ -300,9 +312,9 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
   int* s_lpre = reinterpret_cast<int*>(smem + L.lpre);
   int* s_lpost = reinterpret_cast<int*>(smem + L.lpost);
   uint32_t* s_offs = reinterpret_cast<uint32_t*>(smem + L.offs);
+  uint32_t* s_binfo = reinterpret_cast<uint32_t*>(smem + L.binfo);
   uint16_t* s_rows = reinterpret_cast<uint16_t*>(smem + L.rows);
-  uint32_t* s_woff = reinterpret_cast<uint32_t*>(smem + L.rows16);
-  uint16_t* s_rstep = reinterpret_cast<uint16_t*>(smem + L.rstep);
+  uint32_t* s_meta = reinterpret_cast<uint32_t*>(smem + L.meta);
   uint32_t* s_ev = reinterpret_cast<uint32_t*>(smem + L.ev);
   uint32_t* s_acc = reinterpret_cast<uint32_t*>(smem + L.acc);
   uint32_t* s_log = reinterpret_cast<uint32_t*>(smem + L.log);
@@ -420,18 +432,41 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
         const uint32_t nrows = s_offs[nsteps] - wbase;
         for (uint32_t x = tid; x < nrows; x += nthr) s_rows[x] = rows_g[wbase + x];
         __syncthreads();
-        for (uint32_t x = tid; x < nrows; x += nthr) s_woff[x] = (uint32_t)s_rows[x] * (uint32_t)wpr;
-        for (int x = tid; x < nsteps; x += nthr)
-          for (uint32_t r = s_offs[x] - wbase; r < s_offs[x + 1] - wbase; ++r) s_rstep[r] = (uint16_t)x;
+        if (tid < 8) s_meta[nrows + tid] = (uint32_t)(n_in * wpr) | (0x1FFu << 16);   // zero-row pads
+        // row metadata: word offset | window step (the link is added below)
+        for (int x = tid; x < nsteps; x += nthr) {
+          for (uint32_t r = s_offs[x] - wbase; r < s_offs[x + 1] - wbase; ++r)
+            s_meta[r] = (uint32_t)s_rows[r] * (uint32_t)wpr | ((uint32_t)x << 16);
+          // block starting at step x: nb = the most steps (<= kBlk, inside the window) holding <= 64 rows
+          // in all (0: step x alone exceeds 64 rows -> general path), and which of them are non-empty
+          const uint32_t o0 = s_offs[x];
+          uint32_t nb = 0, ne = 0, prev = o0;
+          for (int b = 0; b < kBlk && x + b < nsteps; ++b) {
+            const uint32_t o = s_offs[x + b + 1];
+            if (o - o0 > 64u) break;
+            nb = b + 1;
+            if (o != prev) ne |= 1u << b;
+            prev = o;
+          }
+          s_binfo[x] = nb | (ne << 8);
+        }
         __syncthreads();
-        // bits 9..15 of s_rstep[r]: distance to the next occurrence of the same input within the next 64
-        // rows, 0 if none (a block holds <= 64 rows; LTD corrections follow these links, block_correct)
-        for (uint32_t x = tid; x < nrows; x += nthr) {
-          const uint16_t id = s_rows[x];
+        // link to the next occurrence of the same input within the next 64 rows and 8 steps (a block
+        // holds <= 64 rows and <= kBlk steps; LTD sum corrections follow the links, block_correct)
+        for (uint32_t r = tid; r < nrows; r += nthr) {
+          const uint32_t mr = s_meta[r];
+          const int x = meta_step(mr);
+          const uint32_t id = s_rows[r];
+          const uint32_t pat = id * 0x10001u;
+          const uint32_t lim = min(min(nrows, r + 65u), s_offs[min(x + kBlk, nsteps)] - wbase);
           uint32_t link = 0;
-          const uint32_t lim = min(nrows, x + 65u);
-          for (uint32_t y = x + 1; y < lim && !link; ++y) if (s_rows[y] == id) link = y - x;
-          if (link) s_rstep[x] = (uint16_t)(s_rstep[x] | (link << 9));
+          uint32_t y = r + 1;
+          if (y & 1u) { if (y < lim && s_rows[y] == id) link = 1; ++y; }
+          for (; !link && y < lim; y += 2) {   // two ids per 32-bit load (y + 1 <= rows_cap: allocated)
+            const uint32_t eq = __vcmpeq2(*reinterpret_cast<const uint32_t*>(s_rows + y), pat);
+            if (eq) { const uint32_t yy = y + ((eq & 0xFFFFu) ? 0u : 1u); if (yy < lim) link = yy - r; }
+          }
+          if (link) s_meta[r] = mr | (link << 25);
         }
         __syncthreads();
       }
@@ -497,22 +532,9 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
           // decrement at step b is subtracted from the sums of the later block steps that contain
           // the same row (exact: the sum was taken with the pre-decrement code).
           {
-            int nb = 0;
-            uint32_t nonempty = 0u;                            // block steps with >= 1 active row
-            {
-              int prev = r0;
-#pragma unroll
-              for (int b = 0; b < kBlk; ++b) {
-                if (nb == b && kk + b < kend) {
-                  const int o = (int)(s_offs[kk - ka + b + 1] - wbase);
-                  if (o - r0 <= 64) {
-                    nb = b + 1;
-                    if (o != prev) nonempty |= 1u << b;
-                    prev = o;
-                  }
-                }
-              }
-            }
+            const uint32_t bi = s_binfo[kk - ka];                // block shape (window staging)
+            const int nb = (int)(bi & 0xFFu);
+            const uint32_t nonempty = bi >> 8;                   // block steps with >= 1 active row
             if (nb > 0) {
               const int kb0 = kk;
               const bool prof = trace && lane == 0;
@@ -550,29 +572,24 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
               }
               if (!done && warp_live) {
                 // (a2) eq.(3) for all block steps in one flattened pass over the block's rows: the running
-                // SWAR sum is stored into the slot of the row's step; lanes never overflow (<= 64 rows), so
-                // the sum at the end of step b is the lane-wise max of slots 0..b.
-#pragma unroll 1
-                for (int b = 0; b < nb; ++b) my_acc[b * nthr] = 0u;
+                // SWAR sum is stored into the slot of the row's step, so the slot of a non-empty step holds
+                // the running sum at its end (lanes never overflow: <= 64 + 7 rows).  Branch-free groups of
+                // 8 rows: rows past the block belong to later steps (or are zero-row pads) and land in
+                // slots >= nb or the spill slot kBlk, which are never read.  All loads of a group are
+                // issued before its stores (the slots share the buffer: the compiler would serialise).
                 uint32_t run = 0u;
                 const int sbase = kb0 - ka;
-                // groups of 8 rows: all loads of a group are issued before its stores (the slots live in
-                // the same shared buffer, so the compiler would otherwise serialise load after store)
 #pragma unroll 1
                 for (int r = rblk0; r < rblk1; r += 8) {
-                  uint32_t o[8], st[8], w[8];
+                  uint32_t m[8], w[8];
 #pragma unroll
-                  for (int x = 0; x < 8; ++x) {
-                    const bool in = r + x < rblk1;
-                    o[x] = in ? s_woff[r + x] : (uint32_t)(n_in * wpr);   // the all-zero row
-                    st[x] = in ? (uint32_t)(s_rstep[r + x] & 0x1FFu) : 0xFFFFu;
-                  }
+                  for (int x = 0; x < 8; ++x) m[x] = s_meta[r + x];
 #pragma unroll
-                  for (int x = 0; x < 8; ++x) w[x] = (wcol[o[x]] >> fsh) & Z::LMASK;
+                  for (int x = 0; x < 8; ++x) w[x] = (wcol[meta_woff(m[x])] >> fsh) & Z::LMASK;
 #pragma unroll
                   for (int x = 0; x < 8; ++x) {
                     run += w[x];
-                    if (st[x] != 0xFFFFu) my_acc[((int)st[x] - sbase) * nthr] = run;
+                    my_acc[min(meta_step(m[x]) - sbase, kBlk) * nthr] = run;
                   }
                 }
               }
@@ -585,10 +602,10 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
                   if ((ltd_cols >> c & 1u) && (tbase + kb0 - lpost[c]) < L_dep) ltd_blk |= 1u << c;
               }
               const int nrows_blk = rblk1 - rblk0;
-              if (__any_sync(FULL, ltd_blk != 0)) {
+              if (SNN_EXP != 2 && __any_sync(FULL, ltd_blk != 0)) {
                 // this lane's rows of the block and their steps (the same for every pair)
-                const int bsel0 = lane < nrows_blk ? (int)(s_rstep[rblk0 + lane] & 0x1FFu) - (kb0 - ka) : 0;
-                const int bsel1 = lane + 32 < nrows_blk ? (int)(s_rstep[rblk0 + 32 + lane] & 0x1FFu) - (kb0 - ka) : 0;
+                const int bsel0 = lane < nrows_blk ? meta_step(s_meta[rblk0 + lane]) - (kb0 - ka) : 0;
+                const int bsel1 = lane + 32 < nrows_blk ? meta_step(s_meta[rblk0 + 32 + lane]) - (kb0 - ka) : 0;
                 const uint32_t row0 = lane < nrows_blk ? (uint32_t)s_rows[rblk0 + lane] : 0u;
                 const uint32_t row1 = lane + 32 < nrows_blk ? (uint32_t)s_rows[rblk0 + 32 + lane] : 0u;
 #pragma unroll 1
@@ -620,18 +637,32 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
                 }
               }
               long long pc2 = prof ? clock64() : 0;
+              // ---- this lane's LTD events of the block, once: 64-bit row masks per column and the block
+              // steps that hold at least one event (the LIF chain below only branches on those)
+              unsigned long long e64c[CPT];
+              uint32_t evsteps = 0u;
+#pragma unroll
+              for (int c = 0; c < CPT; ++c) {
+                e64c[c] = 0ull;
+                if (SNN_EXP != 2 && (ltd_blk >> c & 1u)) {
+                  e64c[c] = (unsigned long long)s_ev[(c * 2) * nthr + tid] |
+                            ((unsigned long long)s_ev[(c * 2 + 1) * nthr + tid] << 32);
+                  for (unsigned long long m = e64c[c]; m; m &= m - 1ull)
+                    evsteps |= 1u << (meta_step(s_meta[rblk0 + __ffsll((long long)m) - 1]) - (kb0 - ka));
+                }
+              }
               // ---- sequential LIF over the block (the only step-to-step dependency)
               if (!done) {
                 int rlo = rblk0;
                 uint32_t run_prev = 0u;
+                int bdone = nb;                                      // block steps committed by this lane
 #pragma unroll 1
                 for (int b = 0; b < nb; ++b) {
                   const int kk_b = kb0 + b;
                   // a crossing before kk_b exists in the cluster: stop here (state is that after kk_b - 1)
-                  if (b > 0 && kk_b > ld_volatile_shared_u32addr(flag_addr)) { done = true; p = kk_b; break; }
-                  const int t = tbase + kk_b;
+                  if (b > 0 && kk_b > ld_volatile_shared_u32addr(flag_addr)) { done = true; p = kk_b; bdone = b; break; }
                   const int rhi = (int)(s_offs[kk_b - ka + 1] - wbase);
-                  const uint32_t snap = vmax_lanes<CPT>(run_prev, my_acc[b * nthr]);
+                  const uint32_t snap = (nonempty >> b & 1u) ? my_acc[b * nthr] : run_prev;
                   const uint32_t a = snap - run_prev;              // this step's SWAR sums
                   run_prev = snap;
                   uint32_t cm_b = 0;
@@ -650,27 +681,19 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
                       v[c] = cnt[c] == 0 ? vn[c] : v[c];
                       cnt[c] = cnt[c] == 0 ? 0 : cnt[c] - 1;
                     }
-                    cmask = cm_b; cand = true; done = true; p = kk_b; signal(kk_b);
+                    cmask = cm_b; cand = true; done = true; p = kk_b; bdone = b; signal(kk_b);
                     break;
                   }
-                  uint32_t on_b = 0;
-                  if (ltd_blk) {
-#pragma unroll
-                    for (int c = 0; c < CPT; ++c)
-                      if ((ltd_blk >> c & 1u) && (t - lpost[c]) < L_dep) on_b |= 1u << c;
-                  }
                   const long long pe0 = prof ? clock64() : 0;
-                  if (on_b) {                                         // LTD events of step b (rare)
+                  if (SNN_EXP != 1 && (evsteps >> b & 1u)) {          // LTD events of step b (rare)
                     const int lo = rlo - rblk0, nrb = rhi - rlo;
                     const int nlog_step = nlog;
                     bool overflow = false;
                     uint32_t ev_step = 0;
-#pragma unroll 1
-                    for (uint32_t cmm = on_b; cmm && !overflow; cmm &= cmm - 1) {
-                      const int c = __ffs(cmm) - 1;
-                      const unsigned long long e64 = (unsigned long long)s_ev[(c * 2) * nthr + tid] |
-                                                     ((unsigned long long)s_ev[(c * 2 + 1) * nthr + tid] << 32);
-                      unsigned long long em = nrb ? ((e64 >> lo) & ((1ull << nrb) - 1ull)) : 0ull;
+#pragma unroll
+                    for (int c = 0; c < CPT; ++c) {
+                      if (overflow || !(ltd_blk >> c & 1u)) continue;
+                      unsigned long long em = nrb ? ((e64c[c] >> lo) & ((1ull << nrb) - 1ull)) : 0ull;
                       const int shc = fsh + c * Z::LW;
                       while (em) {
                         const int xr = __ffsll((long long)em) - 1;
@@ -682,8 +705,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
                         if (applied) {
                           atomicSub(pw, 1u << shc);
                           // the later block steps that contain row i were summed with the old code
-                          if (s_rstep[rlo + xr] >> 9)
-                            block_correct(s_rstep, my_acc, nthr, rlo + xr, rblk1, kb0 - ka, nonempty, 0u - (1u << (c * Z::LW)));
+                          if (meta_link(s_meta[rlo + xr]))
+                            block_correct(s_meta, my_acc, nthr, rlo + xr, rblk1, kb0 - ka, nonempty, 0u - (1u << (c * Z::LW)));
                         }
                         ++ev_step;
                         if (kk_b > k0) s_log[nlog++ * nthr + tid] = log_entry(kk_b - k0, c, applied, i);
@@ -697,16 +720,15 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
                           atomicAdd(wcol + i * wpr, 1u << (fsh + c * Z::LW));
                           int rpos = rlo;                             // the event's row position in step b
                           while (rpos < rhi - 1 && (int)s_rows[rpos] != i) ++rpos;
-                          block_correct(s_rstep, my_acc, nthr, rpos, rblk1, kb0 - ka, nonempty, 1u << (c * Z::LW));
+                          block_correct(s_meta, my_acc, nthr, rpos, rblk1, kb0 - ka, nonempty, 1u << (c * Z::LW));
                         }
                         --nlog;
                       }
-                      hz = true; done = true; p = kk_b; ++eng_hz;     // v / cnt of step b were not committed
+                      hz = true; done = true; p = kk_b; bdone = b; ++eng_hz;   // v / cnt of step b were not committed
                       signal(kk_b - 1);
                       break;
                     }
                     ltd_events += ev_step;
-                    ltd_trials += (uint32_t)__popc(on_b) * (uint32_t)nrb;
                     if (trace) prof_nev += ev_step;
                   }
                   if (prof) { __syncwarp(__activemask()); prof_ev += clock64() - pe0; }
@@ -720,6 +742,15 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
                     for (int c = 0; c < CPT; ++c) { v1[c] = v[c]; cnt1[c] = cnt[c]; }
                   }
                   rlo = rhi;
+                }
+                // LTD trials of the committed block steps: rows of steps b < bdone with D = t - last_post < L_dep
+                if (ltd_blk) {
+#pragma unroll
+                  for (int c = 0; c < CPT; ++c) {
+                    if (!(ltd_blk >> c & 1u)) continue;
+                    const int blim = min(bdone, lpost[c] + L_dep - tbase - kb0);
+                    if (blim > 0) ltd_trials += s_offs[kb0 - ka + blim] - s_offs[kb0 - ka];
+                  }
                 }
               }
               if (prof) {

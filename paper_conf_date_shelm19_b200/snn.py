@@ -10,7 +10,7 @@ from typing import Optional, Sequence
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libsnn_b200.so")
+LIB_PATH = os.environ.get("SNN_LIB_PATH") or os.path.join(_HERE, "libsnn_b200.so")   # override: experiments only
 
 SNN_OK, SNN_EINVAL, SNN_ENOMEM, SNN_ECUDA, SNN_ENCCL, SNN_ESIZE, SNN_ECOOP = 0, -1, -2, -3, -4, -5, -6
 SNN_RASTER_INPUT, SNN_KEEP_STATE, SNN_RECORD_INPUT, SNN_ASYNC, SNN_FLOOR_PROBE = 1, 2, 4, 8, 16
