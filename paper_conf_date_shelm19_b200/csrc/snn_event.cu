@@ -653,16 +653,21 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
               }
               // ---- sequential LIF over the block (the only step-to-step dependency)
               if (!done) {
-                int rlo = rblk0;
                 uint32_t run_prev = 0u;
                 int bdone = nb;                                      // block steps committed by this lane
+                // software pipelined: the next step's sum slot and the early-stop flag are loaded one step
+                // ahead (a flag seen one step late only speculates one step further, which the resolution
+                // rolls back like any overrun)
+                uint32_t slot_nx = my_acc[0];
+                int flag_nx = INT_MAX;
 #pragma unroll 1
                 for (int b = 0; b < nb; ++b) {
                   const int kk_b = kb0 + b;
                   // a crossing before kk_b exists in the cluster: stop here (state is that after kk_b - 1)
-                  if (b > 0 && kk_b > ld_volatile_shared_u32addr(flag_addr)) { done = true; p = kk_b; bdone = b; break; }
-                  const int rhi = (int)(s_offs[kk_b - ka + 1] - wbase);
-                  const uint32_t snap = (nonempty >> b & 1u) ? my_acc[b * nthr] : run_prev;
+                  if (b > 0 && kk_b > flag_nx) { done = true; p = kk_b; bdone = b; break; }
+                  const uint32_t snap = (nonempty >> b & 1u) ? slot_nx : run_prev;
+                  if (b + 1 < nb) slot_nx = my_acc[(b + 1) * nthr];
+                  flag_nx = ld_volatile_shared_u32addr(flag_addr);
                   const uint32_t a = snap - run_prev;              // this step's SWAR sums
                   run_prev = snap;
                   uint32_t cm_b = 0;
@@ -686,6 +691,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
                   }
                   const long long pe0 = prof ? clock64() : 0;
                   if (SNN_EXP != 1 && (evsteps >> b & 1u)) {          // LTD events of step b (rare)
+                    const int rlo = (int)(s_offs[kk_b - ka] - wbase), rhi = (int)(s_offs[kk_b - ka + 1] - wbase);
                     const int lo = rlo - rblk0, nrb = rhi - rlo;
                     const int nlog_step = nlog;
                     bool overflow = false;
@@ -730,6 +736,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
                     }
                     ltd_events += ev_step;
                     if (trace) prof_nev += ev_step;
+                    if (b + 1 < nb) slot_nx = my_acc[(b + 1) * nthr];   // the corrections may have changed it
                   }
                   if (prof) { __syncwarp(__activemask()); prof_ev += clock64() - pe0; }
 #pragma unroll
@@ -741,7 +748,6 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_event_kernel(const _
 #pragma unroll
                     for (int c = 0; c < CPT; ++c) { v1[c] = v[c]; cnt1[c] = cnt[c]; }
                   }
-                  rlo = rhi;
                 }
                 // LTD trials of the committed block steps: rows of steps b < bdone with D = t - last_post < L_dep
                 if (ltd_blk) {
