@@ -86,6 +86,9 @@ typedef struct snn_params {
 /* engine: both give bit-identical results */
 #define SNN_ENGINE_EVENT 0   /* one cluster exchange per post-spike epoch; T <= 32767 */
 #define SNN_ENGINE_STEP  1   /* one cluster exchange per timestep */
+#define SNN_ENGINE_EVENT_GENERAL 2   /* the event engine's general kernel even where the lean one applies */
+/* SNN_ENGINE_EVENT runs the lean kernel for HARD WTA + RESET inhibition + stochastic STDP
+ * on an unsharded network (the paper's default mode) and the general event kernel otherwise. */
 
 /* Table I rows */
 #define SNN_PRESET_2B  0
@@ -162,8 +165,9 @@ int snn_reset_stats(snn_handle* h);
 /* Introspection: [0] cluster size, [1] threads per CTA, [2] dynamic smem bytes per CTA,
  * [3] words per weight row in a CTA slice, [4] q_max, [5] L_pot, [6] L_dep, [7] kernel launches so far,
  * [8] engine, [9] columns per thread (event engine), [10] on-chip row window, [11] LTD undo-log depth,
- * [12] first global column (col_base), [13] columns of the whole network, [14] world, [15] shard. */
-#define SNN_NINFO 16
+ * [12] first global column (col_base), [13] columns of the whole network, [14] world, [15] shard,
+ * [16] 1 if the lean event kernel runs, [17] its dynamic smem bytes per CTA. */
+#define SNN_NINFO 18
 int snn_get_info(const snn_handle* h, int64_t info[SNN_NINFO]);
 
 /* Tracing: with max_epochs > 0 the event engine records, per CTA and epoch,

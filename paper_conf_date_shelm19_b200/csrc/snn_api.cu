@@ -100,6 +100,8 @@ struct snn_handle {
   int engine = SNN_ENGINE_EVENT;
   int rows_cap = 0, offs_cap = 0, logn = 0;
   int cpt = 1;                    // columns per thread of the event engine
+  bool lean = false;              // event engine runs the lean kernel (HARD / RESET / stochastic)
+  size_t smem_lean = 0;
   uint32_t* d_words = nullptr;   size_t words_cap = 0;
   uint32_t* d_ecnt = nullptr;    size_t ecnt_cap = 0;
   uint32_t* d_offs = nullptr;    size_t offs_buf_cap = 0;
@@ -139,7 +141,8 @@ int validate(int n_in, int n_exc, int bits, const snn_params* p) {
   if (p->stdp_mode == 1 && !(p->alpha_p >= 0 && p->alpha_d >= 0 && p->beta_p >= 0 && p->beta_d >= 0))
     return fail(SNN_EINVAL, "alpha/beta must be >= 0");
   if (p->cluster_size < 0 || p->cluster_size > snn::kMaxCluster) return fail(SNN_EINVAL, "cluster_size outside [0, 16]");
-  if (p->engine != SNN_ENGINE_EVENT && p->engine != SNN_ENGINE_STEP) return fail(SNN_EINVAL, "engine must be 0 or 1");
+  if (p->engine != SNN_ENGINE_EVENT && p->engine != SNN_ENGINE_STEP && p->engine != SNN_ENGINE_EVENT_GENERAL)
+    return fail(SNN_EINVAL, "engine must be 0, 1 or 2");
   return SNN_OK;
 }
 
@@ -342,8 +345,12 @@ int present_impl(snn_handle* h, const void* input, int n_images, int T, const ui
     if (rc) return rc;
     if ((rc = shard_arm(h, d))) return rc;
     lp.single = d;
-    CUDA_TRY(snn::launch_present_event_mode(lp, 1, h->cs, h->nthr, h->smem, h->bits, h->cpt, h->p.membrane_mode,
-                                            h->stream));
+    if (h->lean)
+      CUDA_TRY(snn::launch_present_lean(lp, 1, h->cs, h->nthr, h->smem_lean, h->bits, h->cpt, h->p.membrane_mode,
+                                        h->stream));
+    else
+      CUDA_TRY(snn::launch_present_event_mode(lp, 1, h->cs, h->nthr, h->smem, h->bits, h->cpt, h->p.membrane_mode,
+                                              h->stream));
   } else {
     lp.single = d;
     CUDA_TRY(snn::launch_present(lp, 1, h->cs, h->nthr, h->smem, h->stream));
@@ -463,7 +470,11 @@ int create_impl(int n_in, int n_exc, int bits, const snn_params* p, int col_base
   int smem_optin = 0;
   cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, h->dev);
   h->ngroups = (n_exc + 31) / 32;
-  h->engine = p->engine;
+  h->engine = p->engine == SNN_ENGINE_STEP ? SNN_ENGINE_STEP : SNN_ENGINE_EVENT;
+  // the lean kernel covers the paper's default learning mode; SNN_NO_LEAN=1 disables it
+  const bool lean_mode = p->engine == SNN_ENGINE_EVENT && p->wta_mode == SNN_WTA_HARD &&
+                         p->inh_mode == SNN_INH_RESET && p->stdp_mode == SNN_STDP_STOCH && world == 1 &&
+                         !(getenv("SNN_NO_LEAN") && atoi(getenv("SNN_NO_LEAN")) != 0);
   int chosen = 0;
   const bool ev = h->engine == SNN_ENGINE_EVENT;
   const int max_thr = ev ? snn::kEvMaxThreads : snn::kMaxThreads;
@@ -508,6 +519,10 @@ int create_impl(int n_in, int n_exc, int bits, const snn_params* p, int col_base
     if (smem > (size_t)smem_optin) continue;
     h->cs = cs; h->nthr = nthr; h->wpr = wpr; h->slice_words = sw; h->smem = smem;
     h->rows_cap = rows_cap; h->offs_cap = offs_cap; h->logn = logn; h->cpt = cpt;
+    if (ev && lean_mode) {
+      h->smem_lean = snn::lean_smem_bytes(n_in, sw, h->L_pot, h->L_dep, nthr, rows_cap, offs_cap, logn);
+      h->lean = h->smem_lean <= (size_t)smem_optin;
+    }
     chosen = 1;
     break;
   }
@@ -531,6 +546,11 @@ int create_impl(int n_in, int n_exc, int bits, const snn_params* p, int col_base
     nclusters *= sms;
   }
   h->max_clusters = nclusters;
+  if (h->lean) {
+    int nl = 0;
+    ce = snn::query_max_clusters_lean(bits, h->cpt, p->membrane_mode, h->cs, h->nthr, h->smem_lean, &nl);
+    if (ce != cudaSuccess || nl < 1) { cudaGetLastError(); h->lean = false; }
+  }
 
 #define ALLOC(ptr, n)                                                            \
   do {                                                                           \
@@ -847,7 +867,9 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
     std::memset(&lp, 0, sizeof(lp));
     lp.descs = d_descs + off;
     size_t smem = 0;
-    for (int k : g) smem = std::max(smem, hs[k]->smem);
+    bool lean = ev;
+    for (int k : g) lean = lean && hs[k]->lean;
+    for (int k : g) smem = std::max(smem, lean ? hs[k]->smem_lean : hs[k]->smem);
     cudaStream_t st = h0->stream;
     if (groups.size() > 1) {
       e = cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking);
@@ -862,9 +884,11 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
     for (int k : g)
       if (hs[k]->cpt != hs[g[0]]->cpt) { e = cudaErrorInvalidValue; break; }
     if (e != cudaSuccess) break;
-    e = ev ? snn::launch_present_event_mode(lp, (int)g.size(), h0->cs, hs[g[0]]->nthr, smem, hs[g[0]]->bits,
-                                            hs[g[0]]->cpt, h0->p.membrane_mode, st)
-           : snn::launch_present(lp, (int)g.size(), h0->cs, h0->nthr, smem, st);
+    e = lean ? snn::launch_present_lean(lp, (int)g.size(), h0->cs, hs[g[0]]->nthr, smem, hs[g[0]]->bits,
+                                        hs[g[0]]->cpt, h0->p.membrane_mode, st)
+        : ev ? snn::launch_present_event_mode(lp, (int)g.size(), h0->cs, hs[g[0]]->nthr, smem, hs[g[0]]->bits,
+                                              hs[g[0]]->cpt, h0->p.membrane_mode, st)
+             : snn::launch_present(lp, (int)g.size(), h0->cs, h0->nthr, smem, st);
     off += g.size();
   }
   for (cudaStream_t st : forks) {
@@ -1046,6 +1070,7 @@ int snn_get_info(const snn_handle* h, int64_t info[SNN_NINFO]) {
   info[4] = h->q_max; info[5] = h->L_pot; info[6] = h->L_dep; info[7] = h->launches;
   info[8] = h->engine; info[9] = h->cpt; info[10] = h->rows_cap; info[11] = h->logn;
   info[12] = h->col_base; info[13] = h->n_exc_total; info[14] = h->world; info[15] = h->shard;
+  info[16] = h->lean ? 1 : 0; info[17] = (int64_t)h->smem_lean;
   return SNN_OK;
 }
 

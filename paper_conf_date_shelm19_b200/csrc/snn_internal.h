@@ -111,6 +111,12 @@ cudaError_t launch_compact(const uint32_t* words, const uint32_t* counts, int n_
 cudaError_t launch_present_event_mode(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, int bits,
                                       int cpt, int fixed, cudaStream_t s);
 cudaError_t configure_present_kernel(size_t smem, int cs);
+// lean event kernel (snn_lean.cu)
+size_t lean_smem_bytes(int n_in, int slice_words, int L_pot, int L_dep, int nthr, int rows_cap, int offs_cap,
+                       int logn);
+cudaError_t query_max_clusters_lean(int bits, int cpt, int fixed, int cs, int nthr, size_t smem, int* out);
+cudaError_t launch_present_lean(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, int bits, int cpt,
+                                int fixed, cudaStream_t s);
 cudaError_t query_max_clusters(int cs, int nthr, size_t smem, int* out);
 cudaError_t launch_init_weights(const NetDesc& d, uint64_t init_seed, cudaStream_t s);
 cudaError_t launch_pack_weights(const NetDesc& d, const uint8_t* codes, cudaStream_t s);

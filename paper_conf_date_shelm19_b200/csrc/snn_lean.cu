@@ -1,0 +1,767 @@
+// snn_lean.cu -- lean event-engine kernel for the paper's default learning mode:
+// HARD winner-take-all with RESET inhibition (R7) and stochastic 1-LSB STDP (eqs.(6)(7),
+// P:89).  Same epoch protocol as snn_event.cu (one cluster exchange per post-spike epoch; the
+// columns run ahead independently between spikes), restructured around what that mode makes true:
+//   * after every post spike EVERY column restarts from a state fixed by its own countdown
+//     (v <- v_reset, cnt <- max(cnt, t_inh), the winner cnt <- t_ref), so a column that ran past the
+//     first crossing t* is rebuilt in O(1) -- no membrane snapshot, no re-simulation;
+//   * LTD of a column depends only on its own last_post and the input raster (R10, R14), so the
+//     Philox draws of a warp's LTD-active columns are taken for 32 upcoming input rows at once
+//     (lanes over rows), off the LIF chain; the decrements are applied in step order as the chain
+//     reaches them, so every integration reads the codes of its own step and no sum is ever corrected;
+//   * integration is inline per step from a padded row list (one 16-byte load yields 4 row offsets),
+//     summing the thread's CPT columns in SWAR lanes (eq.(3)); held (refractory / inhibited) warps skip
+//     whole runs of steps in O(1);
+//   * LTP of the winner (eq.(6)) needs last_pre only in the winner's CTA: the input spike timers are
+//     brought up to date lazily there, and nowhere else.
+// Results are bit-identical to the oracle (tests/test_gpu_parity.py runs every case on this kernel and
+// on the general one).
+#include "snn_internal.h"
+#include "snn_device.cuh"
+
+#include <climits>
+#include <cstdio>
+#include <cstdint>
+
+namespace snn {
+
+namespace {
+
+template <int BITS, int CPT_> struct LSwar {
+  static constexpr int CPT = CPT_;
+  static constexpr int CPW = 32 / BITS;
+  static constexpr int TPW = CPW / CPT_;
+  static constexpr int LW = 32 / CPT_;
+  static constexpr uint32_t FM = (1u << BITS) - 1u;
+  static constexpr uint32_t LMASK = CPT_ == 1 ? FM : (CPT_ == 2 ? (FM | (FM << 16)) : (FM * 0x01010101u));
+  // rows that can be summed into one SWAR word before a lane could overflow (multiple of 4)
+  static constexpr int CHUNK = CPT_ == 1 ? (1 << 28) : (int)((((1u << (LW & 31)) - 1u) / FM) & ~3u);
+};
+
+struct LeanLayout {
+  size_t slots, wsum, flags, misc, w, pot, dep, lpre, offs, pst, prow, rraw, log, total;
+};
+
+__host__ __device__ inline LeanLayout lean_layout(int n_in, int slice_words, int L_pot, int L_dep, int nthr,
+                                                  int rows_cap, int offs_cap, int logn) {
+  LeanLayout L;
+  size_t o = 0;
+  L.slots = o; o = align16(o + 2 * kMaxCluster * 2 * 8);     // [parity][rank][2] u64: steps, key
+  L.wsum = o;  o = align16(o + 32 * 2 * 8);                  // per warp: steps, key
+  L.flags = o; o = align16(o + 4 * 4);                       // early-stop flag per epoch parity
+  L.misc = o;  o = align16(o + 16 * 4);
+  L.w = o;     o = align16(o + (size_t)slice_words * 4);
+  L.pot = o;   o = align16(o + (size_t)(L_pot > 0 ? L_pot : 1) * 4);
+  L.dep = o;   o = align16(o + (size_t)(L_dep > 0 ? L_dep : 1) * 4);
+  L.lpre = o;  o = align16(o + (size_t)n_in * 4);
+  L.offs = o;  o = align16(o + (size_t)(offs_cap + 1) * 4);          // raw row offset of every window step
+  L.pst = o;   o = align16(o + (size_t)(offs_cap + 1) * 4);          // padded (x4) start of every window step
+  L.prow = o;  o = align16(o + (size_t)(rows_cap + 3 * offs_cap + 4) * 4);   // padded word offsets row*wpr
+  L.rraw = o;  o = align16(o + (size_t)(rows_cap + 32) * 4);         // raw rows: step << 16 | row id
+  L.log = o;   o = align16(o + (size_t)logn * nthr * 4);
+  L.total = o;
+  return L;
+}
+
+// undo-log entry: rel step (16) | column slot c (2) | applied (1) | row (13)
+__device__ __forceinline__ uint32_t lean_log_entry(int rel, int c, bool applied, int row) {
+  return ((uint32_t)rel << 16) | ((uint32_t)c << 14) | (applied ? 0x2000u : 0u) | (uint32_t)row;
+}
+
+constexpr int kNoStep = 0x7FFFFFFF;
+
+}  // namespace
+
+size_t lean_smem_bytes(int n_in, int slice_words, int L_pot, int L_dep, int nthr, int rows_cap, int offs_cap,
+                       int logn) {
+  return lean_layout(n_in, slice_words, L_pot, L_dep, nthr, rows_cap, offs_cap, logn).total;
+}
+
+template <int BITS, int CPT_, bool FIXED>
+__global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __grid_constant__ LaunchParams lp) {
+  using Z = LSwar<BITS, CPT_>;
+  constexpr int CPT = Z::CPT;
+  constexpr int CPW = Z::CPW;
+  constexpr int TPW = Z::TPW;
+  constexpr uint32_t FMASK = Z::FM;
+  extern __shared__ __align__(16) unsigned char smem[];
+  const NetDesc& d0 = lp.descs ? lp.descs[0] : lp.single;
+  const int cs = d0.cs;
+  const int net = blockIdx.x / cs;
+  const int rank = blockIdx.x - net * cs;
+  const NetDesc& d = lp.descs ? lp.descs[net] : lp.single;
+
+  const int n_in = d.n_in, n_exc = d.n_exc, qmax = d.q_max, wpr = d.wpr;
+  const int T = d.T, flags = d.flags, n_images = d.n_images;
+  const int L_pot = d.L_pot, L_dep = d.L_dep, rows_cap = d.rows_cap, offs_cap = d.offs_cap, logn = d.logn;
+  const int slice_words = d.slice_words;
+  const int nthr = blockDim.x;
+  const LeanLayout L = lean_layout(n_in, slice_words, L_pot, L_dep, nthr, rows_cap, offs_cap, logn);
+  unsigned long long* s_slots = reinterpret_cast<unsigned long long*>(smem + L.slots);
+  unsigned long long* s_wsum = reinterpret_cast<unsigned long long*>(smem + L.wsum);
+  int* s_flag = reinterpret_cast<int*>(smem + L.flags);
+  int* s_misc = reinterpret_cast<int*>(smem + L.misc);
+  uint32_t* s_w = reinterpret_cast<uint32_t*>(smem + L.w);
+  uint32_t* s_pot = reinterpret_cast<uint32_t*>(smem + L.pot);
+  uint32_t* s_dep = reinterpret_cast<uint32_t*>(smem + L.dep);
+  int* s_lpre = reinterpret_cast<int*>(smem + L.lpre);
+  uint32_t* s_offs = reinterpret_cast<uint32_t*>(smem + L.offs);
+  uint32_t* s_pst = reinterpret_cast<uint32_t*>(smem + L.pst);
+  uint32_t* s_prow = reinterpret_cast<uint32_t*>(smem + L.prow);
+  uint32_t* s_rraw = reinterpret_cast<uint32_t*>(smem + L.rraw);
+  uint32_t* s_log = reinterpret_cast<uint32_t*>(smem + L.log);
+
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwarps = nthr >> 5;
+  const int g0 = (rank * d.ngroups) / cs, g1 = ((rank + 1) * d.ngroups) / cs;
+  const int col0 = g0 * 32;
+  const int cbase = d.col_base;
+  const int ncols = min(g1 * 32, n_exc) - col0;
+  const int wj = tid / TPW, f = tid % TPW;
+  const int fsh = f * BITS;
+  const uint32_t* const wcol = s_w + min(wj, wpr - 1);     // threads past the slice read a real word
+  int jcol[CPT];                       // local column of slot c (or -1)
+  uint32_t valid = 0;
+#pragma unroll
+  for (int c = 0; c < CPT; ++c) {
+    const int jl = wj * CPW + f + TPW * c;
+    jcol[c] = (jl < ncols && wj < wpr) ? jl : -1;
+    if (jcol[c] >= 0) valid |= 1u << c;
+  }
+  const uint32_t zero_off = (uint32_t)(n_in * wpr);   // the all-zero row n_in of the slice
+  const int nq4 = (n_in + 3) >> 2;
+
+  Lif lif;
+  lif.load(d);
+  const int vreset = FIXED ? d.Vreset : __float_as_int(d.vresetf);
+  const int vinit = FIXED ? d.Vinit : __float_as_int(d.vinitf);
+  const int t_ref = d.t_ref, t_inh = d.t_inh;
+  const bool keep = (flags & FLAG_KEEP_STATE) != 0;
+  const int tbase = keep ? d.t0 : 0;
+
+  // ---- one-time staging
+  for (int k = tid; k < L_pot; k += nthr) s_pot[k] = d.pot_m1[k];
+  for (int k = tid; k < L_dep; k += nthr) s_dep[k] = d.dep_m1[k];
+  {
+    const uint4* src = reinterpret_cast<const uint4*>(d.wslices + (size_t)rank * slice_words);
+    uint4* dst = reinterpret_cast<uint4*>(s_w);
+    for (int k = tid; k < slice_words / 4; k += nthr) dst[k] = src[k];
+  }
+  if (tid == 0) { s_flag[0] = INT_MAX; s_flag[1] = INT_MAX; }
+  int v[CPT], cnt[CPT], lpost[CPT];
+#pragma unroll
+  for (int c = 0; c < CPT; ++c) {
+    v[c] = vinit; cnt[c] = 0; lpost[c] = kNever;
+    if (keep && (valid >> c & 1u)) {
+      const int jg = col0 + jcol[c];
+      v[c] = d.v[jg]; cnt[c] = d.cnt[jg]; lpost[c] = d.last_post[jg];
+    }
+  }
+  if (keep) for (int i = tid; i < n_in; i += nthr) s_lpre[i] = d.last_pre[i];
+  uint32_t ltd_trials = 0, ltd_events = 0, ltp_trials = 0, ltp_events = 0;
+  unsigned long long act_sum = 0, post_sum = 0;
+  uint32_t eng_epochs = 0, eng_hz = 0, eng_resim = 0, eng_spec = 0, eng_undo = 0;
+  if (cs > 1) { cluster_arrive(); cluster_wait(); } else { __syncthreads(); }
+
+  int ep = 0;
+  for (int b = 0; b < n_images; ++b) {
+    const unsigned long long seed = d.seeds[b];
+    if (!keep) {
+#pragma unroll
+      for (int c = 0; c < CPT; ++c) { v[c] = vinit; cnt[c] = 0; lpost[c] = kNever; }
+      for (int i = tid; i < n_in; i += nthr) s_lpre[i] = kNever;
+    }
+    const uint32_t* offs_g = d.ev_offs + (size_t)b * (T + 1);
+    const uint16_t* rows_g = d.ev_rows + (size_t)b * d.rows_stride;
+    const bool last_img = (b == n_images - 1);
+    const bool rec_out = last_img && d.raster_out != nullptr;
+    int img_spikes = 0;
+    int ka = 0, kb = 0;            // window steps [ka, kb)
+    int lpre_upto = -1;            // s_lpre holds the input spike timers through window step lpre_upto
+    int k0 = 0;
+    if (rank == 0 && tid == 0 && T > 0) act_sum += (unsigned long long)(offs_g[T] - offs_g[0]);
+    __syncthreads();
+
+    // input spike timers of window steps (lpre_upto, upto]: every CTA thread takes raw rows
+    auto lpre_catch_up = [&](int upto) {
+      if (upto > lpre_upto) {
+        const uint32_t r0 = s_offs[lpre_upto + 1], r1 = s_offs[upto + 1];
+        for (uint32_t r = r0 + tid; r < r1; r += nthr) {
+          const uint32_t rr = s_rraw[r];
+          atomicMax(&s_lpre[rr & 0xFFFFu], tbase + ka + (int)(rr >> 16));
+        }
+        lpre_upto = upto;
+      }
+    };
+
+    while (k0 < T) {
+      // ---------------------------------------------------------- stage the active-row window
+      if (k0 >= kb) {
+        __syncthreads();
+        if (kb > ka) lpre_catch_up(kb - 1 - ka);                   // finish the old window's timers
+        __syncthreads();
+        ka = k0;
+        lpre_upto = -1;
+        const int n_o = min(offs_cap, T - ka);
+        const uint32_t wbase = offs_g[ka];
+        for (int x = tid; x <= n_o; x += nthr) s_offs[x] = offs_g[ka + x] - wbase;
+        if (tid == 0) s_misc[0] = 0;
+        __syncthreads();
+        int fit = 0;
+        for (int x = tid + 1; x <= n_o; x += nthr) {
+          const uint32_t padded = s_offs[x] + 3u * (uint32_t)x;      // upper bound of the padded length
+          fit += (s_offs[x] <= (uint32_t)rows_cap && padded <= (uint32_t)(rows_cap + 3 * offs_cap)) ? 1 : 0;
+        }
+        if (fit) atomicAdd(&s_misc[0], fit);
+        __syncthreads();
+        const int nsteps = max(1, s_misc[0]);    // rows_cap >= n_in: one step always fits
+        kb = ka + nsteps;
+        // padded starts: warp 0 scans the per-step group counts
+        if (warp == 0) {
+          const int per = (nsteps + 31) / 32;
+          const int lo = min(nsteps, lane * per), hi = min(nsteps, lo + per);
+          uint32_t sum = 0;
+          for (int x = lo; x < hi; ++x) sum += (s_offs[x + 1] - s_offs[x] + 3u) & ~3u;
+          uint32_t incl = sum;
+#pragma unroll
+          for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(FULL, incl, o);
+            if (lane >= o) incl += y;
+          }
+          uint32_t run = incl - sum;
+          for (int x = lo; x < hi; ++x) { s_pst[x] = run; run += (s_offs[x + 1] - s_offs[x] + 3u) & ~3u; }
+          if (lane == 31) s_pst[nsteps] = incl;
+        }
+        __syncthreads();
+        // raw rows (step << 16 | id) and padded word offsets; one thread per step
+        const uint32_t nrows = s_offs[nsteps];
+        for (int x = tid; x < nsteps; x += nthr) {
+          const uint32_t o0 = s_offs[x], o1 = s_offs[x + 1], p0 = s_pst[x], p1 = s_pst[x + 1];
+          for (uint32_t r = o0; r < o1; ++r) {
+            const uint32_t i = rows_g[wbase + r];
+            s_rraw[r] = ((uint32_t)x << 16) | i;
+            s_prow[p0 + (r - o0)] = i * (uint32_t)wpr;
+          }
+          for (uint32_t q = p0 + (o1 - o0); q < p1; ++q) s_prow[q] = zero_off;
+        }
+        for (int x = tid; x < 32; x += nthr) s_rraw[nrows + x] = 0xFFFF0000u;   // draw pads (never an event)
+        __syncthreads();
+      }
+      const int kend = kb;
+      const int fp = ep & 1;
+      const uint32_t flag_addr = smem_u32(&s_flag[fp]);
+
+      // ---------------------------------------------------------- speculation (warp-synchronous)
+      int cnt0[CPT], v1[CPT], cnt1[CPT];
+#pragma unroll
+      for (int c = 0; c < CPT; ++c) { cnt0[c] = cnt[c]; v1[c] = v[c]; cnt1[c] = cnt[c]; }
+      uint32_t dmask = 0;                                  // LTD-active columns of this thread (R10)
+#pragma unroll
+      for (int c = 0; c < CPT; ++c)
+        if ((valid >> c & 1u) && lpost[c] >= 0 && (tbase + k0 - lpost[c]) < L_dep) dmask |= 1u << c;
+      const uint32_t wdirty = __ballot_sync(FULL, dmask != 0);
+      int kk = k0;
+      int p_done = k0 - 1;           // last step fully processed by this thread
+      int cstep = kNoStep;           // crossing step (the warp stops right after it)
+      int hstep = kNoStep;           // undo log full: stopped before this step
+      unsigned long long ckey = 0ull;
+      int nlog = 0;
+      int dr0 = INT_MIN;             // warp-uniform raw start of the drawn LTD row range [dr0, dr0 + 32)
+      uint32_t evm[CPT];
+#pragma unroll
+      for (int c = 0; c < CPT; ++c) evm[c] = 0u;
+
+      // LTD draws of every (lane, column) pair of the warp for raw rows [base, base + 32): lanes over rows
+      auto draw = [&](int base) {
+        const uint32_t rr = s_rraw[base + lane];
+        const int t = tbase + ka + (int)(rr >> 16);
+        const uint32_t i = rr & 0xFFFFu;
+        const bool ok = (rr >> 16) != 0xFFFFu && base + lane < (int)s_offs[kend - ka];
+#pragma unroll 1
+        for (uint32_t lm = wdirty; lm; lm &= lm - 1) {
+          const int Ls = __ffs(lm) - 1;
+          const uint32_t dm = __shfl_sync(FULL, dmask, Ls);
+#pragma unroll
+          for (int c = 0; c < CPT; ++c) {
+            if (!(dm >> c & 1u)) continue;                 // warp-uniform
+            const int jl = __shfl_sync(FULL, jcol[c], Ls);
+            const int lp = __shfl_sync(FULL, lpost[c], Ls);
+            const int jg = cbase + col0 + jl;
+            const int D = t - lp;
+            bool bit = false;
+            if (ok && D < L_dep) {
+              const uint4 u = philox((uint32_t)t, i, (uint32_t)(jg >> 2), TAG_LTD, seed);   // eq.(7), R13
+              bit = pick(u, jg & 3) <= s_dep[D];
+            }
+            const uint32_t m = __ballot_sync(FULL, bit);
+            if (lane == Ls) evm[c] = m;
+          }
+        }
+      };
+
+#ifdef SNN_LEAN_DEBUG
+      long long dbg_it = 0;
+#endif
+      while (true) {
+#ifdef SNN_LEAN_DEBUG
+        if (++dbg_it > 20000) {
+          if (lane == 0) printf("SPIN rank %d warp %d k0 %d kk %d kend %d flag %d\n", rank, warp, k0, kk, kend,
+                                ld_volatile_shared_u32addr(flag_addr));
+          __trap();
+        }
+#endif
+        // one lane's read of the early-stop flag decides for the warp (lanes that executed the load apart
+        // could otherwise see different values and leave the loop apart)
+        const int fl = __shfl_sync(FULL, ld_volatile_shared_u32addr(flag_addr), 0);
+        if (kk >= kend || kk > fl) break;                        // warp-uniform
+        const int x = kk - ka;
+        const int o0 = (int)s_offs[x], o1 = (int)s_offs[x + 1];
+        bool live = false;
+#pragma unroll
+        for (int c = 0; c < CPT; ++c) live |= (valid >> c & 1u) && cnt[c] == 0;
+        const bool wlive = __any_sync(FULL, live);
+        if (!wlive && wdirty == 0u) {                            // held warp: skip the run in O(1)
+          int mc = INT_MAX;
+#pragma unroll
+          for (int c = 0; c < CPT; ++c) if (valid >> c & 1u) mc = min(mc, cnt[c]);
+          mc = __reduce_min_sync(FULL, mc);
+          int n = min(mc, kend - kk);
+          if (fl != INT_MAX) n = min(n, fl - kk + 1);
+          if (kk == k0) {
+#pragma unroll
+            for (int c = 0; c < CPT; ++c) { v1[c] = v[c]; cnt1[c] = (valid >> c & 1u) ? cnt[c] - 1 : cnt[c]; }
+          }
+#pragma unroll
+          for (int c = 0; c < CPT; ++c) if (valid >> c & 1u) cnt[c] -= n;
+          kk += n;
+          p_done = kk - 1;
+          continue;
+        }
+        // ---- this step's LTD events of the warp's LTD-active pairs (draws cover 32 rows ahead)
+        const bool big = (o1 - o0) > 32;
+        int nev = 0;
+        if (wdirty) {
+          if (!big && (o0 < dr0 || o1 > dr0 + 32)) { draw(o0); dr0 = o0; }
+          if (!big) {
+            const uint32_t sm = (o1 > o0) ? (((o1 - o0) == 32 ? FULL : ((1u << (o1 - o0)) - 1u)) << (o0 - dr0)) : 0u;
+#pragma unroll
+            for (int c = 0; c < CPT; ++c) nev += __popc(evm[c] & sm);
+          } else {
+            nev = __popc(dmask) * (o1 - o0);                     // conservative bound (steps of > 32 rows)
+          }
+          // undo-log space for this step (steps after k0 are logged); else stop before it
+          const bool full = kk > k0 && nlog + nev > logn;
+          if (__any_sync(FULL, full)) {
+            if (full) hstep = kk;
+            break;
+          }
+        }
+        // ---- (a2) eq.(3) + (a3) eqs.(1)(2): integrate the step's rows, Euler step of live columns
+        uint32_t cm = 0;
+        if (wlive) {
+          int S[CPT];
+#pragma unroll
+          for (int c = 0; c < CPT; ++c) S[c] = 0;
+          const int ps = (int)s_pst[x], pe = (int)s_pst[x + 1];
+          int q = ps;
+          while (q < pe) {
+            const int qe = min(pe, q + Z::CHUNK);
+            uint32_t acc = 0u;
+            for (; q < qe; q += 4) {
+              const uint4 m = *reinterpret_cast<const uint4*>(s_prow + q);
+              acc += ((wcol[m.x] >> fsh) & Z::LMASK) + ((wcol[m.y] >> fsh) & Z::LMASK) +
+                     ((wcol[m.z] >> fsh) & Z::LMASK) + ((wcol[m.w] >> fsh) & Z::LMASK);
+            }
+#pragma unroll
+            for (int c = 0; c < CPT; ++c)
+              S[c] += (int)(Z::LW == 32 ? acc : ((acc >> (c * Z::LW)) & ((1u << (Z::LW & 31)) - 1u)));
+          }
+#pragma unroll
+          for (int c = 0; c < CPT; ++c) {
+            if (!(valid >> c & 1u)) continue;
+            if (cnt[c] > 0) { --cnt[c]; continue; }                 // refractory / inhibited: hold v (R6, R7)
+            if (lif.step_t<FIXED>(v[c], S[c])) cm |= 1u << c;       // eq.(2): v > v_th
+          }
+        } else {
+#pragma unroll
+          for (int c = 0; c < CPT; ++c) if ((valid >> c & 1u) && cnt[c] > 0) --cnt[c];
+        }
+        // ---- (a5) LTD events of the step (old last_post, R14), applied in step order
+        if (wdirty && dmask) {
+          const int t = tbase + kk;
+          if (!big) {
+#pragma unroll
+            for (int c = 0; c < CPT; ++c) {
+              if (!(dmask >> c & 1u)) continue;
+              uint32_t em = (o1 > o0) ? ((evm[c] >> (o0 - dr0)) & ((o1 - o0) == 32 ? FULL : ((1u << (o1 - o0)) - 1u))) : 0u;
+              const int shc = fsh + c * Z::LW;
+              while (em) {
+                const int xr = __ffs(em) - 1;
+                em &= em - 1;
+                const int i = (int)(s_rraw[o0 + xr] & 0xFFFFu);
+                uint32_t* pw = s_w + i * wpr + wj;
+                const bool applied = ((*pw >> shc) & FMASK) != 0u;
+                if (applied) atomicSub(pw, 1u << shc);
+                ++ltd_events;
+                if (kk > k0) s_log[nlog++ * nthr + tid] = lean_log_entry(kk - k0, c, applied, i);
+              }
+            }
+          } else {
+            // steps with more than 32 active rows: the lane draws its own rows serially (rare)
+#pragma unroll
+            for (int c = 0; c < CPT; ++c) {
+              if (!(dmask >> c & 1u)) continue;
+              const int D = t - lpost[c];
+              if (D >= L_dep) continue;
+              const uint32_t thr = s_dep[D];
+              const int jg = cbase + col0 + jcol[c];
+              const int shc = fsh + c * Z::LW;
+              for (int r = o0; r < o1; ++r) {
+                const int i = (int)(s_rraw[r] & 0xFFFFu);
+                const uint4 u = philox((uint32_t)t, (uint32_t)i, (uint32_t)(jg >> 2), TAG_LTD, seed);
+                if (pick(u, jg & 3) <= thr) {
+                  uint32_t* pw = s_w + i * wpr + wj;
+                  const bool applied = ((*pw >> shc) & FMASK) != 0u;
+                  if (applied) atomicSub(pw, 1u << shc);
+                  ++ltd_events;
+                  if (kk > k0) s_log[nlog++ * nthr + tid] = lean_log_entry(kk - k0, c, applied, i);
+                }
+              }
+            }
+          }
+        }
+        if (kk == k0) {
+#pragma unroll
+          for (int c = 0; c < CPT; ++c) { v1[c] = v[c]; cnt1[c] = cnt[c]; }
+        }
+        p_done = kk;
+        if (cm) {                                                // crossing: the WTA key (R7)
+          cstep = kk;
+#pragma unroll
+          for (int c = 0; c < CPT; ++c) {
+            if (!(cm >> c & 1u)) continue;
+            const unsigned long long key = ((unsigned long long)lif.ord(v[c]) << 32) |
+                                           (0xFFFFFFFFu - (uint32_t)(cbase + col0 + jcol[c]));
+            ckey = key > ckey ? key : ckey;
+          }
+          atomicMin(&s_flag[fp], kk);
+          for (int r = 0; r < cs; ++r)
+            if (r != rank) red_min_cluster(&s_flag[fp], (uint32_t)r, kk);
+        }
+        if (__any_sync(FULL, cm != 0)) break;
+        ++kk;
+      }
+      if (hstep != kNoStep) {                                    // tell the cluster where to stop
+        ++eng_hz;
+        atomicMin(&s_flag[fp], hstep - 1);
+        for (int r = 0; r < cs; ++r)
+          if (r != rank) red_min_cluster(&s_flag[fp], (uint32_t)r, hstep - 1);
+      }
+      if (valid) eng_spec += (uint32_t)(p_done - k0 + 1) * (uint32_t)__popc(valid);
+
+      // ---------------------------------------------------------- CTA summary -> cluster exchange
+#ifdef SNN_LEAN_DEBUG
+      if (lane == 0 && k0 >= 116) printf("SPEC r %d w %d k0 %d kk %d p_done %d cstep %d hstep %d\n", rank, warp, k0, kk, p_done, cstep, hstep);
+#endif
+      {
+        const int wc = __reduce_min_sync(FULL, cstep);
+        const int wh = __reduce_min_sync(FULL, hstep);
+        const uint32_t kh = __reduce_max_sync(FULL, cstep == wc ? (uint32_t)(ckey >> 32) : 0u);
+        const uint32_t kl = __reduce_max_sync(FULL, (cstep == wc && (uint32_t)(ckey >> 32) == kh) ? (uint32_t)ckey : 0u);
+        if (lane == 0) {
+          s_wsum[2 * warp] = ((unsigned long long)(uint32_t)wc << 32) | (uint32_t)wh;
+          s_wsum[2 * warp + 1] = ((unsigned long long)kh << 32) | kl;
+        }
+      }
+      __syncthreads();
+      if (warp == 0) {
+        const unsigned long long none = ((unsigned long long)kNoStep << 32) | (uint32_t)kNoStep;
+        const unsigned long long a = lane < nwarps ? s_wsum[2 * lane] : none;
+        const unsigned long long k = lane < nwarps ? s_wsum[2 * lane + 1] : 0ull;
+        const int wc = (int)(a >> 32), wh = (int)(uint32_t)a;
+        const int C = __reduce_min_sync(FULL, wc);
+        const int H = __reduce_min_sync(FULL, wh);
+        const uint32_t kh = __reduce_max_sync(FULL, wc == C ? (uint32_t)(k >> 32) : 0u);
+        const uint32_t kl = __reduce_max_sync(FULL, (wc == C && (uint32_t)(k >> 32) == kh) ? (uint32_t)k : 0u);
+        const unsigned long long A = ((unsigned long long)(uint32_t)C << 32) | (uint32_t)H;
+        const unsigned long long K = ((unsigned long long)kh << 32) | kl;
+        unsigned long long* slot = s_slots + (size_t)(fp * kMaxCluster + rank) * 2;
+        if (cs == 1) {
+          if (lane == 0) { slot[0] = A; slot[1] = K; }
+        } else if (lane < cs) {
+          st_cluster_u64(slot, (uint32_t)lane, A);
+          st_cluster_u64(slot + 1, (uint32_t)lane, K);
+        }
+        if (lane == 0) s_flag[fp ^ 1] = INT_MAX;
+      }
+      if (cs > 1) { cluster_arrive(); cluster_wait(); } else { __syncthreads(); }   // the one cross-SM exchange
+
+      // ---------------------------------------------------------- global decision
+      int P, H;
+      unsigned long long K;
+      {
+        const unsigned long long none = ((unsigned long long)kNoStep << 32) | (uint32_t)kNoStep;
+        const unsigned long long A = lane < cs ? s_slots[(size_t)(fp * kMaxCluster + lane) * 2] : none;
+        const unsigned long long Kr = lane < cs ? s_slots[(size_t)(fp * kMaxCluster + lane) * 2 + 1] : 0ull;
+        const int c = (int)(A >> 32), h = (int)(uint32_t)A;
+        P = __reduce_min_sync(FULL, c);
+        H = __reduce_min_sync(FULL, h);
+        const uint32_t kh = __reduce_max_sync(FULL, c == P ? (uint32_t)(Kr >> 32) : 0u);
+        const uint32_t kl = __reduce_max_sync(FULL, (c == P && (uint32_t)(Kr >> 32) == kh) ? (uint32_t)Kr : 0u);
+        K = ((unsigned long long)kh << 32) | kl;
+      }
+      const bool event = P < kend && P < H;          // a post spike at t* = P
+#ifdef SNN_LEAN_DEBUG
+      if (tid == 0 && k0 >= 116) printf("EP r %d b %d k0 %d ka %d kend %d P %d H %d\n", rank, b, k0, ka, kend, P, H);
+#endif
+      const int k_last = event ? P : (H < kend ? H - 1 : kend - 1);   // last committed step
+
+      // ---------------------------------------------------------- per-thread resolution
+      auto undo_after = [&](int rel_keep) {           // undo logged LTD of steps k0 + rel > k0 + rel_keep
+        while (nlog > 0) {
+          const uint32_t e = s_log[(nlog - 1) * nthr + tid];
+          if ((int)(e >> 16) <= rel_keep) break;
+          if (e & 0x2000u) atomicAdd(s_w + (int)(e & 0x1FFFu) * wpr + wj, 1u << (fsh + (int)((e >> 14) & 3u) * Z::LW));
+          --ltd_events;
+          --nlog;
+          ++eng_undo;
+        }
+      };
+      if (event) {
+        const uint32_t W = 0xFFFFFFFFu - (uint32_t)K;
+        undo_after(P - k0);
+        bool me_any = false;
+#pragma unroll
+        for (int c = 0; c < CPT; ++c) {
+          if (!(valid >> c & 1u)) continue;
+          const bool me = (uint32_t)(cbase + col0 + jcol[c]) == W;
+          // no crossing in [k0, t*) anywhere: the countdown only ran down (R6, R7), v is reset anyway
+          const int cnt_p = max(cnt0[c] - (P - k0 + 1), 0);
+          if (me) {
+            v[c] = vreset; cnt[c] = t_ref;
+            if (rec_out) atomicOr(&d.raster_out[(size_t)P * d.nwe + ((col0 + jcol[c]) >> 5)], 1u << ((col0 + jcol[c]) & 31));
+            me_any = true;
+          } else {
+            v[c] = vreset; cnt[c] = max(cnt_p, t_inh);
+          }
+        }
+        (void)me_any;
+        ++img_spikes;
+      } else if (p_done > k_last) {                    // undo log full somewhere: replay [k0 + 1, k_last]
+        ++eng_resim;
+        undo_after(0);
+#pragma unroll
+        for (int c = 0; c < CPT; ++c) { v[c] = v1[c]; cnt[c] = cnt1[c]; }
+        const int t_unused = 0; (void)t_unused;
+        for (int k2 = k0 + 1; k2 <= k_last; ++k2) {
+          const int x2 = k2 - ka;
+          int S[CPT];
+#pragma unroll
+          for (int c = 0; c < CPT; ++c) S[c] = 0;
+          for (int r = (int)s_offs[x2]; r < (int)s_offs[x2 + 1]; ++r) {
+            const int i = (int)(s_rraw[r] & 0xFFFFu);
+            const uint32_t w = s_w[i * wpr + wj];
+#pragma unroll
+            for (int c = 0; c < CPT; ++c) S[c] += (int)((w >> (fsh + c * Z::LW)) & FMASK);
+          }
+#pragma unroll
+          for (int c = 0; c < CPT; ++c) {
+            if (!(valid >> c & 1u)) continue;
+            if (cnt[c] > 0) --cnt[c]; else lif.step_t<FIXED>(v[c], S[c]);
+          }
+          const int t = tbase + k2;
+#pragma unroll
+          for (int c = 0; c < CPT; ++c) {
+            if (!(dmask >> c & 1u) || (t - lpost[c]) >= L_dep) continue;
+            const uint32_t thr = s_dep[t - lpost[c]];
+            const int jg = cbase + col0 + jcol[c];
+            const int shc = fsh + c * Z::LW;
+            for (int r = (int)s_offs[x2]; r < (int)s_offs[x2 + 1]; ++r) {
+              const int i = (int)(s_rraw[r] & 0xFFFFu);
+              const uint4 u = philox((uint32_t)t, (uint32_t)i, (uint32_t)(jg >> 2), TAG_LTD, seed);
+              if (pick(u, jg & 3) <= thr) {
+                uint32_t* pw = s_w + i * wpr + wj;
+                if ((*pw >> shc) & FMASK) atomicSub(pw, 1u << shc);
+                ++ltd_events;
+              }
+            }
+          }
+        }
+      }
+      // LTD trials of the committed steps (draws with D < L_dep, R20)
+#pragma unroll
+      for (int c = 0; c < CPT; ++c) {
+        if (!(dmask >> c & 1u)) continue;
+        const int last = min(k_last, lpost[c] + L_dep - 1 - tbase);
+        if (last >= k0) ltd_trials += s_offs[last + 1 - ka] - s_offs[k0 - ka];
+      }
+      nlog = 0;
+
+      // ---------------------------------------------------------- LTP at t* in the winner's CTA (eq.(6))
+      if (event) {
+        const int Wl = (int)(0xFFFFFFFFu - (uint32_t)K) - cbase - col0;     // winner's local column
+        const int tP = tbase + P;
+#pragma unroll
+        for (int c = 0; c < CPT; ++c)
+          if ((valid >> c & 1u) && jcol[c] == Wl) lpost[c] = tP;             // after LTD at t* (R14)
+        if (Wl >= 0 && Wl < ncols) {                                           // CTA-uniform
+          __syncthreads();
+          lpre_catch_up(P - ka);                                               // last_pre includes step t*
+          __syncthreads();
+          const int Wg = cbase + col0 + Wl;
+          const int ww = Wl / CPW, wsh = (Wl % CPW) * BITS;
+          for (int grp = tid; grp < nq4; grp += nthr) {
+            const uint4 u = philox((uint32_t)tP, (uint32_t)Wg, (uint32_t)grp, TAG_LTP, seed);
+#pragma unroll
+            for (int r = 0; r < 4; ++r) {
+              const int i = 4 * grp + r;
+              if (i >= n_in) break;
+              const int lpi = s_lpre[i];
+              if (lpi < 0) continue;
+              const int D = tP - lpi;                                          // R10: Dt = D >= 0
+              if (D >= L_pot) continue;
+              ++ltp_trials;
+              if (pick(u, r) <= s_pot[D]) {
+                ++ltp_events;
+                uint32_t* pw = s_w + i * wpr + ww;
+                if (((*pw >> wsh) & FMASK) < (uint32_t)qmax) atomicAdd(pw, 1u << wsh);
+              }
+            }
+          }
+          __syncthreads();
+        }
+      }
+      k0 = k_last + 1;
+      ++ep;
+      ++eng_epochs;
+    }  // epochs
+
+    if (rank == 0 && tid == 0) {
+      post_sum += (unsigned long long)img_spikes;
+      if (d.spike_counts) d.spike_counts[b] = img_spikes;
+    }
+    if (last_img) {
+#pragma unroll
+      for (int c = 0; c < CPT; ++c)
+        if (valid >> c & 1u) {
+          const int jg = col0 + jcol[c];
+          d.v[jg] = v[c]; d.cnt[jg] = cnt[c]; d.last_post[jg] = lpost[c];
+        }
+      __syncthreads();
+      if (kb > ka) lpre_catch_up(kb - 1 - ka);
+      __syncthreads();
+      if (rank == 0) for (int i = tid; i < n_in; i += nthr) d.last_pre[i] = s_lpre[i];
+    } else if (kb > ka) {
+      // the next image resets the timers (R5); nothing to finish
+    }
+    __syncthreads();
+  }  // images
+
+  {
+    uint4* dst = reinterpret_cast<uint4*>(d.wslices + (size_t)rank * slice_words);
+    const uint4* src = reinterpret_cast<const uint4*>(s_w);
+    for (int k = tid; k < slice_words / 4; k += nthr) dst[k] = src[k];
+  }
+  {
+    unsigned long long a = ltd_trials, b2 = ltd_events, c = ltp_trials, e = ltp_events;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      a += __shfl_xor_sync(FULL, a, o); b2 += __shfl_xor_sync(FULL, b2, o);
+      c += __shfl_xor_sync(FULL, c, o); e += __shfl_xor_sync(FULL, e, o);
+    }
+    if (lane == 0) {
+      if (a) atomicAdd(&d.stats[2], a);
+      if (b2) atomicAdd(&d.stats[3], b2);
+      if (c) atomicAdd(&d.stats[4], c);
+      if (e) atomicAdd(&d.stats[5], e);
+    }
+    if (rank == 0 && tid == 0) {
+      atomicAdd(&d.stats[0], act_sum);
+      atomicAdd(&d.stats[1], post_sum);
+      atomicAdd(&d.stats[6], (unsigned long long)n_images);
+      atomicAdd(&d.stats[7], (unsigned long long)n_images * (unsigned long long)T);
+      atomicAdd(&d.stats[8], (unsigned long long)eng_epochs);
+    }
+    unsigned long long h2 = eng_hz, r2 = eng_resim, s2 = eng_spec, u2 = eng_undo;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      h2 += __shfl_xor_sync(FULL, h2, o); r2 += __shfl_xor_sync(FULL, r2, o);
+      s2 += __shfl_xor_sync(FULL, s2, o); u2 += __shfl_xor_sync(FULL, u2, o);
+    }
+    if (lane == 0) {
+      if (h2) atomicAdd(&d.stats[9], h2);
+      if (r2) atomicAdd(&d.stats[10], r2);
+      if (s2) atomicAdd(&d.stats[11], s2);
+      if (u2) atomicAdd(&d.stats[12], u2);
+    }
+  }
+#ifdef SNN_LEAN_DEBUG
+  if (tid == 0) printf("END r %d\n", rank);
+#endif
+  if (cs > 1) { cluster_arrive(); cluster_wait(); }
+}
+
+// ====================================================================== host launchers
+template <int BITS, int CPT, bool FIXED>
+static cudaError_t lean_launch_t(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, cudaStream_t s,
+                                 int* occupancy_out) {
+  cudaError_t e = cudaFuncSetAttribute(present_lean_kernel<BITS, CPT, FIXED>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)smem);
+  if (e != cudaSuccess) return e;
+  if (cs > 8) {
+    e = cudaFuncSetAttribute(present_lean_kernel<BITS, CPT, FIXED>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+    if (e != cudaSuccess) return e;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cudaLaunchAttribute attr[1];
+  cfg.gridDim = dim3((unsigned)(n_nets * cs));
+  cfg.blockDim = dim3((unsigned)nthr);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cfg.attrs = attr;
+  cfg.numAttrs = 0;
+  if (cs > 1) {
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = (unsigned)cs;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.numAttrs = 1;
+  }
+  if (occupancy_out) {
+    if (cs == 1) return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occupancy_out, present_lean_kernel<BITS, CPT, FIXED>, nthr, smem);
+    return cudaOccupancyMaxActiveClusters(occupancy_out, present_lean_kernel<BITS, CPT, FIXED>, &cfg);
+  }
+  return cudaLaunchKernelEx(&cfg, present_lean_kernel<BITS, CPT, FIXED>, lp);
+}
+
+template <int BITS, int CPT>
+static cudaError_t lean_dispatch_f(int fixed, const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem,
+                                   cudaStream_t s, int* occ) {
+  return fixed ? lean_launch_t<BITS, CPT, true>(lp, n_nets, cs, nthr, smem, s, occ)
+               : lean_launch_t<BITS, CPT, false>(lp, n_nets, cs, nthr, smem, s, occ);
+}
+
+static cudaError_t lean_dispatch(int bits, int cpt, int fixed, const LaunchParams& lp, int n_nets, int cs, int nthr,
+                                 size_t smem, cudaStream_t s, int* occ) {
+  if (bits == 2) {
+    if (cpt == 4) return lean_dispatch_f<2, 4>(fixed, lp, n_nets, cs, nthr, smem, s, occ);
+    if (cpt == 1) return lean_dispatch_f<2, 1>(fixed, lp, n_nets, cs, nthr, smem, s, occ);
+    return lean_dispatch_f<2, 2>(fixed, lp, n_nets, cs, nthr, smem, s, occ);
+  }
+  if (bits == 4) {
+    if (cpt == 1) return lean_dispatch_f<4, 1>(fixed, lp, n_nets, cs, nthr, smem, s, occ);
+    return lean_dispatch_f<4, 2>(fixed, lp, n_nets, cs, nthr, smem, s, occ);
+  }
+  return lean_dispatch_f<8, 1>(fixed, lp, n_nets, cs, nthr, smem, s, occ);
+}
+
+cudaError_t query_max_clusters_lean(int bits, int cpt, int fixed, int cs, int nthr, size_t smem, int* out) {
+  LaunchParams lp{};
+  return lean_dispatch(bits, cpt, fixed, lp, 1, cs, nthr, smem, 0, out);
+}
+
+cudaError_t launch_present_lean(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, int bits, int cpt,
+                                int fixed, cudaStream_t s) {
+  return lean_dispatch(bits, cpt, fixed, lp, n_nets, cs, nthr, smem, s, nullptr);
+}
+
+}  // namespace snn

@@ -26,7 +26,7 @@ EXPORTS = [
     "snn_create_shard", "snn_shard_ipc_handle", "snn_shard_connect", "snn_shard_link",
 ]
 SNN_IPC_HANDLE_BYTES = 64
-NINFO = 16
+NINFO = 18
 
 
 class SnnParams(ctypes.Structure):
@@ -195,7 +195,8 @@ class Network:
         a = (ctypes.c_int64 * NINFO)()
         _check(lib().snn_get_info(self._h, a), "snn_get_info")
         keys = ["cluster_size", "threads", "smem_bytes", "words_per_row", "q_max", "L_pot", "L_dep", "launches",
-                "engine", "cols_per_thread", "row_window", "log_depth", "col_base", "n_exc_total", "world", "shard"]
+                "engine", "cols_per_thread", "row_window", "log_depth", "col_base", "n_exc_total", "world", "shard",
+                "lean", "smem_lean"]
         return dict(zip(keys, [int(x) for x in a]))
 
     def set_stream(self, stream_ptr: int):

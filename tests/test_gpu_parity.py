@@ -14,7 +14,9 @@ from oracle import oracle as O
 pytestmark = pytest.mark.gpu
 
 
-ENGINES = [0, 1]   # SNN_ENGINE_EVENT (event-driven epochs), SNN_ENGINE_STEP (per-step exchange)
+# SNN_ENGINE_EVENT (event-driven epochs; the lean kernel where HARD + RESET + stochastic applies),
+# SNN_ENGINE_STEP (per-step exchange), SNN_ENGINE_EVENT_GENERAL (the general event kernel everywhere)
+ENGINES = [0, 1, 2]
 
 
 def _pair(n_in, n_exc, bits, p, engine=0):
@@ -163,6 +165,18 @@ def test_C4_hf_variant(gpu, engine):
     _compare_presentations(g, o, synthdata.images(1, "fashion", start=5), 100, synthdata.seeds(1, 9), 784, 6400, 1)
 
 
+@pytest.mark.parametrize("preset,wta,inh,stdp,lean", [("2b", 0, 0, 0, 1), ("8b", 0, 0, 0, 1), ("8b", 1, 0, 0, 0),
+                                                      ("8b", 0, 1, 0, 0), ("8b", 0, 0, 1, 0)])
+def test_lean_kernel_selection(gpu, preset, wta, inh, stdp, lean):
+    """The default learning mode (HARD WTA, RESET inhibition, stochastic STDP) runs the lean kernel;
+    every other mode, and SNN_ENGINE_EVENT_GENERAL, runs the general event kernel."""
+    p = O.params(preset, wta_mode=wta, inh_mode=inh, stdp_mode=stdp)
+    g, _ = _pair(784, 400, 8 if preset == "8b" else 2, p, engine=0)
+    assert g.info()["lean"] == lean
+    g2, _ = _pair(784, 400, 8 if preset == "8b" else 2, p, engine=2)
+    assert g2.info()["lean"] == 0
+
+
 # ------------------------------------------------------------------ C5: ensemble, one launch
 @pytest.mark.parametrize("engine", ENGINES)
 def test_C5_ensemble_present_many(gpu, engine):
@@ -266,5 +280,5 @@ def test_undo_log_overflow_path(gpu, engine):
                  membrane_mode=1, init_seed=13)
     g, o = _pair(784, 256, 2, p, engine=engine)
     _compare_presentations(g, o, synthdata.images(2, "fashion", start=3), 120, synthdata.seeds(2, 13), 784, 256, 1)
-    if engine == 0:
+    if engine in (0, 2):
         assert int(g.stats()[9]) > 0, "undo-log overflow path not exercised"
