@@ -342,8 +342,16 @@ def main():
     smclk = (clocks.get("sm_max_mhz") or 1965.0)
     peak_smem = SMEM_BYTES_PER_CLK_PER_SM * N_SM * smclk * 1e6 / 1e9   # GB/s, whole chip
     achieved = per_launch_bytes / per_launch_s / 1e9
+    traffic, traffic_src = None, "no committed ncu --set full capture at this launch shape"
+    try:                               # dram bytes of ONE launch of the same shape, from a committed capture
+        cap = json.load(open(os.path.join(ROOT, "profiles", "ncu_full_latest.json")))
+        if cap.get("images_per_launch") == B and cap.get("n_exc") == N_EXC and K == 1 and not sharded:
+            traffic = cap["dram_bytes_per_launch"]
+            traffic_src = f"profiles/ncu_full_latest.json ({cap['kernel']}, {cap['source']})"
+    except (OSError, ValueError, KeyError):
+        pass
     roofline = {"bound": "smem", "achieved": achieved, "peak": peak_smem, "unit": "GB/s", "frac": achieved / peak_smem,
-                "traffic": None,
+                "traffic": traffic, "traffic_source": traffic_src,
                 "peak_source": f"derived: 128 B/clk/SM (B300_MICROARCH smem crossbar) x {N_SM} SMs x {smclk:.0f} MHz",
                 "alg_bytes_per_launch": per_launch_bytes,
                 "note": "latency-bound step loop; see latency_roofline"}

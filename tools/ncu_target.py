@@ -11,7 +11,7 @@ import synthdata  # noqa: E402
 import paper_conf_date_shelm19_b200 as P  # noqa: E402
 
 ap = argparse.ArgumentParser()
-ap.add_argument("--images", type=int, default=4)
+ap.add_argument("--images", type=int, default=32)
 ap.add_argument("--n-exc", type=int, default=6400)
 a = ap.parse_args()
 net = P.Network(784, a.n_exc, 2, P.preset("2b", membrane_mode=0))
