@@ -18,6 +18,7 @@ _LIB_PATH = os.path.join(_HERE, "liboracle.so")
 
 ORACLE_RASTER_INPUT = 1
 ORACLE_KEEP_STATE = 2
+ORACLE_NO_LEARN = 8
 
 
 class OracleParams(ctypes.Structure):
@@ -116,6 +117,12 @@ def lib():
         L.oracle_lif_step_fp32.restype = ctypes.c_float
         L.oracle_lif_step_fixed.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32]
         L.oracle_lif_step_fixed.restype = ctypes.c_int32
+        L.oracle_infer.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int, ctypes.c_int, ctypes.c_void_p,
+                                   ctypes.c_void_p]
+        L.oracle_label.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_int,
+                                   ctypes.c_void_p]
+        L.oracle_classify.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_int,
+                                      ctypes.c_void_p]
         _lib = L
     return _lib
 
@@ -234,6 +241,38 @@ class OracleNet:
 
     def lif_step_fixed(self, v: int, S: int) -> int:
         return int(lib().oracle_lif_step_fixed(self._h, int(v), int(S)))
+
+    def infer(self, images: np.ndarray, T: int, seeds) -> np.ndarray:
+        """NEXT-1: spike counts (n_images, n_exc) u32 with frozen weights (R21)."""
+        imgs = np.ascontiguousarray(images, dtype=np.uint8).reshape(-1, self.n_in)
+        sd = np.ascontiguousarray(np.asarray(seeds, dtype=np.uint64).reshape(-1))
+        assert sd.size == imgs.shape[0]
+        out = np.zeros((imgs.shape[0], self.n_exc), dtype=np.uint32)
+        self._check(lib().oracle_infer(self._h, _ptr(imgs), imgs.shape[0], T, _ptr(sd), _ptr(out)), "oracle_infer")
+        self.last_T = T
+        return out
+
+
+def label(counts: np.ndarray, classes, n_classes: int) -> np.ndarray:
+    """R22: per-neuron class label from spike counts of labelled images (-1 = never spiked)."""
+    c = np.ascontiguousarray(counts, dtype=np.uint32)
+    cl = np.ascontiguousarray(np.asarray(classes, dtype=np.int32).reshape(-1))
+    out = np.zeros(c.shape[1], dtype=np.int32)
+    rc = lib().oracle_label(_ptr(c), c.shape[0], c.shape[1], _ptr(cl), n_classes, _ptr(out))
+    if rc != 0:
+        raise OracleError(rc, "oracle_label")
+    return out
+
+
+def classify(counts: np.ndarray, labels, n_classes: int) -> np.ndarray:
+    """R23: per-image predicted class by the labelled neurons' mean spike count (-1 = no vote)."""
+    c = np.ascontiguousarray(counts, dtype=np.uint32)
+    lb = np.ascontiguousarray(np.asarray(labels, dtype=np.int32).reshape(-1))
+    out = np.zeros(c.shape[0], dtype=np.int32)
+    rc = lib().oracle_classify(_ptr(c), c.shape[0], c.shape[1], _ptr(lb), n_classes, _ptr(out))
+    if rc != 0:
+        raise OracleError(rc, "oracle_classify")
+    return out
 
 
 def unpack_state(blob: np.ndarray, n_in: int, n_exc: int) -> dict:

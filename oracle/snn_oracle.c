@@ -320,8 +320,10 @@ int oracle_present_ex(oracle_net* n, const void* input, int T, uint64_t seed, in
       }
     }
 
-    /* 5 STDP */
-    if (p->stdp_mode == 0) {
+    /* 5 STDP (skipped with frozen weights: inference, R21) */
+    if (flags & ORACLE_NO_LEARN) {
+      /* no plasticity */
+    } else if (p->stdp_mode == 0) {
       /* LTD at a pre spike against the last post spike, eq.(7), Dt = -D < 0 [R10][R14]; dG = 1 LSB */
       for (int i = 0; i < n_in; ++i) {
         if (!s[i]) continue;
@@ -475,4 +477,78 @@ int oracle_lut(const oracle_net* n, int which, uint64_t* out, int cap) {
   if (cap < len) return E_SIZE;
   for (int k = 0; k < len; ++k) out[k] = src ? src[k] : (uint64_t)srci[k];
   return len;
+}
+
+/* ---------------------------------------------------------------- NEXT-1: labelling + inference
+ * P:88 §III-B: "After learning is complete, the first 1000 images in the test set are used to label all
+ * the neurons in the first layer. The rest of the test set, which contains 9000 images, are used for
+ * inference."  The labelling and voting rules are not stated; readings R21-R23. */
+int oracle_infer(oracle_net* n, const uint8_t* images, int n_images, int T, const uint64_t* seeds,
+                 uint32_t* counts) {
+  if (!n || n_images < 0 || T < 0 || (n_images > 0 && (!images || !seeds || !counts))) return E_INVAL;
+  const int we = (n->n_exc + 31) / 32;
+  for (int k = 0; k < n_images; ++k) {
+    int rc = oracle_present_ex(n, images + (size_t)k * n->n_in, T, seeds[k], ORACLE_NO_LEARN, 0);
+    if (rc) return rc;
+    for (int j = 0; j < n->n_exc; ++j) {
+      uint32_t c = 0;
+      for (int t = 0; t < T; ++t) c += (n->raster[(size_t)t * we + j / 32] >> (j % 32)) & 1u;
+      counts[(size_t)k * n->n_exc + j] = c;
+    }
+  }
+  return 0;
+}
+
+/* r_a / n_a > r_b / n_b, exactly (n_a, n_b > 0) */
+static int ratio_gt(uint64_t r_a, uint64_t n_a, uint64_t r_b, uint64_t n_b) {
+  return (unsigned __int128)r_a * n_b > (unsigned __int128)r_b * n_a;
+}
+
+int oracle_label(const uint32_t* counts, int n_images, int n_exc, const int32_t* classes, int n_classes,
+                 int32_t* labels) {
+  if (!counts || !classes || !labels || n_images < 0 || n_exc < 1 || n_classes < 1) return E_INVAL;
+  uint64_t* N = (uint64_t*)calloc((size_t)n_classes, sizeof(uint64_t));
+  uint64_t* r = (uint64_t*)calloc((size_t)n_classes, sizeof(uint64_t));
+  if (!N || !r) { free(N); free(r); return E_NOMEM; }
+  for (int k = 0; k < n_images; ++k) {
+    if (classes[k] < 0 || classes[k] >= n_classes) { free(N); free(r); return E_INVAL; }
+    N[classes[k]]++;
+  }
+  for (int j = 0; j < n_exc; ++j) {
+    for (int c = 0; c < n_classes; ++c) r[c] = 0;
+    for (int k = 0; k < n_images; ++k) r[classes[k]] += counts[(size_t)k * n_exc + j];
+    int best = -1;
+    for (int c = 0; c < n_classes; ++c) {
+      if (N[c] == 0 || r[c] == 0) continue;            /* no response to class c */
+      if (best < 0 || ratio_gt(r[c], N[c], r[best], N[best])) best = c;
+    }
+    labels[j] = best;
+  }
+  free(N); free(r);
+  return 0;
+}
+
+int oracle_classify(const uint32_t* counts, int n_images, int n_exc, const int32_t* labels, int n_classes,
+                    int32_t* pred) {
+  if (!counts || !labels || !pred || n_images < 0 || n_exc < 1 || n_classes < 1) return E_INVAL;
+  uint64_t* M = (uint64_t*)calloc((size_t)n_classes, sizeof(uint64_t));
+  uint64_t* s = (uint64_t*)calloc((size_t)n_classes, sizeof(uint64_t));
+  if (!M || !s) { free(M); free(s); return E_NOMEM; }
+  for (int j = 0; j < n_exc; ++j) {
+    if (labels[j] >= n_classes || labels[j] < -1) { free(M); free(s); return E_INVAL; }
+    if (labels[j] >= 0) M[labels[j]]++;
+  }
+  for (int k = 0; k < n_images; ++k) {
+    for (int c = 0; c < n_classes; ++c) s[c] = 0;
+    for (int j = 0; j < n_exc; ++j)
+      if (labels[j] >= 0) s[labels[j]] += counts[(size_t)k * n_exc + j];
+    int best = -1;
+    for (int c = 0; c < n_classes; ++c) {
+      if (M[c] == 0 || s[c] == 0) continue;
+      if (best < 0 || ratio_gt(s[c], M[c], s[best], M[best])) best = c;
+    }
+    pred[k] = best;
+  }
+  free(M); free(s);
+  return 0;
 }

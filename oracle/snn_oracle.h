@@ -49,6 +49,8 @@ int oracle_destroy(oracle_net* net);
 #define ORACLE_RASTER_INPUT 1  /* `input` is a T x ceil(n_in/32) u32 spike raster, encoder bypassed */
 #define ORACLE_KEEP_STATE   2  /* do not reset v/cnt/timers (R5); step indices start at t0 */
 
+#define ORACLE_NO_LEARN     8  /* frozen weights: steps 1-4 only, no STDP (inference; R21) */
+
 /* One presentation: T steps of the per-step loop.  image: n_in bytes (ignored with RASTER_INPUT). */
 int oracle_present(oracle_net* net, const uint8_t* image, int T, uint64_t seed);
 int oracle_present_ex(oracle_net* net, const void* input, int T, uint64_t seed, int flags, int t0);
@@ -67,6 +69,23 @@ int oracle_set_state(oracle_net* net, const void* buf, size_t n);
 /* counters of the last presentation: [0] sum_t act(t), [1] post spikes, [2] LTD trials,
  * [3] LTD events, [4] LTP trials, [5] LTP events */
 int oracle_get_stats(const oracle_net* net, uint64_t stats[8]);
+
+/* ---- NEXT-1: labelling and inference with frozen weights (§III-B "the first 1000 images in the
+ * test set are used to label all the neurons in the first layer. The rest of the test set ... are used
+ * for inference"; readings DESIGN.md R21-R23).
+ * oracle_infer: each image presented for T steps with ORACLE_NO_LEARN, state reset per image (R5);
+ *   counts[k*n_exc + j] = number of spikes of neuron j during image k.  Weights are not changed.
+ * oracle_label: labels[j] = argmax_c (sum_{k: classes[k]==c} counts[k][j]) / N_c over classes with
+ *   N_c > 0 images, ties -> lowest c; -1 if neuron j never spiked (R22).  classes[k] in [0, n_classes).
+ * oracle_classify: pred[k] = argmax_c (sum_{j: labels[j]==c} counts[k][j]) / M_c over classes with
+ *   M_c > 0 labelled neurons, ties -> lowest c; -1 if no labelled neuron spiked (R23).
+ * Ratios are compared exactly as integer cross products. */
+int oracle_infer(oracle_net* net, const uint8_t* images, int n_images, int T, const uint64_t* seeds,
+                 uint32_t* counts);
+int oracle_label(const uint32_t* counts, int n_images, int n_exc, const int32_t* classes, int n_classes,
+                 int32_t* labels);
+int oracle_classify(const uint32_t* counts, int n_images, int n_exc, const int32_t* labels, int n_classes,
+                    int32_t* pred);
 
 /* Exposed for the pin tests. */
 int oracle_q_max(const oracle_net* net);
