@@ -207,6 +207,37 @@ int snn_shard_connect(snn_handle* h, const void* handles, size_t n_bytes);
  * distinct peer-capable devices may be presented from one thread each. */
 int snn_shard_link(snn_handle* const* hs, int world);
 
+/* ---- NEXT-1: labelling and inference with frozen weights (R21-R23).
+ * P:88 §III-B: "After learning is complete, the first 1000 images in the test set are used to label
+ * all the neurons in the first layer. The rest of the test set, which contains 9000 images, are used
+ * for inference."
+ *
+ * snn_infer: present each of n_images images (n_images x n_in bytes) for T steps with the handle's
+ * current weights FROZEN (steps 1-4 of the loop, no STDP, R21): encoder, integration, LIF and WTA as
+ * in snn_present, state reset per image (R5), image k keyed by seeds[k].  counts (n_images x n_exc u32,
+ * row-major [k][j]) receives the number of spikes of neuron j during image k.  The images are
+ * independent and run in parallel (one CTA per image at a time, weights streamed from L2).
+ * Weights, state, rasters and the learning stats are not touched; stats [0]/[1] of snn_get_stats are
+ * not updated either (inference counters: snn_get_infer_stats).  All pointers host or device (the call
+ * stages host buffers); SNN_ASYNC returns after enqueueing.  T <= 65535; n_exc <= 7168;
+ * unsharded handles only.  Errors: SNN_EINVAL (arguments), SNN_ESIZE (n_exc too large), SNN_ECUDA.
+ * snn_get_infer_stats: [0] sum over images and steps of active input rows, [1] post spikes, since
+ * the handle was created.
+ *
+ * snn_label (R22): labels[j] (n_exc int32) = the class c maximising the MEAN count of neuron j over
+ * the labelling images of class c (counts: n_images x n_exc u32, classes: n_images int32 in
+ * [0, n_classes)); ties -> lowest class; -1 for a neuron that never spiked.  n_classes <= 64.
+ * snn_classify (R23): pred[k] (n_images int32) = the class whose labelled neurons have the highest
+ * MEAN count in image k; ties -> lowest class; -1 if no labelled neuron spiked.  Ratios are compared
+ * exactly (integer cross products).  Pointers host or device; synchronous. */
+int snn_infer(snn_handle* h, const uint8_t* images, int n_images, int T, const uint64_t* seeds, uint32_t* counts,
+              int flags);
+int snn_get_infer_stats(snn_handle* h, uint64_t stats[2]);
+int snn_label(snn_handle* h, const uint32_t* counts, int n_images, const int32_t* classes, int n_classes,
+              int32_t* labels);
+int snn_classify(snn_handle* h, const uint32_t* counts, int n_images, const int32_t* labels, int n_classes,
+                 int32_t* pred);
+
 const char* snn_last_error(void);
 
 #ifdef __cplusplus

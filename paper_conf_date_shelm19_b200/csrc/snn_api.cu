@@ -116,6 +116,15 @@ struct snn_handle {
   std::vector<void*> ipc_opened;       // peer mailboxes opened with cudaIpcOpenMemHandle
   std::vector<snn_handle*> linked;     // in-process shards (snn_shard_link), rank order
   bool connected = false;
+  // NEXT-1 inference: weights in the inference layout, rebuilt when w_version moves
+  long long w_version = 0, infer_version = -1;
+  uint32_t* d_winf = nullptr;     size_t winf_cap = 0;
+  uint32_t* d_iwords = nullptr;   size_t iwords_cap = 0;
+  uint32_t* d_icounts = nullptr;  size_t icounts_cap = 0;
+  uint32_t* d_iecnt = nullptr;    size_t iecnt_cap = 0;
+  int32_t* d_cls = nullptr;       size_t cls_cap = 0;
+  int32_t* d_lab = nullptr;       size_t lab_cap = 0;
+  unsigned long long* d_istats = nullptr;
 };
 
 namespace {
@@ -200,7 +209,8 @@ void free_all(snn_handle* h) {
                   h->d_v, h->d_cnt, h->d_lpost, h->d_lpre, h->d_stats, h->d_raster, h->d_inrec,
                   h->d_img, h->d_rin, h->d_seeds, h->d_counts, h->d_codes, h->d_bad,
                   h->d_words, h->d_ecnt, h->d_offs, h->d_rows, h->d_rows16, h->d_trace,
-                  h->d_mbox, h->d_peers};
+                  h->d_mbox, h->d_peers, h->d_winf, h->d_iwords, h->d_icounts, h->d_iecnt, h->d_cls,
+                  h->d_lab, h->d_istats};
   for (void* q : ptrs) if (q) cudaFree(q);
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
 }
@@ -303,6 +313,7 @@ int present_impl(snn_handle* h, const void* input, int n_images, int T, const ui
     if (o != h && o->dev == h->dev)
       return fail(SNN_EINVAL, "shards linked on one device must be presented together (snn_present_many)");
   DevGuard g(h->dev);
+  h->w_version++;                      // STDP may change the codes (inference layout is stale)
   NetDesc d;
   fill_static(h, d);
   d.n_images = n_images; d.T = T; d.flags = flags & 0x17; d.t0 = t0;
@@ -794,6 +805,7 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
       return fail(SNN_EINVAL, "ensemble handles must share n_in, cluster size, CTA shape, engine, membrane mode, device");
     for (int m = 0; m < k; ++m)
       if (hs[m] == hs[k]) return fail(SNN_EINVAL, "handle %d appears twice", k);
+    hs[k]->w_version++;
     if (hs[k]->world > 1) {        // every shard of its world must be in this launch (they wait on each other)
       if (hs[k]->linked.empty()) return fail(SNN_EINVAL, "shard handle %d is not linked in this process", k);
       for (snn_handle* o : hs[k]->linked)
@@ -944,6 +956,7 @@ int snn_set_weights(snn_handle* h, const uint8_t* codes, size_t n) {
   fill_static(h, d);
   CUDA_TRY(snn::launch_pack_weights(d, h->d_codes, h->stream));
   CUDA_TRY(cudaStreamSynchronize(h->stream));
+  h->w_version++;
   return SNN_OK;
 }
 
@@ -1072,6 +1085,197 @@ int snn_get_info(const snn_handle* h, int64_t info[SNN_NINFO]) {
   info[12] = h->col_base; info[13] = h->n_exc_total; info[14] = h->world; info[15] = h->shard;
   info[16] = h->lean ? 1 : 0; info[17] = (int64_t)h->smem_lean;
   return SNN_OK;
+}
+
+}  // extern "C"
+
+// ---------------------------------------------------------------- NEXT-1: inference, labelling, vote
+namespace {
+
+// Ring geometry of the inference kernel for this handle: the largest power-of-two ring (<= 64 rows)
+// that leaves room for two CTAs per SM, else one CTA per SM, at least 8 rows.
+int infer_geometry(const snn_handle* h, int* wpr, int* R, int* nthr, size_t* smem) {
+  const int ncols = (h->n_exc + 31) / 32;
+  *wpr = ((ncols * h->bits) + 3) & ~3;
+  const int row_bytes = *wpr * 4;
+  *nthr = (((ncols + 31) / 32) + 1) * 32;
+  int r = 64;
+  while (r > 8 && snn::infer_smem_bytes(r, row_bytes) > 110 * 1024) r >>= 1;
+  while (r > 8 && snn::infer_smem_bytes(r, row_bytes) > 220 * 1024) r >>= 1;
+  if (snn::infer_smem_bytes(r, row_bytes) > 220 * 1024) return fail(SNN_ESIZE, "inference ring does not fit");
+  *R = r;
+  *smem = snn::infer_smem_bytes(r, row_bytes);
+  return SNN_OK;
+}
+
+int infer_weights(snn_handle* h, int wpr) {
+  if (h->infer_version == h->w_version && h->d_winf) return SNN_OK;
+  int rc = ensure(h, &h->d_winf, &h->winf_cap, (size_t)h->n_in * wpr);
+  if (rc) return rc;
+  NetDesc d;
+  fill_static(h, d);
+  CUDA_TRY(snn::launch_unpack_weights(d, h->d_codes, h->stream));
+  CUDA_TRY(snn::launch_pack_infer(h->d_codes, h->n_in, h->n_exc, h->bits, wpr, h->d_winf, h->stream));
+  h->launches += 2;
+  h->infer_version = h->w_version;
+  return SNN_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int snn_infer(snn_handle* h, const uint8_t* images, int n_images, int T, const uint64_t* seeds, uint32_t* counts,
+              int flags) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  if (n_images < 0 || T < 0) return fail(SNN_EINVAL, "negative n_images / T");
+  if (T > 65535) return fail(SNN_EINVAL, "T=%d exceeds 65535 for inference", T);
+  if (h->world > 1) return fail(SNN_EINVAL, "inference runs on unsharded handles");
+  if (h->n_exc > snn::kInferMaxCols) return fail(SNN_ESIZE, "n_exc=%d exceeds %d for inference", h->n_exc,
+                                                 snn::kInferMaxCols);
+  if (n_images == 0) return SNN_OK;
+  if (!images || !seeds || !counts) return fail(SNN_EINVAL, "images / seeds / counts is NULL");
+  DevGuard g(h->dev);
+  int wpr, R, nthr;
+  size_t smem;
+  if ((rc = infer_geometry(h, &wpr, &R, &nthr, &smem))) return rc;
+  if ((rc = infer_weights(h, wpr))) return rc;
+  if (!h->d_istats) {
+    CUDA_TRY(dalloc(&h->d_istats, 2));
+    CUDA_TRY(cudaMemsetAsync(h->d_istats, 0, 2 * sizeof(unsigned long long), h->stream));
+  }
+  const uint8_t* img = nullptr;
+  if ((rc = stage(h, images, (size_t)n_images * h->n_in, &h->d_img, &h->img_cap, &img))) return rc;
+  const unsigned long long* sd = nullptr;
+  if ((rc = stage(h, reinterpret_cast<const unsigned long long*>(seeds), (size_t)n_images, &h->d_seeds,
+                  &h->seeds_cap, &sd)))
+    return rc;
+  const bool counts_dev = is_device_ptr(counts);
+  uint32_t* cnt = counts;
+  if (!counts_dev) {
+    if ((rc = ensure(h, &h->d_icounts, &h->icounts_cap, (size_t)n_images * h->n_exc))) return rc;
+    cnt = h->d_icounts;
+  }
+  int occ = 0;
+  CUDA_TRY(snn::infer_occupancy(h->bits, h->p.membrane_mode, nthr, smem, &occ));
+  if (occ < 1) return fail(SNN_ESIZE, "inference kernel cannot be resident (smem %zu B, %d threads)", smem, nthr);
+  int nsm = 0;
+  CUDA_TRY(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, h->dev));
+  const int nwi = (h->n_in + 31) / 32;
+  // the encoder pre-pass writes T x nwi words per image: process the batch in chunks of bounded scratch
+  const long long per_img = (long long)T * nwi;
+  const int chunk = (int)std::max(1LL, std::min<long long>(n_images, (256LL << 20) / 4 / std::max(1LL, per_img)));
+  if ((rc = ensure(h, &h->d_iwords, &h->iwords_cap, (size_t)chunk * per_img))) return rc;
+  if ((rc = ensure(h, &h->d_iecnt, &h->iecnt_cap, (size_t)chunk * T))) return rc;
+  CUDA_TRY(cudaMemsetAsync(cnt, 0, (size_t)n_images * h->n_exc * sizeof(uint32_t), h->stream));
+  snn::InferDesc d{};
+  const snn_params& p = h->p;
+  const double lsb = std::ldexp(1.0, -h->frac_bits);
+  d.n_in = h->n_in; d.n_exc = h->n_exc; d.bits = h->bits; d.T = T; d.nwi = nwi;
+  d.nthr_cols = (h->n_exc + 31) / 32; d.wpr = wpr; d.R = R; d.rmax = R / 2; d.row_bytes = wpr * 4;
+  d.af = (float)p.a; d.bf = (float)p.b; d.cf = (float)p.c; d.dtf = (float)p.dt_ms;
+  d.kI = (float)(p.v_spike * lsb); d.ief = (float)p.i_ext;
+  d.vthf = (float)p.v_th; d.vresetf = (float)p.v_reset; d.vinitf = (float)p.v_init;
+  d.A = h->A; d.B = h->B; d.C = h->C; d.E = h->E; d.Vth = h->Vth; d.Vreset = h->Vreset; d.Vinit = h->Vinit;
+  d.t_ref = p.t_ref_steps; d.t_inh = p.t_inh_steps; d.wta_mode = p.wta_mode; d.inh_mode = p.inh_mode;
+  d.w = h->d_winf; d.words = h->d_iwords; d.stats = h->d_istats;
+  for (int k0 = 0; k0 < n_images; k0 += chunk) {
+    const int nb = std::min(chunk, n_images - k0);
+    CUDA_TRY(snn::launch_encode(img + (size_t)k0 * h->n_in, h->d_enc, sd + k0, h->n_in, T, nb, 0, h->d_iwords,
+                                h->d_iecnt, h->stream));
+    d.n_images = nb;
+    d.counts = cnt + (size_t)k0 * h->n_exc;
+    int grid = std::min(nb, occ * nsm);
+    if (const char* e = std::getenv("SNN_INFER_MAX_GRID"))   // test hook: force the persistent image loop
+      if (std::atoi(e) > 0) grid = std::min(grid, std::atoi(e));
+    CUDA_TRY(snn::launch_infer(d, grid, nthr, smem, h->p.membrane_mode, h->stream));
+    h->launches += 2;
+  }
+  if (!counts_dev)
+    CUDA_TRY(cudaMemcpyAsync(counts, cnt, (size_t)n_images * h->n_exc * sizeof(uint32_t), cudaMemcpyDeviceToHost,
+                             h->stream));
+  return finish(h, flags);
+}
+
+int snn_get_infer_stats(snn_handle* h, uint64_t stats[2]) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  if (!stats) return fail(SNN_EINVAL, "stats is NULL");
+  stats[0] = stats[1] = 0;
+  if (!h->d_istats) return SNN_OK;
+  DevGuard g(h->dev);
+  CUDA_TRY(cudaMemcpyAsync(stats, h->d_istats, 2 * sizeof(uint64_t), cudaMemcpyDeviceToHost, h->stream));
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  return SNN_OK;
+}
+
+int snn_label(snn_handle* h, const uint32_t* counts, int n_images, const int32_t* classes, int n_classes,
+              int32_t* labels) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  if (!counts || !classes || !labels || n_images < 0) return fail(SNN_EINVAL, "bad labelling arguments");
+  if (n_classes < 1 || n_classes > snn::kMaxClasses) return fail(SNN_EINVAL, "n_classes outside [1, %d]", snn::kMaxClasses);
+  DevGuard g(h->dev);
+  std::vector<int32_t> hc;
+  if (!is_device_ptr(classes)) {       // validated on the host: a bad class id must not index out of bounds
+    for (int k = 0; k < n_images; ++k)
+      if (classes[k] < 0 || classes[k] >= n_classes) return fail(SNN_EINVAL, "classes[%d]=%d outside [0, %d)", k,
+                                                                  classes[k], n_classes);
+  } else {
+    hc.resize((size_t)n_images);
+    CUDA_TRY(cudaMemcpyAsync(hc.data(), classes, hc.size() * 4, cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    for (int k = 0; k < n_images; ++k)
+      if (hc[k] < 0 || hc[k] >= n_classes) return fail(SNN_EINVAL, "classes[%d]=%d outside [0, %d)", k, hc[k], n_classes);
+  }
+  const uint32_t* c = nullptr;
+  if ((rc = stage(h, counts, (size_t)n_images * h->n_exc, &h->d_icounts, &h->icounts_cap, &c))) return rc;
+  const int32_t* cl = nullptr;
+  if ((rc = stage(h, classes, (size_t)n_images, &h->d_cls, &h->cls_cap, &cl))) return rc;
+  const bool out_dev = is_device_ptr(labels);
+  int32_t* out = labels;
+  if (!out_dev) {
+    if ((rc = ensure(h, &h->d_lab, &h->lab_cap, (size_t)h->n_exc))) return rc;
+    out = h->d_lab;
+  }
+  CUDA_TRY(snn::launch_label(c, n_images, h->n_exc, cl, n_classes, out, h->stream));
+  h->launches++;
+  if (!out_dev) CUDA_TRY(cudaMemcpyAsync(labels, out, (size_t)h->n_exc * 4, cudaMemcpyDeviceToHost, h->stream));
+  return finish(h, 0);
+}
+
+int snn_classify(snn_handle* h, const uint32_t* counts, int n_images, const int32_t* labels, int n_classes,
+                 int32_t* pred) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  if (!counts || !labels || !pred || n_images < 0) return fail(SNN_EINVAL, "bad classification arguments");
+  if (n_classes < 1 || n_classes > snn::kMaxClasses) return fail(SNN_EINVAL, "n_classes outside [1, %d]", snn::kMaxClasses);
+  DevGuard g(h->dev);
+  std::vector<int32_t> hl((size_t)h->n_exc);
+  if (is_device_ptr(labels)) {
+    CUDA_TRY(cudaMemcpyAsync(hl.data(), labels, hl.size() * 4, cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+  } else {
+    std::memcpy(hl.data(), labels, hl.size() * 4);
+  }
+  for (int j = 0; j < h->n_exc; ++j)
+    if (hl[j] < -1 || hl[j] >= n_classes) return fail(SNN_EINVAL, "labels[%d]=%d outside [-1, %d)", j, hl[j], n_classes);
+  if (n_images == 0) return SNN_OK;
+  const uint32_t* c = nullptr;
+  if ((rc = stage(h, counts, (size_t)n_images * h->n_exc, &h->d_icounts, &h->icounts_cap, &c))) return rc;
+  const int32_t* lb = nullptr;
+  if ((rc = stage(h, labels, (size_t)h->n_exc, &h->d_lab, &h->lab_cap, &lb))) return rc;
+  const bool out_dev = is_device_ptr(pred);
+  int32_t* out = pred;
+  if (!out_dev) {
+    if ((rc = ensure(h, &h->d_cls, &h->cls_cap, (size_t)n_images))) return rc;
+    out = h->d_cls;
+  }
+  CUDA_TRY(snn::launch_classify(c, n_images, h->n_exc, lb, n_classes, out, h->stream));
+  h->launches++;
+  if (!out_dev) CUDA_TRY(cudaMemcpyAsync(pred, out, (size_t)n_images * 4, cudaMemcpyDeviceToHost, h->stream));
+  return finish(h, 0);
 }
 
 }  // extern "C"

@@ -124,4 +124,32 @@ cudaError_t launch_unpack_weights(const NetDesc& d, uint8_t* codes, cudaStream_t
 cudaError_t launch_check_codes(const uint8_t* codes, size_t n, int q_max, int* bad, cudaStream_t s);
 size_t present_smem_bytes(int n_in, int wpr, int L_pot, int L_dep, int q_max, int nthr);
 
+// ---- NEXT-1: batch-parallel inference with frozen weights (snn_infer.cu)
+constexpr int kMaxClasses = 64;
+constexpr int kInferMaxCols = 7 * 32 * 32;   // 224 column threads x 32 columns
+struct InferDesc {
+  int n_in, n_exc, bits, T, n_images, nwi;
+  int nthr_cols;      // column threads: ceil(n_exc / 32)
+  int wpr;            // u32 words per weight row of the inference layout (multiple of 4)
+  int R, rmax;        // ring slots (power of two) and the largest step served from the ring (R / 2)
+  int row_bytes;      // wpr * 4
+  float af, bf, cf, dtf, kI, ief, vthf, vresetf, vinitf;
+  long long A, B, C, E;
+  int Vth, Vreset, Vinit;
+  int t_ref, t_inh, wta_mode, inh_mode;
+  const uint32_t* w;                 // [n_in][wpr] codes, column j at word j / (32/bits), bits (j % (32/bits)) * bits
+  const uint32_t* words;             // [n_images][T][nwi] encoded input spikes
+  uint32_t* counts;                  // [n_images][n_exc] spike counts (zeroed by the caller)
+  unsigned long long* stats;         // [2] += sum_t act(t), post spikes (may be null)
+};
+size_t infer_smem_bytes(int R, int row_bytes);
+cudaError_t infer_occupancy(int bits, int fixed, int nthr, size_t smem, int* out);
+cudaError_t launch_infer(const InferDesc& d, int grid, int nthr, size_t smem, int fixed, cudaStream_t s);
+cudaError_t launch_pack_infer(const uint8_t* codes, int n_in, int n_exc, int bits, int wpr, uint32_t* w,
+                              cudaStream_t s);
+cudaError_t launch_label(const uint32_t* counts, int n_images, int n_exc, const int32_t* classes, int n_classes,
+                         int32_t* labels, cudaStream_t s);
+cudaError_t launch_classify(const uint32_t* counts, int n_images, int n_exc, const int32_t* labels, int n_classes,
+                            int32_t* pred, cudaStream_t s);
+
 }  // namespace snn

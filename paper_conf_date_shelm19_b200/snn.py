@@ -24,6 +24,7 @@ EXPORTS = [
     "snn_state_bytes", "snn_get_state", "snn_set_state", "snn_get_stats", "snn_reset_stats",
     "snn_get_info", "snn_set_trace", "snn_get_trace", "snn_last_error",
     "snn_create_shard", "snn_shard_ipc_handle", "snn_shard_connect", "snn_shard_link",
+    "snn_infer", "snn_get_infer_stats", "snn_label", "snn_classify",
 ]
 SNN_IPC_HANDLE_BYTES = 64
 NINFO = 18
@@ -94,6 +95,10 @@ def lib():
             "snn_shard_ipc_handle": ([vp, vp, sz], i32),
             "snn_shard_connect": ([vp, vp, sz], i32),
             "snn_shard_link": ([vp, i32], i32),
+            "snn_infer": ([vp, vp, i32, i32, vp, vp, i32], i32),
+            "snn_get_infer_stats": ([vp, vp], i32),
+            "snn_label": ([vp, vp, i32, vp, i32, vp], i32),
+            "snn_classify": ([vp, vp, i32, vp, i32, vp], i32),
         }
         for name, (args, res) in sig.items():
             f = getattr(L, name)
@@ -272,6 +277,35 @@ class Network:
 
     def reset_stats(self):
         _check(lib().snn_reset_stats(self._h), "snn_reset_stats")
+
+    # ---- NEXT-1: inference with frozen weights, labelling, vote (include/snn.h)
+    def infer(self, images, T: int, seeds, counts=None, flags: int = 0):
+        """Spike counts (n_images, n_exc) u32 of each image presented with frozen weights.  images/seeds/
+        counts: numpy (host) or torch CUDA tensors; counts is allocated on the host if not given."""
+        n = int(images.shape[0])
+        if counts is None:
+            counts = np.zeros((n, self.n_exc), dtype=np.uint32)
+        _check(lib().snn_infer(self._h, _ptr(images), n, T, _ptr(seeds), _ptr(counts), flags), "snn_infer")
+        return counts
+
+    def infer_stats(self) -> np.ndarray:
+        out = np.zeros(2, dtype=np.uint64)
+        _check(lib().snn_get_infer_stats(self._h, _ptr(out)), "snn_get_infer_stats")
+        return out
+
+    def label(self, counts, classes, n_classes: int, labels=None):
+        n = int(counts.shape[0])
+        if labels is None:
+            labels = np.zeros(self.n_exc, dtype=np.int32)
+        _check(lib().snn_label(self._h, _ptr(counts), n, _ptr(classes), n_classes, _ptr(labels)), "snn_label")
+        return labels
+
+    def classify(self, counts, labels, n_classes: int, pred=None):
+        n = int(counts.shape[0])
+        if pred is None:
+            pred = np.zeros(n, dtype=np.int32)
+        _check(lib().snn_classify(self._h, _ptr(counts), n, _ptr(labels), n_classes, _ptr(pred)), "snn_classify")
+        return pred
 
     # ---- column sharding (include/snn.h, DESIGN.md §10)
     def ipc_handle(self) -> bytes:
