@@ -1093,13 +1093,17 @@ int snn_get_info(const snn_handle* h, int64_t info[SNN_NINFO]) {
 namespace {
 
 // Ring geometry of the inference kernel for this handle: the largest power-of-two ring (<= 64 rows)
-// that leaves room for two CTAs per SM, else one CTA per SM, at least 8 rows.
+// (>= 32 rows) that leaves room for three CTAs per SM, else two, else one (>= 8 rows).  r01 sweep on
+// 784->6400 2-bit: R=32 / 3 CTAs 370k images/s, R=64 / 2 CTAs 333k, R=32 / 2 CTAs 329k, R=16 / 3 CTAs 125k.
 int infer_geometry(const snn_handle* h, int* wpr, int* R, int* nthr, size_t* smem) {
   const int ncols = (h->n_exc + 31) / 32;
   *wpr = ((ncols * h->bits) + 3) & ~3;
   const int row_bytes = *wpr * 4;
   *nthr = (((ncols + 31) / 32) + 1) * 32;
   int r = 64;
+  if (const char* e = std::getenv("SNN_INFER_RING"))   // experiment hook: ring rows (power of two, 8..64)
+    if (std::atoi(e) >= 8 && std::atoi(e) <= 64 && !(std::atoi(e) & (std::atoi(e) - 1))) r = std::atoi(e);
+  while (r > 32 && snn::infer_smem_bytes(r, row_bytes) > 74 * 1024) r >>= 1;   // three CTAs per SM (measured best)
   while (r > 8 && snn::infer_smem_bytes(r, row_bytes) > 110 * 1024) r >>= 1;
   while (r > 8 && snn::infer_smem_bytes(r, row_bytes) > 220 * 1024) r >>= 1;
   if (snn::infer_smem_bytes(r, row_bytes) > 220 * 1024) return fail(SNN_ESIZE, "inference ring does not fit");
@@ -1157,8 +1161,11 @@ int snn_infer(snn_handle* h, const uint8_t* images, int n_images, int T, const u
     if ((rc = ensure(h, &h->d_icounts, &h->icounts_cap, (size_t)n_images * h->n_exc))) return rc;
     cnt = h->d_icounts;
   }
+  int minb = smem <= 74 * 1024 ? 3 : 2;           // register budget (<= 80 / <= 128) matching the smem occupancy
+  if (const char* e = std::getenv("SNN_INFER_MINB"))   // experiment hook
+    if (std::atoi(e) == 2 || std::atoi(e) == 3) minb = std::atoi(e);
   int occ = 0;
-  CUDA_TRY(snn::infer_occupancy(h->bits, h->p.membrane_mode, nthr, smem, &occ));
+  CUDA_TRY(snn::infer_occupancy(h->bits, h->p.membrane_mode, minb, nthr, smem, &occ));
   if (occ < 1) return fail(SNN_ESIZE, "inference kernel cannot be resident (smem %zu B, %d threads)", smem, nthr);
   int nsm = 0;
   CUDA_TRY(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, h->dev));
@@ -1189,7 +1196,7 @@ int snn_infer(snn_handle* h, const uint8_t* images, int n_images, int T, const u
     int grid = std::min(nb, occ * nsm);
     if (const char* e = std::getenv("SNN_INFER_MAX_GRID"))   // test hook: force the persistent image loop
       if (std::atoi(e) > 0) grid = std::min(grid, std::atoi(e));
-    CUDA_TRY(snn::launch_infer(d, grid, nthr, smem, h->p.membrane_mode, h->stream));
+    CUDA_TRY(snn::launch_infer(d, grid, nthr, smem, h->p.membrane_mode, minb, h->stream));
     h->launches += 2;
   }
   if (!counts_dev)

@@ -25,6 +25,7 @@ namespace snn {
 
 constexpr int kSR = 64;                  // step ring of the producer's per-step (base, count) records
 constexpr uint32_t kDirect = 0x80000000u;
+constexpr int kWB = 8;                   // steps per producer word-prefetch batch (cp.async, double-buffered)
 constexpr int kInfMaxThreads = 256;      // <= 224 column threads (n_exc <= 7168) + the producer warp: 255 registers
 
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
@@ -73,8 +74,8 @@ struct Swar {
   }
 };
 
-template <int BITS, bool FIXED>
-__global__ void __launch_bounds__(kInfMaxThreads, 2) infer_kernel(const InferDesc d) {
+template <int BITS, bool FIXED, int MINB>
+__global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const InferDesc d) {
   using SW = Swar<BITS>;
   extern __shared__ __align__(128) unsigned char smem[];
   unsigned char* ring = smem;                                                   // [R][row_bytes]
@@ -83,6 +84,7 @@ __global__ void __launch_bounds__(kInfMaxThreads, 2) infer_kernel(const InferDes
   uint32_t* s_base = s_nrows + kSR;                                             // [kSR] first ring position
   unsigned long long* s_key = reinterpret_cast<unsigned long long*>(s_base + kSR);  // [32]
   int* s_cnt = reinterpret_cast<int*>(s_key + 32);                              // [32]
+  uint32_t* s_wbuf = reinterpret_cast<uint32_t*>(s_cnt + 32);                   // [2][kWB][32] producer's word prefetch
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int ncw = (d.nthr_cols + 31) >> 5;        // consumer warps
@@ -107,6 +109,27 @@ __global__ void __launch_bounds__(kInfMaxThreads, 2) infer_kernel(const InferDes
   // Issue steps [p_step, min(G, limit)) while their rows fit the ring; ring positions before the first
   // row of step `first_live` are released (their readers passed a barrier).  Steps with more than rmax
   // rows are marked direct (read from global memory by the consumers, no ring slots).
+  // Encoded input words of upcoming steps (n_in <= 1024: one word per lane) are prefetched by the producer
+  // warp with cp.async in batches of kWB steps, two batches in flight, so that issuing a step never waits
+  // on a global-memory round trip.
+  const bool wfast = d.nwi <= 32;
+  long long pf_step = 0;      // next step to prefetch
+  long long wb_entered = -1;  // last batch whose words the producer started to read
+  int pf_img = 0, pf_t = 0;
+  auto prefetch_batch = [&]() {
+    uint32_t* dst = s_wbuf + ((pf_step / kWB) & 1) * (kWB * 32);
+#pragma unroll 1
+    for (int q = 0; q < kWB; ++q) {
+      if (pf_step < G && lane < d.nwi) {
+        const long long k = (long long)blockIdx.x + (long long)pf_img * gridDim.x;
+        const uint32_t* src = d.words + ((size_t)k * T + pf_t) * d.nwi + lane;
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst + q * 32 + lane)), "l"(src) : "memory");
+      }
+      ++pf_step;
+      if (++pf_t == T) { pf_t = 0; ++pf_img; }
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
   auto produce = [&](long long limit, long long first_live) {
     long long released = p_pos;
     if (first_live < p_step) released = p_pos - (long long)(uint32_t)((uint32_t)p_pos - s_base[first_live & (kSR - 1)]);
@@ -116,8 +139,19 @@ __global__ void __launch_bounds__(kInfMaxThreads, 2) infer_kernel(const InferDes
       const int s = (int)(p_step & (kSR - 1));
       const long long k = (long long)blockIdx.x + (long long)p_img * gridDim.x;
       const uint32_t* wr = d.words + ((size_t)k * T + p_t) * d.nwi;
+      uint32_t w_l = 0;                                // this lane's word of the step (fast path)
       int n = 0;
-      for (int w = lane; w < d.nwi; w += 32) n += __popc(__ldg(&wr[w]));
+      if (wfast) {
+        if (p_step / kWB > wb_entered) {   // entering batch b: refill the buffer of batch b-1 with batch b+1,
+          wb_entered = p_step / kWB;       // then wait for batch b (each lane reads only its own words)
+          if (p_step > 0) prefetch_batch();
+          asm volatile("cp.async.wait_group 1;" ::: "memory");
+        }
+        w_l = lane < d.nwi ? s_wbuf[((p_step / kWB) & 1) * (kWB * 32) + (p_step % kWB) * 32 + lane] : 0u;
+        n = __popc(w_l);
+      } else {
+        for (int w = lane; w < d.nwi; w += 32) n += __popc(__ldg(&wr[w]));
+      }
 #pragma unroll
       for (int o = 16; o; o >>= 1) n += __shfl_xor_sync(FULL, n, o);
       if (n <= d.rmax && (long long)d.R - (p_pos - released) < n) break;   // ring full: after the next barrier
@@ -127,7 +161,7 @@ __global__ void __launch_bounds__(kInfMaxThreads, 2) infer_kernel(const InferDes
         long long pos = p_pos;
         for (int w0 = 0; w0 < d.nwi; w0 += 32) {
           const int w = w0 + lane;
-          uint32_t bits = w < d.nwi ? __ldg(&wr[w]) : 0u;
+          uint32_t bits = wfast ? w_l : (w < d.nwi ? __ldg(&wr[w]) : 0u);
           const int c = __popc(bits);
           int incl = c;
 #pragma unroll
@@ -160,7 +194,8 @@ __global__ void __launch_bounds__(kInfMaxThreads, 2) infer_kernel(const InferDes
   const int j0 = 32 * tcol;
   int v[32];
   uint32_t fr[16];                               // free-from step, u16 x 2 (column c at half c & 1 of fr[c >> 1])
-  int my_min_free = 0;
+  int my_min_free = 0;                           // min / max over this thread's columns (padding: 0xFFFF)
+  int my_max_free = 0;
   const int vinit = FIXED ? d.Vinit : __float_as_int(d.vinitf);
   const int vreset = FIXED ? d.Vreset : __float_as_int(d.vresetf);
   Lif lif;
@@ -169,7 +204,10 @@ __global__ void __launch_bounds__(kInfMaxThreads, 2) infer_kernel(const InferDes
   const bool consumer = !is_producer && tcol < d.nthr_cols;
   unsigned long long act_sum = 0, spikes = 0;
 
-  if (is_producer) produce(2, 0);                // steps 0 and 1 before the first barrier
+  if (is_producer) {
+    if (wfast) { prefetch_batch(); prefetch_batch(); }
+    produce(2, 0);                               // steps 0 and 1 before the first barrier
+  }
   __syncthreads();
 
   uint32_t* counts_img = nullptr;
@@ -192,6 +230,7 @@ __global__ void __launch_bounds__(kInfMaxThreads, 2) infer_kernel(const InferDes
           const uint32_t hi = (j0 + 2 * h + 1 < d.n_exc) ? 0u : 0xFFFFu;
           fr[h] = lo | (hi << 16);
         }
+        my_max_free = j0 + 32 > d.n_exc ? 0xFFFF : 0;
         if (j0 + 32 > d.n_exc) my_min_free = j0 >= d.n_exc ? 0xFFFF : 0;
       }
     }
@@ -219,15 +258,28 @@ __global__ void __launch_bounds__(kInfMaxThreads, 2) infer_kernel(const InferDes
           }
           SW::add(acc, w);
         }
+        // LIF (eqs.(1)(2)) of the non-held columns; keys only if some column crossed
+        bool cross = false;
+        if ((int)tt >= my_max_free) {                             // no column of this thread is held
 #pragma unroll
-        for (int c = 0; c < 32; ++c) {
-          const uint32_t f = (fr[c >> 1] >> ((c & 1) * 16)) & 0xFFFFu;
-          if (tt < f) continue;                                   // refractory / inhibited: hold v (R6, R7)
-          const bool x = lif.step_t<FIXED>(v[c], SW::get(acc, c));   // eqs.(1)(3), DESIGN.md §3.3
-          if (x) {
-            const unsigned long long key = ((unsigned long long)lif.ord(v[c]) << 32) | (0xFFFFFFFFu - (uint32_t)(j0 + c));
-            best = key > best ? key : best;
-            ++ncand;
+          for (int c = 0; c < 32; ++c) cross |= lif.step_t<FIXED>(v[c], SW::get(acc, c));
+        } else {
+#pragma unroll
+          for (int c = 0; c < 32; ++c) {
+            const uint32_t f = (fr[c >> 1] >> ((c & 1) * 16)) & 0xFFFFu;
+            if (tt >= f) cross |= lif.step_t<FIXED>(v[c], SW::get(acc, c));   // held: keep v (R6, R7)
+          }
+        }
+        if (cross) {
+#pragma unroll
+          for (int c = 0; c < 32; ++c) {
+            const uint32_t f = (fr[c >> 1] >> ((c & 1) * 16)) & 0xFFFFu;
+            const bool above = FIXED ? (v[c] > d.Vth) : (__int_as_float(v[c]) > d.vthf);
+            if (tt >= f && above) {
+              const unsigned long long key = ((unsigned long long)lif.ord(v[c]) << 32) | (0xFFFFFFFFu - (uint32_t)(j0 + c));
+              best = key > best ? key : best;
+              ++ncand;
+            }
           }
         }
       } else {
@@ -286,7 +338,7 @@ __global__ void __launch_bounds__(kInfMaxThreads, 2) infer_kernel(const InferDes
       if (consumer) {
         const uint32_t f_ref = min(tt + 1u + (uint32_t)d.t_ref, 0xFFFFu);
         const uint32_t f_inh = min(tt + 1u + (uint32_t)d.t_inh, 0xFFFFu);
-        int mn = 0xFFFF;
+        int mn = 0xFFFF, mx = 0;
 #pragma unroll
         for (int c = 0; c < 32; ++c) {
           const int j = j0 + c;
@@ -313,8 +365,10 @@ __global__ void __launch_bounds__(kInfMaxThreads, 2) infer_kernel(const InferDes
             fr[c >> 1] = (fr[c >> 1] & ~(0xFFFFu << sh)) | (f << sh);
           }
           mn = min(mn, (int)f);
+          mx = max(mx, (int)f);
         }
         my_min_free = mn;
+        my_max_free = mx;
       }
     }
   }
@@ -407,47 +461,60 @@ __global__ void __launch_bounds__(kVoteWarps * 32) classify_kernel(
 
 // ---------------------------------------------------------------- host side
 size_t infer_smem_bytes(int R, int row_bytes) {
-  return (size_t)R * row_bytes + (size_t)R * 8 + 2 * kSR * 4 + 32 * 8 + 32 * 4;
+  return (size_t)R * row_bytes + (size_t)R * 8 + 2 * kSR * 4 + 32 * 8 + 32 * 4 + 2 * kWB * 32 * 4;
 }
 
-template <int BITS, bool FIXED>
+template <int BITS, bool FIXED, int MINB>
 static cudaError_t launch_infer_t(const InferDesc& d, int grid, int nthr, size_t smem, cudaStream_t s) {
-  auto k = infer_kernel<BITS, FIXED>;
+  auto k = infer_kernel<BITS, FIXED, MINB>;
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   k<<<grid, nthr, smem, s>>>(d);
   return cudaGetLastError();
 }
 
-template <int BITS, bool FIXED>
+template <int BITS, bool FIXED, int MINB>
 static cudaError_t occ_t(int nthr, size_t smem, int* out) {
-  auto k = infer_kernel<BITS, FIXED>;
+  auto k = infer_kernel<BITS, FIXED, MINB>;
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   return cudaOccupancyMaxActiveBlocksPerMultiprocessor(out, k, nthr, smem);
 }
 
-cudaError_t infer_occupancy(int bits, int fixed, int nthr, size_t smem, int* out) {
-  switch (bits * 2 + fixed) {
-    case 4: return occ_t<2, false>(nthr, smem, out);
-    case 5: return occ_t<2, true>(nthr, smem, out);
-    case 8: return occ_t<4, false>(nthr, smem, out);
-    case 9: return occ_t<4, true>(nthr, smem, out);
-    case 16: return occ_t<8, false>(nthr, smem, out);
-    case 17: return occ_t<8, true>(nthr, smem, out);
+// minb: register budget variant (2 -> <= 128 registers, 3 -> <= 80 registers per thread)
+cudaError_t infer_occupancy(int bits, int fixed, int minb, int nthr, size_t smem, int* out) {
+  switch ((bits * 2 + fixed) * 4 + minb) {
+    case 18: return occ_t<2, false, 2>(nthr, smem, out);
+    case 19: return occ_t<2, false, 3>(nthr, smem, out);
+    case 22: return occ_t<2, true, 2>(nthr, smem, out);
+    case 23: return occ_t<2, true, 3>(nthr, smem, out);
+    case 34: return occ_t<4, false, 2>(nthr, smem, out);
+    case 35: return occ_t<4, false, 3>(nthr, smem, out);
+    case 38: return occ_t<4, true, 2>(nthr, smem, out);
+    case 39: return occ_t<4, true, 3>(nthr, smem, out);
+    case 66: return occ_t<8, false, 2>(nthr, smem, out);
+    case 67: return occ_t<8, false, 3>(nthr, smem, out);
+    case 70: return occ_t<8, true, 2>(nthr, smem, out);
+    case 71: return occ_t<8, true, 3>(nthr, smem, out);
   }
   return cudaErrorInvalidValue;
 }
 
-cudaError_t launch_infer(const InferDesc& d, int grid, int nthr, size_t smem, int fixed, cudaStream_t s) {
+cudaError_t launch_infer(const InferDesc& d, int grid, int nthr, size_t smem, int fixed, int minb, cudaStream_t s) {
   if (d.n_images <= 0 || d.T <= 0) return cudaSuccess;
-  switch (d.bits * 2 + fixed) {
-    case 4: return launch_infer_t<2, false>(d, grid, nthr, smem, s);
-    case 5: return launch_infer_t<2, true>(d, grid, nthr, smem, s);
-    case 8: return launch_infer_t<4, false>(d, grid, nthr, smem, s);
-    case 9: return launch_infer_t<4, true>(d, grid, nthr, smem, s);
-    case 16: return launch_infer_t<8, false>(d, grid, nthr, smem, s);
-    case 17: return launch_infer_t<8, true>(d, grid, nthr, smem, s);
+  switch ((d.bits * 2 + fixed) * 4 + minb) {
+    case 18: return launch_infer_t<2, false, 2>(d, grid, nthr, smem, s);
+    case 19: return launch_infer_t<2, false, 3>(d, grid, nthr, smem, s);
+    case 22: return launch_infer_t<2, true, 2>(d, grid, nthr, smem, s);
+    case 23: return launch_infer_t<2, true, 3>(d, grid, nthr, smem, s);
+    case 34: return launch_infer_t<4, false, 2>(d, grid, nthr, smem, s);
+    case 35: return launch_infer_t<4, false, 3>(d, grid, nthr, smem, s);
+    case 38: return launch_infer_t<4, true, 2>(d, grid, nthr, smem, s);
+    case 39: return launch_infer_t<4, true, 3>(d, grid, nthr, smem, s);
+    case 66: return launch_infer_t<8, false, 2>(d, grid, nthr, smem, s);
+    case 67: return launch_infer_t<8, false, 3>(d, grid, nthr, smem, s);
+    case 70: return launch_infer_t<8, true, 2>(d, grid, nthr, smem, s);
+    case 71: return launch_infer_t<8, true, 3>(d, grid, nthr, smem, s);
   }
   return cudaErrorInvalidValue;
 }

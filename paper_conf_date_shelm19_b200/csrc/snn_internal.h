@@ -143,8 +143,8 @@ struct InferDesc {
   unsigned long long* stats;         // [2] += sum_t act(t), post spikes (may be null)
 };
 size_t infer_smem_bytes(int R, int row_bytes);
-cudaError_t infer_occupancy(int bits, int fixed, int nthr, size_t smem, int* out);
-cudaError_t launch_infer(const InferDesc& d, int grid, int nthr, size_t smem, int fixed, cudaStream_t s);
+cudaError_t infer_occupancy(int bits, int fixed, int minb, int nthr, size_t smem, int* out);
+cudaError_t launch_infer(const InferDesc& d, int grid, int nthr, size_t smem, int fixed, int minb, cudaStream_t s);
 cudaError_t launch_pack_infer(const uint8_t* codes, int n_in, int n_exc, int bits, int wpr, uint32_t* w,
                               cudaStream_t s);
 cudaError_t launch_label(const uint32_t* counts, int n_images, int n_exc, const int32_t* classes, int n_classes,
