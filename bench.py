@@ -157,6 +157,8 @@ def main():
     ap.add_argument("--engine", type=int, default=0, help="0 event-driven epochs, 1 per-step exchange")
     ap.add_argument("--mode", default="replicas", choices=["replicas", "shard"], help="N > 1 layout")
     ap.add_argument("--local-shards", type=int, default=1, help="shards of the network on this GPU (N = 1)")
+    ap.add_argument("--no-infer", action="store_true", help="skip the NEXT-1 inference measurement")
+    ap.add_argument("--infer-images", type=int, default=4096, help="images per inference call")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -356,6 +358,42 @@ def main():
                 "alg_bytes_per_launch": per_launch_bytes,
                 "note": "latency-bound step loop; see latency_roofline"}
 
+    # ---- NEXT-1: inference with the learned weights frozen, images independent.  Device-timed
+    # (CUDA events on the launching stream), images resident in HBM.  Dominant kernel: infer_kernel, bound by
+    # FP32/INT issue: per column-step the LIF recipe is 7 lane-ops (I2F, FMUL, FADD, 3 FFMA, FSETP), per
+    # synaptic event 1 integer add; peak = 148 SMs x 128 lanes x SM clock.
+    inference = None
+    if ws == 1 and K == 1 and not args.no_infer:
+        nb = args.infer_images
+        iimgs = torch.from_numpy(synthdata.images(nb, "fashion", start=200000)).to(dev)
+        iseeds = torch.from_numpy(synthdata.seeds(nb, base_seed=99).view(np.int64)).to(dev)
+        icounts = torch.zeros((nb, N_EXC), dtype=torch.int32, device=dev)
+        net.infer(iimgs, T_STEPS, iseeds, icounts, flags=P.SNN_ASYNC)
+        torch.cuda.synchronize()
+        st0 = net.infer_stats().copy()
+        iev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(3)]
+        for e0, e1 in iev:
+            flush.fill_(7)
+            e0.record(stream)
+            net.infer(iimgs, T_STEPS, iseeds, icounts, flags=P.SNN_ASYNC)
+            e1.record(stream)
+        torch.cuda.synchronize()
+        ims = [a.elapsed_time(b) for a, b in iev]
+        ist = net.infer_stats() - st0
+        its = sum(ims) / 1e3
+        n_inf = 3 * nb
+        lane_ops = 7.0 * N_EXC * T_STEPS * n_inf + float(ist[0]) * N_EXC
+        smclk_i = (clocks.get("sm_max_mhz") or 1965.0)
+        peak_ops = N_SM * 128 * smclk_i * 1e6 / 1e12
+        inference = {"metric": "inference images/s (learned weights frozen, P:88 labelling/inference protocol)",
+                     "value": n_inf / its, "unit": "images/s", "images_per_call": nb, "ms_per_call": sum(ims) / 3,
+                     "synaptic_events_per_s": float(ist[0]) * N_EXC / its,
+                     "post_spikes_per_image": float(ist[1]) / n_inf,
+                     "roofline": {"bound": "alu", "achieved": lane_ops / its / 1e12, "peak": peak_ops,
+                                  "unit": "Tlane-op/s", "frac": lane_ops / its / 1e12 / peak_ops,
+                                  "work": "7 lane-ops per column-step (LIF recipe) + 1 per synaptic event",
+                                  "peak_source": f"derived: 148 SMs x 128 FP32/INT lanes x {smclk_i:.0f} MHz"}}
+
     line = {
         "metric": METRIC, "value": value, "unit": "images/s", "n_gpus": ws, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": 1e3 * dev_s / args.steps, "higher_is_better": True,
@@ -383,6 +421,7 @@ def main():
         "e2e": e2e,
         "roofline": roofline,
         "latency_roofline": floor,
+        "inference": inference,
     }
     if rank == 0 and ws == 1 and args.cpu_images > 0:
         line["cpu_baseline"] = cpu_baseline(args.cpu_images)
