@@ -121,6 +121,9 @@ def lib():
                                    ctypes.c_void_p]
         L.oracle_label.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_int,
                                    ctypes.c_void_p]
+        L.oracle_sparse_run.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p,
+                                        ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int, ctypes.c_int, ctypes.c_void_p,
+                                        ctypes.c_void_p, ctypes.c_void_p]
         L.oracle_classify.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_int,
                                       ctypes.c_void_p]
         _lib = L
@@ -251,6 +254,20 @@ class OracleNet:
         self._check(lib().oracle_infer(self._h, _ptr(imgs), imgs.shape[0], T, _ptr(sd), _ptr(out)), "oracle_infer")
         self.last_T = T
         return out
+
+    def sparse_run(self, n_lif: int, src_off, tgt, q, images, T: int, seeds, raster: bool = False):
+        """NEXT-4 (P:92, R24-R26): counts (n_trials, n_lif) u32 [, raster (n_trials, T, ceil(n_lif/32)) u32]."""
+        imgs = np.ascontiguousarray(images, dtype=np.uint8).reshape(-1, self.n_in)
+        so = np.ascontiguousarray(src_off, dtype=np.int32)
+        tg = np.ascontiguousarray(tgt, dtype=np.uint16)
+        qq = np.ascontiguousarray(q, dtype=np.uint8)
+        sd = np.ascontiguousarray(np.asarray(seeds, dtype=np.uint64).reshape(-1))
+        nt = imgs.shape[0]
+        counts = np.zeros((nt, n_lif), dtype=np.uint32)
+        r = np.zeros((nt, T, (n_lif + 31) // 32), dtype=np.uint32) if raster else None
+        self._check(lib().oracle_sparse_run(self._h, self.n_in, n_lif, _ptr(so), _ptr(tg), _ptr(qq), _ptr(imgs), nt, T,
+                                            _ptr(sd), _ptr(counts), _ptr(r) if raster else None), "oracle_sparse_run")
+        return (counts, r) if raster else counts
 
 
 def label(counts: np.ndarray, classes, n_classes: int) -> np.ndarray:

@@ -552,3 +552,62 @@ int oracle_classify(const uint32_t* counts, int n_images, int n_exc, const int32
   free(M); free(s);
   return 0;
 }
+
+/* ---------------------------------------------------------------- NEXT-4: Fig. 4 sparse workload
+ * P:92 §IV-A: "We first evaluate the accuracy of the spiking neuron simulation (no learning) considering an
+ * SNN of 10^3 LIF neurons and 10^4 synapses."  Topology, drive and delays are unstated: R24-R26. */
+int oracle_sparse_run(const oracle_net* n, int n_in, int n_lif, const int32_t* src_off, const uint16_t* tgt,
+                      const uint8_t* q, const uint8_t* images, int n_trials, int T, const uint64_t* seeds,
+                      uint32_t* counts, uint32_t* raster) {
+  if (!n || n_in < 1 || n_lif < 1 || n_lif > 65536 || !src_off || n_trials < 0 || T < 0) return E_INVAL;
+  if (n_trials > 0 && (!images || !seeds || !counts)) return E_INVAL;
+  const int n_src = n_in + n_lif;
+  if (src_off[0] != 0) return E_INVAL;
+  for (int s = 0; s < n_src; ++s) if (src_off[s + 1] < src_off[s]) return E_INVAL;
+  const int n_syn = src_off[n_src];
+  for (int k = 0; k < n_syn; ++k) if (tgt[k] >= n_lif || q[k] > n->q_max) return E_INVAL;
+  const oracle_params* p = &n->p;
+  const int fixed = p->membrane_mode == 1;
+  const int wl = (n_lif + 31) / 32;
+  float* vf = (float*)malloc(sizeof(float) * (size_t)n_lif);
+  int32_t* vx = (int32_t*)malloc(sizeof(int32_t) * (size_t)n_lif);
+  int32_t* cnt = (int32_t*)malloc(sizeof(int32_t) * (size_t)n_lif);
+  int32_t* S = (int32_t*)malloc(sizeof(int32_t) * (size_t)n_lif);
+  uint8_t* act = (uint8_t*)malloc((size_t)n_src);          /* source active at this step */
+  uint8_t* spk = (uint8_t*)malloc((size_t)n_lif);          /* neuron spiked at this step */
+  if (!vf || !vx || !cnt || !S || !act || !spk) { free(vf); free(vx); free(cnt); free(S); free(act); free(spk); return E_NOMEM; }
+  for (int tr = 0; tr < n_trials; ++tr) {
+    const uint8_t* img = images + (size_t)tr * n_in;
+    for (int j = 0; j < n_lif; ++j) { vf[j] = n->vinitf; vx[j] = n->Vinit; cnt[j] = 0; spk[j] = 0; }   /* [R5] */
+    for (int j = 0; j < n_lif; ++j) counts[(size_t)tr * n_lif + j] = 0;
+    for (int t = 0; t < T; ++t) {
+      /* sources: input pixels (encoder, R8, R13) at t; neurons that spiked at t-1 (one-step delay, R25) */
+      for (int i = 0; i < n_in; ++i) {
+        uint32_t u = draw(seeds[tr], (uint32_t)t, (uint32_t)(i >> 2), 0u, TAG_ENC, i & 3);
+        act[i] = (uint8_t)((uint64_t)u < n->thr_enc[img[i]]);
+      }
+      for (int j = 0; j < n_lif; ++j) act[n_in + j] = spk[j];
+      /* eq.(3) over the synapses of active sources */
+      for (int j = 0; j < n_lif; ++j) S[j] = 0;
+      for (int s = 0; s < n_src; ++s)
+        if (act[s])
+          for (int k = src_off[s]; k < src_off[s + 1]; ++k) S[tgt[k]] += q[k];
+      /* eqs.(1)(2) + refractory [R6]; no inhibition, no WTA [R26] */
+      for (int j = 0; j < n_lif; ++j) {
+        spk[j] = 0;
+        if (cnt[j] > 0) { cnt[j]--; continue; }
+        int cross;
+        if (fixed) { vx[j] = oracle_lif_step_fixed(n, vx[j], S[j]); cross = vx[j] > n->Vth; }
+        else       { vf[j] = oracle_lif_step_fp32(n, vf[j], S[j]);  cross = vf[j] > n->vthf; }
+        if (cross) {
+          spk[j] = 1;
+          vf[j] = n->vresetf; vx[j] = n->Vreset; cnt[j] = p->t_ref_steps;
+          counts[(size_t)tr * n_lif + j]++;
+          if (raster) raster[((size_t)tr * T + t) * wl + j / 32] |= 1u << (j % 32);
+        }
+      }
+    }
+  }
+  free(vf); free(vx); free(cnt); free(S); free(act); free(spk);
+  return 0;
+}

@@ -87,6 +87,20 @@ int oracle_label(const uint32_t* counts, int n_images, int n_exc, const int32_t*
 int oracle_classify(const uint32_t* counts, int n_images, int n_exc, const int32_t* labels, int n_classes,
                     int32_t* pred);
 
+/* ---- NEXT-4: the Fig. 4 workload (§IV-A "an SNN of 10^3 LIF neurons and 10^4 synapses", no
+ * learning; readings DESIGN.md R24-R26).  Sources 0..n_in-1 are the rate-coded input pixels (encoder as
+ * in oracle_present, R8/R13), sources n_in..n_in+n_lif-1 are the LIF neurons themselves (recurrent, one
+ * step of synaptic delay).  Synapse k of source s (k in [src_off[s], src_off[s+1])) targets LIF neuron
+ * tgt[k] with code q[k] (G = q * 2^-bits, R9).  Per step t: S_j = sum of q[k] over synapses whose source
+ * is active (input spike at t, or neuron spike at t-1); LIF recipe (membrane_mode) with refractory
+ * t_ref; v > v_th -> spike, v = v_reset.  No WTA, no inhibition, no STDP.  State reset per trial (R5).
+ * counts[k*n_lif + j] = spikes of neuron j in trial k; raster (optional, n_trials x T x ceil(n_lif/32)).
+ * Uses the net's parameter block only (a, b, c, v_*, dt, v_spike, i_ext, t_ref, f_min/f_max, membrane
+ * mode, bits). */
+int oracle_sparse_run(const oracle_net* net, int n_in, int n_lif, const int32_t* src_off, const uint16_t* tgt,
+                      const uint8_t* q, const uint8_t* images, int n_trials, int T, const uint64_t* seeds,
+                      uint32_t* counts, uint32_t* raster);
+
 /* Exposed for the pin tests. */
 int oracle_q_max(const oracle_net* net);
 int oracle_lut(const oracle_net* net, int which /*0 enc,1 pot,2 dep,3 det_p_base,4 det_p_thr,5 det_d_base,6 det_d_thr*/,

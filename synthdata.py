@@ -101,3 +101,21 @@ def seeds(n: int, base_seed: int = 1, start: int = 0) -> np.ndarray:
 def stats(imgs: np.ndarray) -> dict:
     x = imgs.astype(np.float64) / 255.0
     return dict(mean=float(x.mean()), nonzero=float((imgs > 0).mean()))
+
+
+def sparse_graph(n_in: int = 784, n_lif: int = 1000, n_syn: int = 10000, bits: int = 8, seed: int = DATA_SEED,
+                 recurrent: bool = True):
+    """Random synapse list for the Fig. 4 workload (10^3 LIF neurons, 10^4 synapses; R24):
+    sources uniform over the n_in input pixels (and, if recurrent, the n_lif neurons), targets uniform over
+    the neurons, codes uniform on the 2^bits grid.  CSR by source: (src_off[n_src + 1] int32, tgt u16, q u8).
+    Topology only -- none of the method's arithmetic."""
+    rng = np.random.default_rng(seed)
+    n_src = n_in + (n_lif if recurrent else 0)
+    src = rng.integers(0, n_src, size=n_syn)
+    tgt = rng.integers(0, n_lif, size=n_syn)
+    q = rng.integers(0, 1 << bits, size=n_syn)
+    order = np.lexsort((tgt, src))
+    src, tgt, q = src[order], tgt[order], q[order]
+    off = np.zeros(n_in + n_lif + 1, dtype=np.int32)
+    np.add.at(off, src + 1, 1)
+    return np.cumsum(off).astype(np.int32), tgt.astype(np.uint16), q.astype(np.uint8)

@@ -11,7 +11,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 def run(env_extra, args):
     env = dict(os.environ, **env_extra)
-    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--cpu-images", "0", "--steps", "8", *args],
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--cpu-images", "0", "--no-infer", "--steps", "8", *args],
                        capture_output=True, text=True, env=env)
     line = [l for l in r.stdout.splitlines() if l.startswith("{")]
     if not line:
