@@ -238,6 +238,24 @@ int snn_label(snn_handle* h, const uint32_t* counts, int n_images, const int32_t
 int snn_classify(snn_handle* h, const uint32_t* counts, int n_images, const int32_t* labels, int n_classes,
                  int32_t* pred);
 
+/* ---- NEXT-4: the Fig. 4 workload (R24-R26).
+ * P:92 §IV-A: "We first evaluate the accuracy of the spiking neuron simulation (no learning) considering
+ * an SNN of 10^3 LIF neurons and 10^4 synapses."
+ * snn_sparse_run simulates n_trials independent trials of a sparse recurrent network of n_lif LIF
+ * neurons with the handle's parameter block (LIF recipe, t_ref, encoder rates, bits -> LSB) and NOT its
+ * weights: sources 0..n_in-1 are the rate-coded pixels of images[k] (the encoder of snn_present, seeds[k]),
+ * sources n_in..n_in+n_lif-1 are the neurons (their spikes arrive one step later, R25).  Synapses CSR by
+ * source: src_off[n_in + n_lif + 1] (int32, src_off[0] = 0, non-decreasing), tgt[n_syn] (u16 < n_lif),
+ * q[n_syn] (u8 codes <= q_max).  Per step S_j = sum of codes of synapses from active sources; LIF with
+ * refractory; no WTA, no inhibition, no STDP (R26).  counts: n_trials x n_lif u32 spikes per neuron;
+ * raster (optional, may be NULL): n_trials x T x ceil(n_lif/32) u32.  Pointers host or device (graph
+ * validated on the host: SNN_EINVAL).  n_lif <= 16384, T <= 2^30.  Synchronous unless SNN_ASYNC.
+ * snn_get_sparse_stats: [0] input spikes, [1] neuron spikes, summed over all sparse runs of the handle. */
+int snn_sparse_run(snn_handle* h, int n_lif, const int32_t* src_off, const uint16_t* tgt, const uint8_t* q,
+                   const uint8_t* images, int n_trials, int T, const uint64_t* seeds, uint32_t* counts,
+                   uint32_t* raster, int flags);
+int snn_get_sparse_stats(snn_handle* h, uint64_t stats[2]);
+
 const char* snn_last_error(void);
 
 #ifdef __cplusplus

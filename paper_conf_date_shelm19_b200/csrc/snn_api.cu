@@ -125,6 +125,13 @@ struct snn_handle {
   int32_t* d_cls = nullptr;       size_t cls_cap = 0;
   int32_t* d_lab = nullptr;       size_t lab_cap = 0;
   unsigned long long* d_istats = nullptr;
+  // NEXT-4 sparse workload
+  int32_t* d_soff = nullptr;      size_t soff_cap = 0;
+  uint16_t* d_stgt = nullptr;     size_t stgt_cap = 0;
+  uint8_t* d_sq = nullptr;        size_t sq_cap = 0;
+  uint32_t* d_scounts = nullptr;  size_t scounts_cap = 0;
+  uint32_t* d_sraster = nullptr;  size_t sraster_cap = 0;
+  unsigned long long* d_sstats = nullptr;
 };
 
 namespace {
@@ -210,7 +217,8 @@ void free_all(snn_handle* h) {
                   h->d_img, h->d_rin, h->d_seeds, h->d_counts, h->d_codes, h->d_bad,
                   h->d_words, h->d_ecnt, h->d_offs, h->d_rows, h->d_rows16, h->d_trace,
                   h->d_mbox, h->d_peers, h->d_winf, h->d_iwords, h->d_icounts, h->d_iecnt, h->d_cls,
-                  h->d_lab, h->d_istats};
+                  h->d_lab, h->d_istats, h->d_soff, h->d_stgt, h->d_sq, h->d_scounts, h->d_sraster,
+                  h->d_sstats};
   for (void* q : ptrs) if (q) cudaFree(q);
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
 }
@@ -1283,6 +1291,108 @@ int snn_classify(snn_handle* h, const uint32_t* counts, int n_images, const int3
   h->launches++;
   if (!out_dev) CUDA_TRY(cudaMemcpyAsync(pred, out, (size_t)n_images * 4, cudaMemcpyDeviceToHost, h->stream));
   return finish(h, 0);
+}
+
+}  // extern "C"
+
+// ---------------------------------------------------------------- NEXT-4: Fig. 4 sparse workload
+extern "C" {
+
+int snn_sparse_run(snn_handle* h, int n_lif, const int32_t* src_off, const uint16_t* tgt, const uint8_t* q,
+                   const uint8_t* images, int n_trials, int T, const uint64_t* seeds, uint32_t* counts,
+                   uint32_t* raster, int flags) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  if (n_lif < 1 || n_lif > snn::kSparseMaxLif) return fail(SNN_EINVAL, "n_lif=%d outside [1, %d]", n_lif, snn::kSparseMaxLif);
+  if (n_trials < 0 || T < 0 || T > (1 << 30)) return fail(SNN_EINVAL, "bad n_trials / T");
+  if (!src_off) return fail(SNN_EINVAL, "src_off is NULL");
+  if (n_trials == 0) return SNN_OK;
+  if (!images || !seeds || !counts) return fail(SNN_EINVAL, "images / seeds / counts is NULL");
+  DevGuard g(h->dev);
+  const int n_in = h->n_in, n_src = n_in + n_lif;
+  // the graph is validated on the host (copied back first if it lives on the device)
+  std::vector<int32_t> off((size_t)n_src + 1);
+  if (is_device_ptr(src_off)) {
+    CUDA_TRY(cudaMemcpy(off.data(), src_off, off.size() * 4, cudaMemcpyDeviceToHost));
+  } else {
+    std::memcpy(off.data(), src_off, off.size() * 4);
+  }
+  if (off[0] != 0) return fail(SNN_EINVAL, "src_off[0] must be 0");
+  for (int s = 0; s < n_src; ++s)
+    if (off[s + 1] < off[s]) return fail(SNN_EINVAL, "src_off not non-decreasing at %d", s);
+  const size_t n_syn = (size_t)off[n_src];
+  if (n_syn > 0 && (!tgt || !q)) return fail(SNN_EINVAL, "tgt / q is NULL");
+  std::vector<uint16_t> ht(n_syn);
+  std::vector<uint8_t> hq(n_syn);
+  if (n_syn) {
+    CUDA_TRY(cudaMemcpy(ht.data(), tgt, n_syn * 2, is_device_ptr(tgt) ? cudaMemcpyDeviceToHost : cudaMemcpyHostToHost));
+    CUDA_TRY(cudaMemcpy(hq.data(), q, n_syn, is_device_ptr(q) ? cudaMemcpyDeviceToHost : cudaMemcpyHostToHost));
+  }
+  for (size_t k = 0; k < n_syn; ++k) {
+    if (ht[k] >= n_lif) return fail(SNN_EINVAL, "tgt[%zu]=%d >= n_lif", k, (int)ht[k]);
+    if (hq[k] > h->q_max) return fail(SNN_EINVAL, "q[%zu]=%d > q_max=%d", k, (int)hq[k], h->q_max);
+  }
+  if ((rc = ensure(h, &h->d_soff, &h->soff_cap, off.size()))) return rc;
+  if ((rc = ensure(h, &h->d_stgt, &h->stgt_cap, std::max<size_t>(n_syn, 1)))) return rc;
+  if ((rc = ensure(h, &h->d_sq, &h->sq_cap, std::max<size_t>(n_syn, 1)))) return rc;
+  CUDA_TRY(cudaMemcpyAsync(h->d_soff, off.data(), off.size() * 4, cudaMemcpyHostToDevice, h->stream));
+  if (n_syn) {
+    CUDA_TRY(cudaMemcpyAsync(h->d_stgt, ht.data(), n_syn * 2, cudaMemcpyHostToDevice, h->stream));
+    CUDA_TRY(cudaMemcpyAsync(h->d_sq, hq.data(), n_syn, cudaMemcpyHostToDevice, h->stream));
+  }
+  const uint8_t* img = nullptr;
+  if ((rc = stage(h, images, (size_t)n_trials * n_in, &h->d_img, &h->img_cap, &img))) return rc;
+  const unsigned long long* sd = nullptr;
+  if ((rc = stage(h, reinterpret_cast<const unsigned long long*>(seeds), (size_t)n_trials, &h->d_seeds,
+                  &h->seeds_cap, &sd)))
+    return rc;
+  const size_t n_counts = (size_t)n_trials * n_lif;
+  const size_t n_raster = (size_t)n_trials * T * ((n_lif + 31) / 32);
+  const bool counts_dev = is_device_ptr(counts);
+  const bool raster_dev = raster && is_device_ptr(raster);
+  uint32_t* dc = counts;
+  uint32_t* dr = raster;
+  if (!counts_dev) { if ((rc = ensure(h, &h->d_scounts, &h->scounts_cap, n_counts))) return rc; dc = h->d_scounts; }
+  if (raster && !raster_dev) { if ((rc = ensure(h, &h->d_sraster, &h->sraster_cap, n_raster))) return rc; dr = h->d_sraster; }
+  CUDA_TRY(cudaMemsetAsync(dc, 0, n_counts * 4, h->stream));
+  if (dr) CUDA_TRY(cudaMemsetAsync(dr, 0, n_raster * 4, h->stream));
+  if (!h->d_sstats) {
+    CUDA_TRY(dalloc(&h->d_sstats, 2));
+    CUDA_TRY(cudaMemsetAsync(h->d_sstats, 0, 2 * sizeof(unsigned long long), h->stream));
+  }
+  snn::SparseDesc d{};
+  const snn_params& p = h->p;
+  const double lsb = std::ldexp(1.0, -h->frac_bits);
+  d.n_in = n_in; d.n_lif = n_lif; d.T = T; d.n_trials = n_trials; d.t_ref = p.t_ref_steps;
+  d.af = (float)p.a; d.bf = (float)p.b; d.cf = (float)p.c; d.dtf = (float)p.dt_ms;
+  d.kI = (float)(p.v_spike * lsb); d.ief = (float)p.i_ext;
+  d.vthf = (float)p.v_th; d.vresetf = (float)p.v_reset; d.vinitf = (float)p.v_init;
+  d.A = h->A; d.B = h->B; d.C = h->C; d.E = h->E; d.Vth = h->Vth; d.Vreset = h->Vreset; d.Vinit = h->Vinit;
+  d.src_off = h->d_soff; d.tgt = h->d_stgt; d.q = h->d_sq; d.thr_enc = h->d_enc;
+  d.images = img; d.seeds = sd; d.counts = dc; d.raster = dr; d.stats = h->d_sstats;
+  const size_t smem = snn::sparse_smem_bytes(n_in, n_lif);
+  const int nthr = std::max(128, std::min(512, ((n_lif + 31) / 32) * 32));   // threads stride over neurons
+  int occ = 0, nsm = 0;
+  CUDA_TRY(snn::sparse_occupancy(h->p.membrane_mode, nthr, smem, &occ));
+  if (occ < 1) return fail(SNN_ESIZE, "sparse kernel cannot be resident (smem %zu B)", smem);
+  CUDA_TRY(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, h->dev));
+  CUDA_TRY(snn::launch_sparse(d, std::min(n_trials, occ * nsm), nthr, smem, h->p.membrane_mode, h->stream));
+  h->launches++;
+  if (!counts_dev) CUDA_TRY(cudaMemcpyAsync(counts, dc, n_counts * 4, cudaMemcpyDeviceToHost, h->stream));
+  if (raster && !raster_dev) CUDA_TRY(cudaMemcpyAsync(raster, dr, n_raster * 4, cudaMemcpyDeviceToHost, h->stream));
+  return finish(h, (counts_dev && (!raster || raster_dev)) ? flags : 0);
+}
+
+int snn_get_sparse_stats(snn_handle* h, uint64_t stats[2]) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  if (!stats) return fail(SNN_EINVAL, "stats is NULL");
+  stats[0] = stats[1] = 0;
+  if (!h->d_sstats) return SNN_OK;
+  DevGuard g(h->dev);
+  CUDA_TRY(cudaMemcpyAsync(stats, h->d_sstats, 2 * sizeof(uint64_t), cudaMemcpyDeviceToHost, h->stream));
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  return SNN_OK;
 }
 
 }  // extern "C"

@@ -152,4 +152,25 @@ cudaError_t launch_label(const uint32_t* counts, int n_images, int n_exc, const 
 cudaError_t launch_classify(const uint32_t* counts, int n_images, int n_exc, const int32_t* labels, int n_classes,
                             int32_t* pred, cudaStream_t s);
 
+// ---- NEXT-4: Fig. 4 sparse workload (snn_sparse.cu)
+struct SparseDesc {
+  int n_in, n_lif, T, n_trials, t_ref;
+  float af, bf, cf, dtf, kI, ief, vthf, vresetf, vinitf;
+  long long A, B, C, E;
+  int Vth, Vreset, Vinit;
+  const int32_t* src_off;            // [n_in + n_lif + 1] CSR by source
+  const uint16_t* tgt;               // [n_syn] target neuron
+  const uint8_t* q;                  // [n_syn] code
+  const unsigned long long* thr_enc; // [256]
+  const uint8_t* images;             // [n_trials][n_in]
+  const unsigned long long* seeds;   // [n_trials]
+  uint32_t* counts;                  // [n_trials][n_lif] (zeroed by the caller)
+  uint32_t* raster;                  // [n_trials][T][ceil(n_lif/32)] or null (zeroed by the caller)
+  unsigned long long* stats;         // [2] += input spikes, neuron spikes
+};
+constexpr int kSparseMaxLif = 16384;
+size_t sparse_smem_bytes(int n_in, int n_lif);
+cudaError_t sparse_occupancy(int fixed, int nthr, size_t smem, int* out);
+cudaError_t launch_sparse(const SparseDesc& d, int grid, int nthr, size_t smem, int fixed, cudaStream_t s);
+
 }  // namespace snn

@@ -25,6 +25,7 @@ EXPORTS = [
     "snn_get_info", "snn_set_trace", "snn_get_trace", "snn_last_error",
     "snn_create_shard", "snn_shard_ipc_handle", "snn_shard_connect", "snn_shard_link",
     "snn_infer", "snn_get_infer_stats", "snn_label", "snn_classify",
+    "snn_sparse_run", "snn_get_sparse_stats",
 ]
 SNN_IPC_HANDLE_BYTES = 64
 NINFO = 18
@@ -99,6 +100,8 @@ def lib():
             "snn_get_infer_stats": ([vp, vp], i32),
             "snn_label": ([vp, vp, i32, vp, i32, vp], i32),
             "snn_classify": ([vp, vp, i32, vp, i32, vp], i32),
+            "snn_sparse_run": ([vp, i32, vp, vp, vp, vp, i32, i32, vp, vp, vp, i32], i32),
+            "snn_get_sparse_stats": ([vp, vp], i32),
         }
         for name, (args, res) in sig.items():
             f = getattr(L, name)
@@ -306,6 +309,23 @@ class Network:
             pred = np.zeros(n, dtype=np.int32)
         _check(lib().snn_classify(self._h, _ptr(counts), n, _ptr(labels), n_classes, _ptr(pred)), "snn_classify")
         return pred
+
+    # ---- NEXT-4: the Fig. 4 sparse workload (include/snn.h snn_sparse_run)
+    def sparse_run(self, n_lif: int, src_off, tgt, q, images, T: int, seeds, counts=None, raster=None,
+                   flags: int = 0):
+        """Spike counts (n_trials, n_lif) u32 of the sparse recurrent network (this handle's parameters);
+        raster: optional (n_trials, T, ceil(n_lif/32)) u32 output buffer."""
+        n = int(images.shape[0])
+        if counts is None:
+            counts = np.zeros((n, n_lif), dtype=np.uint32)
+        _check(lib().snn_sparse_run(self._h, n_lif, _ptr(src_off), _ptr(tgt), _ptr(q), _ptr(images), n, T,
+                                    _ptr(seeds), _ptr(counts), _ptr(raster), flags), "snn_sparse_run")
+        return counts
+
+    def sparse_stats(self) -> np.ndarray:
+        out = np.zeros(2, dtype=np.uint64)
+        _check(lib().snn_get_sparse_stats(self._h, _ptr(out)), "snn_get_sparse_stats")
+        return out
 
     # ---- column sharding (include/snn.h, DESIGN.md §10)
     def ipc_handle(self) -> bytes:
