@@ -194,13 +194,17 @@ class OracleNet:
         flags = ORACLE_RASTER_INPUT | (ORACLE_KEEP_STATE if keep_state else 0)
         self.present_ex(raster, T, seed, flags, t0)
 
+    @property
+    def code_dtype(self):
+        return np.uint16 if self.bits > 8 else np.uint8
+
     def weights(self) -> np.ndarray:
-        out = np.empty((self.n_in, self.n_exc), dtype=np.uint8)
+        out = np.empty((self.n_in, self.n_exc), dtype=self.code_dtype)
         self._check(lib().oracle_get_weights(self._h, _ptr(out)), "oracle_get_weights")
         return out
 
     def set_weights(self, codes: np.ndarray):
-        c = np.ascontiguousarray(codes, dtype=np.uint8).reshape(self.n_in, self.n_exc)
+        c = np.ascontiguousarray(codes, dtype=self.code_dtype).reshape(self.n_in, self.n_exc)
         self._check(lib().oracle_set_weights(self._h, _ptr(c)), "oracle_set_weights")
 
     def spikes(self) -> np.ndarray:

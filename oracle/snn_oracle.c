@@ -33,11 +33,12 @@
 #define TAG_LTP   3u
 #define TAG_ROUND 4u
 #define TAG_INIT  5u
+#define TAG_ROUND_LTD 6u   /* 16-bit stochastic arm: rounding draw of an LTD step [R27] */
 
 struct oracle_net {
   int n_in, n_exc, bits, frac_bits, q_max;
   oracle_params p;
-  uint8_t* q;                 /* conductance codes q[i*n_exc + j]; G = q * 2^-frac_bits [R9] */
+  uint16_t* q;                /* conductance codes q[i*n_exc + j]; G = q * 2^-frac_bits [R9] */
   /* state [R5] */
   float*   v_f;               /* membrane, fp32 mode */
   int32_t* v_x;               /* membrane, Q15.16 fixed mode */
@@ -49,8 +50,10 @@ struct oracle_net {
   uint64_t thr_enc[256];
   uint64_t thr_pot[LUT_MAX]; int L_pot;
   uint64_t thr_dep[LUT_MAX]; int L_dep;
-  int64_t  det_p_base[256]; uint64_t det_p_thr[256];
-  int64_t  det_d_base[256]; uint64_t det_d_thr[256];
+  /* eqs.(4)(5) magnitudes in LSB per code q (base + rounding threshold), q = 0..q_max [R16][R17]: the
+   * deterministic arm at every width, and the stochastic arm's step size at 16 bits [R27] */
+  int64_t* det_p_base; uint64_t* det_p_thr;
+  int64_t* det_d_base; uint64_t* det_d_thr;
   /* fixed-point constants [R12] */
   int64_t A, B, C, E; int32_t Vth, Vreset, Vinit;
   /* fp32 constants [R12] */
@@ -110,7 +113,7 @@ static int build_exp_lut(double gamma, double tau, double dt, uint64_t* thr, int
 
 static int validate(int n_in, int n_exc, int bits, const oracle_params* p) {
   if (n_in < 1 || n_in > 8192 || n_exc < 1 || n_exc > (1 << 20)) return E_INVAL;
-  if (bits != 2 && bits != 4 && bits != 8) return E_INVAL;
+  if (bits != 2 && bits != 4 && bits != 8 && bits != 16) return E_INVAL;
   if (!(p->dt_ms > 0.0)) return E_INVAL;
   if (!(p->f_min_hz >= 0.0 && p->f_max_hz >= p->f_min_hz)) return E_INVAL;
   if (p->f_max_hz * p->dt_ms * 1e-3 > 1.0) return E_INVAL;
@@ -150,6 +153,11 @@ int oracle_create(int n_in, int n_exc, int bits, const oracle_params* p, oracle_
       build_exp_lut(p->gamma_dep, p->tau_dep, p->dt_ms, n->thr_dep, &n->L_dep)) { free(n); return E_INVAL; }
 
   /* eqs.(4)(5) in units of LSB, rounded by eq.(8) / trunc / nearest [R16][R17] */
+  n->det_p_base = (int64_t*)malloc(sizeof(int64_t) * (size_t)(n->q_max + 1));
+  n->det_d_base = (int64_t*)malloc(sizeof(int64_t) * (size_t)(n->q_max + 1));
+  n->det_p_thr = (uint64_t*)malloc(sizeof(uint64_t) * (size_t)(n->q_max + 1));
+  n->det_d_thr = (uint64_t*)malloc(sizeof(uint64_t) * (size_t)(n->q_max + 1));
+  if (!n->det_p_base || !n->det_d_base || !n->det_p_thr || !n->det_d_thr) { oracle_destroy(n); return E_NOMEM; }
   for (int qq = 0; qq <= n->q_max; ++qq) {
     double G = (double)qq * lsb;
     double xp = ldexp(p->alpha_p * exp(-p->beta_p * (G - p->g_min) / (p->g_max - p->g_min)), n->frac_bits);
@@ -180,7 +188,7 @@ int oracle_create(int n_in, int n_exc, int bits, const oracle_params* p, oracle_
   n->vthf = (float)p->v_th; n->vresetf = (float)p->v_reset; n->vinitf = (float)p->v_init;
 
   size_t nq = (size_t)n_in * (size_t)n_exc;
-  n->q = (uint8_t*)malloc(nq);
+  n->q = (uint16_t*)malloc(nq * sizeof(uint16_t));
   n->v_f = (float*)calloc((size_t)n_exc, sizeof(float));
   n->v_x = (int32_t*)calloc((size_t)n_exc, sizeof(int32_t));
   n->cnt = (int32_t*)calloc((size_t)n_exc, sizeof(int32_t));
@@ -192,7 +200,7 @@ int oracle_create(int n_in, int n_exc, int bits, const oracle_params* p, oracle_
   for (int i = 0; i < n_in; ++i)
     for (int j = 0; j < n_exc; ++j) {
       uint32_t u = draw(p->init_seed, (uint32_t)i, (uint32_t)(j >> 2), 0u, TAG_INIT, j & 3);
-      n->q[(size_t)i * n_exc + j] = (uint8_t)(((uint64_t)u * (uint64_t)(n->q_max + 1)) >> 32);
+      n->q[(size_t)i * n_exc + j] = (uint16_t)(((uint64_t)u * (uint64_t)(n->q_max + 1)) >> 32);
     }
   /* state as after a reset [R5] */
   for (int j = 0; j < n_exc; ++j) { n->v_f[j] = n->vinitf; n->v_x[j] = n->Vinit; n->last_post[j] = NEVER; }
@@ -205,6 +213,7 @@ int oracle_destroy(oracle_net* n) {
   if (!n) return 0;
   free(n->q); free(n->v_f); free(n->v_x); free(n->cnt); free(n->last_post); free(n->last_pre);
   free(n->raster); free(n->in_raster);
+  free(n->det_p_base); free(n->det_d_base); free(n->det_p_thr); free(n->det_d_thr);
   free(n);
   return 0;
 }
@@ -335,8 +344,15 @@ int oracle_present_ex(oracle_net* n, const void* input, int T, uint64_t seed, in
           uint32_t u = draw(seed, (uint32_t)t, (uint32_t)i, (uint32_t)(j >> 2), TAG_LTD, j & 3);
           if ((uint64_t)u < n->thr_dep[D]) {
             n->stats[3]++;
-            uint8_t* qq = &n->q[(size_t)i * n_exc + j];
-            if (*qq > 0) *qq -= 1;
+            uint16_t* qq = &n->q[(size_t)i * n_exc + j];
+            if (n->bits <= 8) {
+              if (*qq > 0) *qq -= 1;                   /* dG = 1 LSB */
+            } else {                                   /* 16 bit: dG = eq.(5), rounded (eq.(8)) [R27] */
+              uint32_t u2 = draw(seed, (uint32_t)t, (uint32_t)i, (uint32_t)(j >> 2), TAG_ROUND_LTD, j & 3);
+              int64_t dq = n->det_d_base[*qq] + ((uint64_t)u2 < n->det_d_thr[*qq] ? 1 : 0);
+              int64_t q1 = (int64_t)*qq - dq;
+              *qq = (uint16_t)(q1 < 0 ? 0 : q1);
+            }
           }
         }
       }
@@ -351,8 +367,15 @@ int oracle_present_ex(oracle_net* n, const void* input, int T, uint64_t seed, in
           uint32_t u = draw(seed, (uint32_t)t, (uint32_t)W, (uint32_t)(i >> 2), TAG_LTP, i & 3);
           if ((uint64_t)u < n->thr_pot[D]) {
             n->stats[5]++;
-            uint8_t* qq = &n->q[(size_t)i * n_exc + W];
-            if (*qq < n->q_max) *qq += 1;
+            uint16_t* qq = &n->q[(size_t)i * n_exc + W];
+            if (n->bits <= 8) {
+              if (*qq < n->q_max) *qq += 1;            /* dG = 1 LSB */
+            } else {                                   /* 16 bit: dG = eq.(4), rounded (eq.(8)) [R27] */
+              uint32_t u2 = draw(seed, (uint32_t)t, (uint32_t)W, (uint32_t)(i >> 2), TAG_ROUND, i & 3);
+              int64_t dq = n->det_p_base[*qq] + ((uint64_t)u2 < n->det_p_thr[*qq] ? 1 : 0);
+              int64_t q1 = (int64_t)*qq + dq;
+              *qq = (uint16_t)(q1 > n->q_max ? n->q_max : q1);
+            }
           }
         }
       }
@@ -362,7 +385,7 @@ int oracle_present_ex(oracle_net* n, const void* input, int T, uint64_t seed, in
       for (int m = 0; m < nsp; ++m) {
         int W = spikers[m];
         for (int i = 0; i < n_in; ++i) {
-          uint8_t* qq = &n->q[(size_t)i * n_exc + W];
+          uint16_t* qq = &n->q[(size_t)i * n_exc + W];
           int q0 = *qq;
           int pot = n->last_pre[i] != NEVER && (t - n->last_pre[i]) <= p->t_ltp_steps;
           int64_t base = pot ? n->det_p_base[q0] : n->det_d_base[q0];
@@ -372,7 +395,7 @@ int oracle_present_ex(oracle_net* n, const void* input, int T, uint64_t seed, in
           int64_t q1 = pot ? q0 + dq : q0 - dq;
           if (q1 < 0) q1 = 0;
           if (q1 > n->q_max) q1 = n->q_max;
-          *qq = (uint8_t)q1;
+          *qq = (uint16_t)q1;
           n->stats[pot ? 4 : 2]++;
           if (dq > 0) n->stats[pot ? 5 : 3]++;
         }
@@ -386,17 +409,23 @@ int oracle_present_ex(oracle_net* n, const void* input, int T, uint64_t seed, in
 }
 
 /* ---------------------------------------------------------------- accessors */
-int oracle_get_weights(const oracle_net* n, uint8_t* codes) {
+/* codes: one byte per code (bits <= 8) or one uint16 per code (bits = 16) */
+int oracle_get_weights(const oracle_net* n, void* codes) {
   if (!n || !codes) return E_INVAL;
-  memcpy(codes, n->q, (size_t)n->n_in * n->n_exc);
+  size_t nq = (size_t)n->n_in * n->n_exc;
+  if (n->bits > 8) { memcpy(codes, n->q, nq * sizeof(uint16_t)); return 0; }
+  for (size_t k = 0; k < nq; ++k) ((uint8_t*)codes)[k] = (uint8_t)n->q[k];
   return 0;
 }
 
-int oracle_set_weights(oracle_net* n, const uint8_t* codes) {
+int oracle_set_weights(oracle_net* n, const void* codes) {
   if (!n || !codes) return E_INVAL;
   size_t nq = (size_t)n->n_in * n->n_exc;
-  for (size_t k = 0; k < nq; ++k) if (codes[k] > n->q_max) return E_INVAL;
-  memcpy(n->q, codes, nq);
+  for (size_t k = 0; k < nq; ++k) {
+    int c = n->bits > 8 ? ((const uint16_t*)codes)[k] : ((const uint8_t*)codes)[k];
+    if (c > n->q_max) return E_INVAL;
+  }
+  for (size_t k = 0; k < nq; ++k) n->q[k] = n->bits > 8 ? ((const uint16_t*)codes)[k] : ((const uint8_t*)codes)[k];
   return 0;
 }
 

@@ -55,8 +55,9 @@ int oracle_destroy(oracle_net* net);
 int oracle_present(oracle_net* net, const uint8_t* image, int T, uint64_t seed);
 int oracle_present_ex(oracle_net* net, const void* input, int T, uint64_t seed, int flags, int t0);
 
-int oracle_get_weights(const oracle_net* net, uint8_t* codes /* n_in*n_exc, row-major [i][j] */);
-int oracle_set_weights(oracle_net* net, const uint8_t* codes);
+/* codes n_in*n_exc row-major [i][j]: uint8 per code for bits <= 8, uint16 per code for bits = 16 */
+int oracle_get_weights(const oracle_net* net, void* codes);
+int oracle_set_weights(oracle_net* net, const void* codes);
 /* last presentation's output raster, T x ceil(n_exc/32) u32, bit j%32 of word j/32 */
 int oracle_get_spikes(const oracle_net* net, uint32_t* raster, size_t cap_words);
 /* last presentation's input raster, T x ceil(n_in/32) u32 */

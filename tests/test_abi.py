@@ -74,7 +74,7 @@ def test_invalid_params_rejected_before_cuda(bad):
     assert e.value.rc == S.SNN_EINVAL
 
 
-@pytest.mark.parametrize("bits", [0, 1, 3, 16])
+@pytest.mark.parametrize("bits", [0, 1, 3, 12, 32])
 def test_invalid_bits_rejected(bits):
     with pytest.raises(P.SnnError) as e:
         P.Network(784, 10, bits, P.preset("8b"))

@@ -364,7 +364,7 @@ def _det_run(bits, rounding, q_init, pre_fires, reps=1, seed0=0):
             raster[2, i // 32] |= np.uint32(1 << (i % 32))
     outs = []
     for r in range(reps):
-        net.set_weights(np.full((n_in, 1), q_init, np.uint8))
+        net.set_weights(np.full((n_in, 1), q_init, net.code_dtype))
         _force_state(net, 5)
         net.present_raster(raster, 6, seed=seed0 + r, keep_state=True, t0=0)
         assert _spike_steps(net, 6) == [5]
@@ -402,6 +402,57 @@ def test_det_arm_stochastic_rounding_eq8():
     assert abs(k - 0.56 * N) <= 3 * math.sqrt(N * 0.56 * 0.44)
 
 
+def test_det_arm_hand_values_16bit():
+    """16 bit (frac 16, LSB 2^-16): eq.(4) at G = 0: 0.01 * 65536 = 655.36 LSB -> trunc 655, nearest 655;
+    eq.(5) at G = 65535/65536: 0.005 e^{-3/65536} * 65536 = 327.665 LSB -> trunc 327, nearest 328."""
+    fires = [True, False]
+    assert _det_run(16, 0, 0, fires)[0].tolist() == [655, 0]
+    assert _det_run(16, 1, 0, fires)[0].tolist() == [655, 0]
+    assert _det_run(16, 0, 65535, fires)[0].tolist() == [65535, 65535 - 327]
+    assert _det_run(16, 1, 65535, fires)[0].tolist() == [65535, 65535 - 328]
+
+
+def _stoch16_run(rounding, q_init, pre_step, reps, gamma_dep=0.0, tau_dep=10.0):
+    """16-bit stochastic arm (R27): one post spike forced at t=5; 64 inputs spike at `pre_step`
+    (5 -> LTP with D = 0, 6 -> LTD with D = 1)."""
+    n_in = 64
+    p = O.params("16b", rounding=rounding, gamma_pot=1.0, gamma_dep=gamma_dep, tau_dep=tau_dep, i_ext=60.0,
+                 v_spike=1e-9, t_ref_steps=100000)
+    net = O.OracleNet(n_in, 1, 16, p)
+    raster = np.zeros((8, 2), np.uint32)
+    raster[pre_step, :] = 0xFFFFFFFF
+    outs = []
+    for r in range(reps):
+        net.set_weights(np.full((n_in, 1), q_init, np.uint16))
+        _force_state(net, 5)
+        net.present_raster(raster, 8, seed=100 + r, keep_state=True, t0=0)
+        assert _spike_steps(net, 8) == [5]
+        outs.append(net.weights()[:, 0].astype(int))
+    return np.concatenate(outs)
+
+
+def test_stochastic_arm_16bit_magnitudes():
+    """P:89 "For 16-bit ... after floating point calculation of change in conductance dG, the result is
+    rounded": an LTP event moves q by eq.(4) rounded (trunc / nearest: 655), and with eq.(8) by 655 or 656
+    with P(656) = 0.36; gamma_pot = 1 at D = 0 makes the event certain (eq.(6))."""
+    assert set(_stoch16_run(0, 0, 5, 2).tolist()) == {655}
+    assert set(_stoch16_run(1, 0, 5, 2).tolist()) == {655}
+    v = _stoch16_run(2, 0, 5, 40)
+    assert set(v.tolist()) <= {655, 656}
+    N, k = v.size, int((v == 656).sum())
+    assert abs(k - 0.36 * N) <= 3 * math.sqrt(N * 0.36 * 0.64)
+
+
+def test_stochastic_arm_16bit_ltd():
+    """A pre spike one step after the post spike: LTD event w.p. P_dep(1) = gamma_dep e^{-1/tau_dep}
+    (eq.(7)), moving q_max by eq.(5) rounded to nearest (328 LSB)."""
+    v = _stoch16_run(1, 65535, 6, 40, gamma_dep=1.0, tau_dep=100.0)
+    assert set(v.tolist()) <= {65535, 65535 - 328}
+    N, k = v.size, int((v == 65535 - 328).sum())
+    P = math.exp(-1.0 / 100.0)
+    assert abs(k - P * N) <= 3 * math.sqrt(N * P * (1 - P)) + 1
+
+
 # ------------------------------------------------------------------ validation
 @pytest.mark.parametrize("bad", [dict(gamma_pot=1.5), dict(tau_dep=0.0), dict(f_max_hz=2000.0),
                                  dict(f_min_hz=30.0, f_max_hz=20.0), dict(wta_mode=3), dict(g_min=0.1),
@@ -412,7 +463,7 @@ def test_invalid_params_rejected(bad):
     assert e.value.rc == -1
 
 
-@pytest.mark.parametrize("bits", [0, 1, 3, 16])
+@pytest.mark.parametrize("bits", [0, 1, 3, 12, 32])
 def test_invalid_bits_rejected(bits):
     with pytest.raises(O.OracleError):
         O.OracleNet(784, 10, bits, O.params("8b"))
