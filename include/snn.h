@@ -94,13 +94,17 @@ typedef struct snn_params {
 #define SNN_PRESET_2B  0
 #define SNN_PRESET_4B  1
 #define SNN_PRESET_8B  2
-#define SNN_PRESET_16B 3   /* parameters only: 16-bit codes are not built (SNN_EINVAL at create) */
+#define SNN_PRESET_16B 3   /* Table I "16 bit" row: use with bits = 16 (R27) */
 #define SNN_PRESET_HF  4   /* "high frequency": 5-78 Hz, tau_pot 80, tau_dep 5 */
 int snn_params_preset(snn_params* p, int preset);
 
 typedef struct snn_handle snn_handle;
 
-/* Create a network n_in -> n_exc with `bits`-bit conductance codes (2, 4 or 8).
+/* Create a network n_in -> n_exc with `bits`-bit conductance codes (2, 4, 8 or 16).
+ * 16 bits (NEXT-2, "For 16-bit ... after floating point calculation of change in conductance dG,
+ * the result is rounded"; R27): every STDP event (stochastic arm) moves the code by the
+ * eq.(4)/(5) magnitude rounded by `rounding` instead of one LSB; 16-bit handles run on the per-step
+ * engine (SNN_ENGINE_STEP is selected automatically) and cannot be sharded or used for snn_infer.
  * Conductances are initialised on the device (R4).  SNN_ESIZE if the network does not fit the
  * on-chip layout.  *out receives the handle. */
 int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** out);
@@ -142,7 +146,8 @@ int snn_present_raster(snn_handle* h, const uint32_t* raster, int T, uint64_t se
 int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images, int n_images, int T,
                      const uint64_t* const* seeds);
 
-/* Readout.  codes: n_in x n_exc bytes, row-major [i][j], one code per byte (G = code * 2^-frac_bits). */
+/* Readout.  codes: n_in x n_exc codes, row-major [i][j], one code per byte (bits <= 8) or one
+ * little-endian uint16 per code (bits = 16); G = code * 2^-frac_bits.  cap / n are in BYTES. */
 int snn_get_weights(snn_handle* h, uint8_t* codes, size_t cap);
 int snn_set_weights(snn_handle* h, const uint8_t* codes, size_t n);
 /* Output raster of the last presented image: T x ceil(n_exc/32) u32, bit j%32 of word j/32. */

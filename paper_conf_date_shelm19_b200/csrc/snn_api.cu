@@ -140,7 +140,7 @@ int validate(int n_in, int n_exc, int bits, const snn_params* p) {
   if (!p) return fail(SNN_EINVAL, "params is NULL");
   if (n_in < 1 || n_in > 8192) return fail(SNN_EINVAL, "n_in=%d outside [1, 8192]", n_in);
   if (n_exc < 1 || n_exc > (1 << 20)) return fail(SNN_EINVAL, "n_exc=%d outside [1, 2^20]", n_exc);
-  if (bits != 2 && bits != 4 && bits != 8) return fail(SNN_EINVAL, "bits=%d not in {2,4,8}", bits);
+  if (bits != 2 && bits != 4 && bits != 8 && bits != 16) return fail(SNN_EINVAL, "bits=%d not in {2,4,8,16}", bits);
   if (!(p->dt_ms > 0.0)) return fail(SNN_EINVAL, "dt_ms must be > 0");
   if (!(p->f_min_hz >= 0.0 && p->f_max_hz >= p->f_min_hz)) return fail(SNN_EINVAL, "need 0 <= f_min <= f_max");
   if (p->f_max_hz * p->dt_ms * 1e-3 > 1.0) return fail(SNN_EINVAL, "f_max * dt > 1 (spike probability > 1)");
@@ -489,9 +489,10 @@ int create_impl(int n_in, int n_exc, int bits, const snn_params* p, int col_base
   int smem_optin = 0;
   cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, h->dev);
   h->ngroups = (n_exc + 31) / 32;
-  h->engine = p->engine == SNN_ENGINE_STEP ? SNN_ENGINE_STEP : SNN_ENGINE_EVENT;
+  // 16-bit codes (NEXT-2, R27) run on the per-step engine: the event kernels pack <= 8-bit codes in SWAR lanes
+  h->engine = (p->engine == SNN_ENGINE_STEP || bits > 8) ? SNN_ENGINE_STEP : SNN_ENGINE_EVENT;
   // the lean kernel covers the paper's default learning mode; SNN_NO_LEAN=1 disables it
-  const bool lean_mode = p->engine == SNN_ENGINE_EVENT && p->wta_mode == SNN_WTA_HARD &&
+  const bool lean_mode = p->engine == SNN_ENGINE_EVENT && bits <= 8 && p->wta_mode == SNN_WTA_HARD &&
                          p->inh_mode == SNN_INH_RESET && p->stdp_mode == SNN_STDP_STOCH && world == 1 &&
                          !(getenv("SNN_NO_LEAN") && atoi(getenv("SNN_NO_LEAN")) != 0);
   int chosen = 0;
@@ -593,7 +594,7 @@ int create_impl(int n_in, int n_exc, int bits, const snn_params* p, int col_base
   ALLOC(h->d_lpost, (size_t)n_exc);
   ALLOC(h->d_lpre, (size_t)n_in);
   ALLOC(h->d_stats, SNN_NSTATS);
-  ALLOC(h->d_codes, (size_t)n_in * n_exc);
+  ALLOC(h->d_codes, (size_t)n_in * n_exc * (bits > 8 ? 2 : 1));
   ALLOC(h->d_bad, 1);
   if (world > 1) {
     ALLOC(h->d_mbox, 1);
@@ -661,7 +662,7 @@ int snn_create_shard(int n_in, int n_exc_total, int bits, const snn_params* p, i
   if (rc) return rc;
   if (world < 1 || world > snn::kMaxWorld) return fail(SNN_EINVAL, "world=%d outside [1, %d]", world, snn::kMaxWorld);
   if (shard < 0 || shard >= world) return fail(SNN_EINVAL, "shard=%d outside [0, %d)", shard, world);
-  if (p->engine != SNN_ENGINE_EVENT) return fail(SNN_EINVAL, "column sharding needs the event engine");
+  if (p->engine != SNN_ENGINE_EVENT || bits > 8) return fail(SNN_EINVAL, "column sharding needs the event engine (bits <= 8)");
   const int G = (n_exc_total + 31) / 32;
   if (G < world) return fail(SNN_EINVAL, "%d column groups of 32 cannot feed %d shards", G, world);
   const int lo = 32 * (int)(((long long)shard * G) / world);
@@ -932,7 +933,7 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
 int snn_get_weights(snn_handle* h, uint8_t* codes, size_t cap) {
   int rc = check_handle(h);
   if (rc) return rc;
-  const size_t n = (size_t)h->n_in * h->n_exc;
+  const size_t n = (size_t)h->n_in * h->n_exc * (h->bits > 8 ? 2 : 1);     // bytes
   if (!codes) return fail(SNN_EINVAL, "codes is NULL");
   if (cap < n) return fail(SNN_ESIZE, "need %zu bytes", n);
   DevGuard g(h->dev);
@@ -948,14 +949,15 @@ int snn_get_weights(snn_handle* h, uint8_t* codes, size_t cap) {
 int snn_set_weights(snn_handle* h, const uint8_t* codes, size_t n) {
   int rc = check_handle(h);
   if (rc) return rc;
-  const size_t need = (size_t)h->n_in * h->n_exc;
+  const size_t ncodes = (size_t)h->n_in * h->n_exc;
+  const size_t need = ncodes * (h->bits > 8 ? 2 : 1);                          // bytes
   if (!codes) return fail(SNN_EINVAL, "codes is NULL");
   if (n < need) return fail(SNN_ESIZE, "need %zu bytes", need);
   DevGuard g(h->dev);
   CUDA_TRY(cudaMemcpyAsync(h->d_codes, codes, need, is_device_ptr(codes) ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice,
                            h->stream));
   CUDA_TRY(cudaMemsetAsync(h->d_bad, 0, sizeof(int), h->stream));
-  CUDA_TRY(snn::launch_check_codes(h->d_codes, need, h->q_max, h->d_bad, h->stream));
+  CUDA_TRY(snn::launch_check_codes(h->d_codes, ncodes, h->bits, h->q_max, h->d_bad, h->stream));
   int bad = 0;
   CUDA_TRY(cudaMemcpyAsync(&bad, h->d_bad, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
   CUDA_TRY(cudaStreamSynchronize(h->stream));
@@ -1144,6 +1146,7 @@ int snn_infer(snn_handle* h, const uint8_t* images, int n_images, int T, const u
   if (n_images < 0 || T < 0) return fail(SNN_EINVAL, "negative n_images / T");
   if (T > 65535) return fail(SNN_EINVAL, "T=%d exceeds 65535 for inference", T);
   if (h->world > 1) return fail(SNN_EINVAL, "inference runs on unsharded handles");
+  if (h->bits > 8) return fail(SNN_EINVAL, "inference supports 2/4/8-bit codes (16-bit: NEXT-2 learning only)");
   if (h->n_exc > snn::kInferMaxCols) return fail(SNN_ESIZE, "n_exc=%d exceeds %d for inference", h->n_exc,
                                                  snn::kInferMaxCols);
   if (n_images == 0) return SNN_OK;

@@ -12,7 +12,7 @@ constexpr int kLutMax = 4096;       // R19
 constexpr int kNever = -1;
 constexpr int kPadRows = 16;        // fixed-width per-step row slots used by the event engine's block integration
 
-enum : uint32_t { TAG_ENC = 1, TAG_LTD = 2, TAG_LTP = 3, TAG_ROUND = 4, TAG_INIT = 5 };
+enum : uint32_t { TAG_ENC = 1, TAG_LTD = 2, TAG_LTP = 3, TAG_ROUND = 4, TAG_INIT = 5, TAG_ROUND_LTD = 6 };
 enum : int { FLAG_RASTER_INPUT = 1, FLAG_KEEP_STATE = 2, FLAG_RECORD_INPUT = 4, FLAG_ASYNC = 8, FLAG_FLOOR = 16 };
 
 // Everything one network needs inside the persistent kernel.  Built per launch on the host.
@@ -119,9 +119,9 @@ cudaError_t launch_present_lean(const LaunchParams& lp, int n_nets, int cs, int 
                                 int fixed, cudaStream_t s);
 cudaError_t query_max_clusters(int cs, int nthr, size_t smem, int* out);
 cudaError_t launch_init_weights(const NetDesc& d, uint64_t init_seed, cudaStream_t s);
-cudaError_t launch_pack_weights(const NetDesc& d, const uint8_t* codes, cudaStream_t s);
-cudaError_t launch_unpack_weights(const NetDesc& d, uint8_t* codes, cudaStream_t s);
-cudaError_t launch_check_codes(const uint8_t* codes, size_t n, int q_max, int* bad, cudaStream_t s);
+cudaError_t launch_pack_weights(const NetDesc& d, const void* codes, cudaStream_t s);      // u8 / u16 (bits 16) codes
+cudaError_t launch_unpack_weights(const NetDesc& d, void* codes, cudaStream_t s);
+cudaError_t launch_check_codes(const void* codes, size_t n, int bits, int q_max, int* bad, cudaStream_t s);
 size_t present_smem_bytes(int n_in, int wpr, int L_pot, int L_dep, int q_max, int nthr);
 
 // ---- NEXT-1: batch-parallel inference with frozen weights (snn_infer.cu)

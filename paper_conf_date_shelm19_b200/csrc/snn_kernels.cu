@@ -33,10 +33,11 @@ __host__ __device__ inline SmemLayout smem_layout(int n_in, int slice_words, int
   L.w = o;      o = align16(o + (size_t)slice_words * 4);
   L.pot = o;    o = align16(o + (size_t)(L_pot > 0 ? L_pot : 1) * 4);
   L.dep = o;    o = align16(o + (size_t)(L_dep > 0 ? L_dep : 1) * 4);
-  L.dbp = o;    o = align16(o + (size_t)(q_max + 1) * 4);
-  L.dbd = o;    o = align16(o + (size_t)(q_max + 1) * 4);
-  L.dtp = o;    o = align16(o + (size_t)(q_max + 1) * 4);
-  L.dtd = o;    o = align16(o + (size_t)(q_max + 1) * 4);
+  const size_t ntab = q_max < 256 ? (size_t)(q_max + 1) : 1;   // 16-bit tables stay in global memory (L2)
+  L.dbp = o;    o = align16(o + ntab * 4);
+  L.dbd = o;    o = align16(o + ntab * 4);
+  L.dtp = o;    o = align16(o + ntab * 4);
+  L.dtd = o;    o = align16(o + ntab * 4);
   L.lpre = o;   o = align16(o + (size_t)n_in * 4);
   L.spk = o;    o = align16(o + (size_t)nwi * 4);
   L.misc = o;   o = align16(o + 16 * 4);
@@ -73,10 +74,11 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
   uint32_t* s_w = reinterpret_cast<uint32_t*>(smem + L.w);
   uint32_t* s_pot = reinterpret_cast<uint32_t*>(smem + L.pot);
   uint32_t* s_dep = reinterpret_cast<uint32_t*>(smem + L.dep);
-  int* s_dbp = reinterpret_cast<int*>(smem + L.dbp);
-  int* s_dbd = reinterpret_cast<int*>(smem + L.dbd);
-  uint32_t* s_dtp = reinterpret_cast<uint32_t*>(smem + L.dtp);
-  uint32_t* s_dtd = reinterpret_cast<uint32_t*>(smem + L.dtd);
+  const bool tab_smem = d.q_max < 256;
+  const int* s_dbp = tab_smem ? reinterpret_cast<const int*>(smem + L.dbp) : d.det_base_p;
+  const int* s_dbd = tab_smem ? reinterpret_cast<const int*>(smem + L.dbd) : d.det_base_d;
+  const uint32_t* s_dtp = tab_smem ? reinterpret_cast<const uint32_t*>(smem + L.dtp) : d.det_thr_p;
+  const uint32_t* s_dtd = tab_smem ? reinterpret_cast<const uint32_t*>(smem + L.dtd) : d.det_thr_d;
   int* s_lpre = reinterpret_cast<int*>(smem + L.lpre);
   uint32_t* s_spk = reinterpret_cast<uint32_t*>(smem + L.spk);
   int* s_misc = reinterpret_cast<int*>(smem + L.misc);
@@ -92,10 +94,11 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
   const int ngrp_cta = g1 - g0;
   const bool mycol = tid < ncols;
   const int j = col0 + tid;
-  const int lg = bits == 2 ? 4 : (bits == 4 ? 3 : 2);   // log2(codes per u32 word)
+  const int lg = bits == 2 ? 4 : (bits == 4 ? 3 : (bits == 8 ? 2 : 1));   // log2(codes per u32 word)
   const int wj = tid >> lg;
   const int sh = (tid & ((1 << lg) - 1)) * bits;
   const uint32_t fmask = (1u << bits) - 1u;
+  const bool wide = bits > 8;       // 16-bit codes: STDP steps by eqs.(4)(5) magnitudes, not 1 LSB (R27)
   const int nq4 = (n_in + 3) >> 2;
   const bool fixed = d.membrane_mode == 1;
   const bool hard = d.wta_mode == 0;
@@ -107,10 +110,11 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
   for (int k = tid; k < 256; k += nthr) s_enc[k] = d.thr_enc[k];
   for (int k = tid; k < L_pot; k += nthr) s_pot[k] = d.pot_m1[k];
   for (int k = tid; k < L_dep; k += nthr) s_dep[k] = d.dep_m1[k];
-  for (int k = tid; k <= qmax; k += nthr) {
-    s_dbp[k] = d.det_base_p[k]; s_dbd[k] = d.det_base_d[k];
-    s_dtp[k] = d.det_thr_p[k];  s_dtd[k] = d.det_thr_d[k];
-  }
+  if (tab_smem)
+    for (int k = tid; k <= qmax; k += nthr) {
+      const_cast<int*>(s_dbp)[k] = d.det_base_p[k]; const_cast<int*>(s_dbd)[k] = d.det_base_d[k];
+      const_cast<uint32_t*>(s_dtp)[k] = d.det_thr_p[k];  const_cast<uint32_t*>(s_dtd)[k] = d.det_thr_d[k];
+    }
   {
     const uint4* src = reinterpret_cast<const uint4*>(d.wslices + (size_t)rank * slice_words);
     uint4* dst = reinterpret_cast<uint4*>(s_w);
@@ -277,7 +281,15 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
             if (pick(u, j & 3) <= thr) {
               ++ltd_events;
               uint32_t* p = wcol + i * wpr;
-              if ((*p >> sh) & fmask) atomicSub(p, 1u << sh);   // other fields of the word may move concurrently
+              if (!wide) {
+                if ((*p >> sh) & fmask) atomicSub(p, 1u << sh);   // other fields of the word may move concurrently
+              } else {                                          // eq.(5) rounded (eq.(8), R27)
+                const int q0 = (int)((*p >> sh) & fmask);
+                const uint4 u2 = philox((uint32_t)t, (uint32_t)i, (uint32_t)(j >> 2), TAG_ROUND_LTD, seed);
+                const int dq = s_dbd[q0] + (pick(u2, j & 3) < s_dtd[q0] ? 1 : 0);
+                const int q1 = q0 - dq < 0 ? 0 : q0 - dq;
+                if (q1 != q0) atomicSub(p, (uint32_t)(q0 - q1) << sh);   // only this thread moves this field
+              }
             }
           }
         }
@@ -351,7 +363,15 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
                 if (pick(u, r) <= s_pot[D]) {
                   ++ltp_events;
                   const uint32_t word = *p;
-                  if (((word >> wsh) & fmask) < (uint32_t)qmax) *p = word + (1u << wsh);
+                  const int q0 = (int)((word >> wsh) & fmask);
+                  if (!wide) {
+                    if (q0 < qmax) *p = word + (1u << wsh);
+                  } else {                                  // eq.(4) rounded (eq.(8), R27)
+                    const uint4 u2 = philox((uint32_t)t, (uint32_t)Wg, (uint32_t)grp, TAG_ROUND, seed);
+                    const int dq = s_dbp[q0] + (pick(u2, r) < s_dtp[q0] ? 1 : 0);
+                    const int q1 = q0 + dq > qmax ? qmax : q0 + dq;
+                    *p = (word & ~(fmask << wsh)) | ((uint32_t)q1 << wsh);
+                  }
                 }
               } else {
                 const uint32_t word = *p;
@@ -489,22 +509,23 @@ __global__ void init_weights_kernel(const NetDesc d, unsigned long long init_see
   if (!word_coords(d, gid, r, i, w, col0, ncols)) return;
   const int cpw = 32 / d.bits;
   uint32_t word = 0;
-  for (int c4 = 0; c4 < cpw; c4 += 4) {
-    const int jl = w * cpw + c4;
+  for (int c = 0; c < cpw; ++c) {
+    const int jl = w * cpw + c;
     if (jl >= ncols) break;
     const int jg = d.col_base + col0 + jl;                  // global column (a shard starts at col_base)
     const uint4 u = philox((uint32_t)i, (uint32_t)(jg >> 2), 0u, TAG_INIT, init_seed);   // R4
-#pragma unroll
-    for (int l = 0; l < 4; ++l) {
-      if (jl + l >= ncols) break;
-      const uint32_t code = (uint32_t)(((unsigned long long)pick(u, l) * (unsigned long long)(d.q_max + 1)) >> 32);
-      word |= code << ((c4 + l) * d.bits);
-    }
+    const uint32_t code = (uint32_t)(((unsigned long long)pick(u, jg & 3) * (unsigned long long)(d.q_max + 1)) >> 32);
+    word |= code << (c * d.bits);
   }
   d.wslices[gid] = word;
 }
 
-__global__ void pack_weights_kernel(const NetDesc d, const uint8_t* __restrict__ codes) {
+// codes: one byte per code (bits <= 8) or one uint16 per code (bits = 16), row-major [i][j]
+__device__ __forceinline__ uint32_t code_at(const NetDesc& d, const void* codes, size_t k) {
+  return d.bits > 8 ? (uint32_t)static_cast<const uint16_t*>(codes)[k] : (uint32_t)static_cast<const uint8_t*>(codes)[k];
+}
+
+__global__ void pack_weights_kernel(const NetDesc d, const void* __restrict__ codes) {
   const size_t gid = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
   int r, i, w, col0, ncols;
   const int sw = slice_words_of(d);
@@ -515,12 +536,12 @@ __global__ void pack_weights_kernel(const NetDesc d, const uint8_t* __restrict__
   for (int c = 0; c < cpw; ++c) {
     const int jl = w * cpw + c;
     if (jl >= ncols) break;
-    word |= ((uint32_t)codes[(size_t)i * d.n_exc + col0 + jl] & ((1u << d.bits) - 1u)) << (c * d.bits);
+    word |= (code_at(d, codes, (size_t)i * d.n_exc + col0 + jl) & ((1u << d.bits) - 1u)) << (c * d.bits);
   }
   d.wslices[gid] = word;
 }
 
-__global__ void unpack_weights_kernel(const NetDesc d, uint8_t* __restrict__ codes) {
+__global__ void unpack_weights_kernel(const NetDesc d, void* __restrict__ codes) {
   const size_t gid = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
   int r, i, w, col0, ncols;
   if (!word_coords(d, gid, r, i, w, col0, ncols)) return;
@@ -529,13 +550,18 @@ __global__ void unpack_weights_kernel(const NetDesc d, uint8_t* __restrict__ cod
   for (int c = 0; c < cpw; ++c) {
     const int jl = w * cpw + c;
     if (jl >= ncols) break;
-    codes[(size_t)i * d.n_exc + col0 + jl] = (uint8_t)((word >> (c * d.bits)) & ((1u << d.bits) - 1u));
+    const uint32_t code = (word >> (c * d.bits)) & ((1u << d.bits) - 1u);
+    const size_t k = (size_t)i * d.n_exc + col0 + jl;
+    if (d.bits > 8) static_cast<uint16_t*>(codes)[k] = (uint16_t)code;
+    else static_cast<uint8_t*>(codes)[k] = (uint8_t)code;
   }
 }
 
-__global__ void check_codes_kernel(const uint8_t* __restrict__ codes, size_t n, int q_max, int* bad) {
+__global__ void check_codes_kernel(const void* __restrict__ codes, size_t n, int bits, int q_max, int* bad) {
   const size_t gid = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (gid < n && codes[gid] > q_max) atomicAdd(bad, 1);
+  if (gid >= n) return;
+  const int c = bits > 8 ? (int)static_cast<const uint16_t*>(codes)[gid] : (int)static_cast<const uint8_t*>(codes)[gid];
+  if (c > q_max) atomicAdd(bad, 1);
 }
 
 static unsigned grid_for(size_t n, int bs) { return (unsigned)((n + bs - 1) / bs); }
@@ -545,18 +571,18 @@ cudaError_t launch_init_weights(const NetDesc& d, uint64_t init_seed, cudaStream
   init_weights_kernel<<<grid_for(n, 256), 256, 0, s>>>(d, init_seed);
   return cudaGetLastError();
 }
-cudaError_t launch_pack_weights(const NetDesc& d, const uint8_t* codes, cudaStream_t s) {
+cudaError_t launch_pack_weights(const NetDesc& d, const void* codes, cudaStream_t s) {
   const size_t n = (size_t)d.cs * d.slice_words;
   pack_weights_kernel<<<grid_for(n, 256), 256, 0, s>>>(d, codes);
   return cudaGetLastError();
 }
-cudaError_t launch_unpack_weights(const NetDesc& d, uint8_t* codes, cudaStream_t s) {
+cudaError_t launch_unpack_weights(const NetDesc& d, void* codes, cudaStream_t s) {
   const size_t n = (size_t)d.cs * d.slice_words;
   unpack_weights_kernel<<<grid_for(n, 256), 256, 0, s>>>(d, codes);
   return cudaGetLastError();
 }
-cudaError_t launch_check_codes(const uint8_t* codes, size_t n, int q_max, int* bad, cudaStream_t s) {
-  check_codes_kernel<<<grid_for(n, 256), 256, 0, s>>>(codes, n, q_max, bad);
+cudaError_t launch_check_codes(const void* codes, size_t n, int bits, int q_max, int* bad, cudaStream_t s) {
+  check_codes_kernel<<<grid_for(n, 256), 256, 0, s>>>(codes, n, bits, q_max, bad);
   return cudaGetLastError();
 }
 

@@ -167,7 +167,7 @@ class Network:
         """shard=(rank, world): this object is shard `rank` of an n_exc-column network split over
         `world` ranks (include/snn.h snn_create_shard); self.n_exc becomes the shard's own columns."""
         self.n_in, self.n_exc, self.bits = n_in, n_exc, bits
-        self.params = params if params is not None else preset({2: "2b", 4: "4b", 8: "8b"}[bits])
+        self.params = params if params is not None else preset({2: "2b", 4: "4b", 8: "8b", 16: "16b"}[bits])
         for k, v in overrides.items():
             setattr(self.params, k, v)
         self._h = ctypes.c_void_p()
@@ -231,13 +231,17 @@ class Network:
                "snn_present_batch")
         self.last_T = T
 
+    @property
+    def code_dtype(self):
+        return np.uint16 if self.bits > 8 else np.uint8
+
     def weights(self) -> np.ndarray:
-        out = np.empty((self.n_in, self.n_exc), dtype=np.uint8)
+        out = np.empty((self.n_in, self.n_exc), dtype=self.code_dtype)
         _check(lib().snn_get_weights(self._h, _ptr(out), out.nbytes), "snn_get_weights")
         return out
 
     def set_weights(self, codes: np.ndarray):
-        c = np.ascontiguousarray(codes, dtype=np.uint8).reshape(self.n_in, self.n_exc)
+        c = np.ascontiguousarray(codes, dtype=self.code_dtype).reshape(self.n_in, self.n_exc)
         _check(lib().snn_set_weights(self._h, _ptr(c), c.nbytes), "snn_set_weights")
 
     def spikes(self) -> np.ndarray:
