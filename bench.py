@@ -363,9 +363,10 @@ def main():
     # FP32/INT issue: per column-step the LIF recipe is 7 lane-ops (I2F, FMUL, FADD, 3 FFMA, FSETP), per
     # synaptic event 1 integer add; peak = 148 SMs x 128 lanes x SM clock.
     inference = None
-    if ws == 1 and K == 1 and not args.no_infer:
+    if K == 1 and not args.no_infer and not sharded:
+        # data-parallel over ranks: every rank classifies its own image range with its own network
         nb = args.infer_images
-        iimgs = torch.from_numpy(synthdata.images(nb, "fashion", start=200000)).to(dev)
+        iimgs = torch.from_numpy(synthdata.images(nb, "fashion", start=200000 + rank * nb)).to(dev)
         iseeds = torch.from_numpy(synthdata.seeds(nb, base_seed=99).view(np.int64)).to(dev)
         icounts = torch.zeros((nb, N_EXC), dtype=torch.int32, device=dev)
         net.infer(iimgs, T_STEPS, iseeds, icounts, flags=P.SNN_ASYNC)
@@ -379,20 +380,29 @@ def main():
             e1.record(stream)
         torch.cuda.synchronize()
         ims = [a.elapsed_time(b) for a, b in iev]
-        ist = net.infer_stats() - st0
+        ist = (net.infer_stats() - st0).astype(np.float64)
         its = sum(ims) / 1e3
         n_inf = 3 * nb
+        if dist:                               # max-over-ranks device time, totals summed over ranks
+            t = torch.tensor([its], device=coll_dev, dtype=torch.float64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            its = float(t.item())
+            tot = torch.tensor([float(ist[0]), float(ist[1]), float(n_inf)], device=coll_dev, dtype=torch.float64)
+            dist.all_reduce(tot, op=dist.ReduceOp.SUM)
+            ist = np.array([tot[0].item(), tot[1].item()])
+            n_inf = int(tot[2].item())
         lane_ops = 7.0 * N_EXC * T_STEPS * n_inf + float(ist[0]) * N_EXC
         smclk_i = (clocks.get("sm_max_mhz") or 1965.0)
-        peak_ops = N_SM * 128 * smclk_i * 1e6 / 1e12
+        peak_ops = ws * N_SM * 128 * smclk_i * 1e6 / 1e12
         inference = {"metric": "inference images/s (learned weights frozen, P:88 labelling/inference protocol)",
-                     "value": n_inf / its, "unit": "images/s", "images_per_call": nb, "ms_per_call": sum(ims) / 3,
+                     "value": n_inf / its, "unit": "images/s", "images_per_call": nb, "ms_per_call": 1e3 * its / 3,
+                     "n_gpus": ws, "scaling": "weak",
                      "synaptic_events_per_s": float(ist[0]) * N_EXC / its,
                      "post_spikes_per_image": float(ist[1]) / n_inf,
                      "roofline": {"bound": "alu", "achieved": lane_ops / its / 1e12, "peak": peak_ops,
                                   "unit": "Tlane-op/s", "frac": lane_ops / its / 1e12 / peak_ops,
                                   "work": "7 lane-ops per column-step (LIF recipe) + 1 per synaptic event",
-                                  "peak_source": f"derived: 148 SMs x 128 FP32/INT lanes x {smclk_i:.0f} MHz"}}
+                                  "peak_source": f"derived: {ws} GPU(s) x 148 SMs x 128 FP32/INT lanes x {smclk_i:.0f} MHz"}}
 
     line = {
         "metric": METRIC, "value": value, "unit": "images/s", "n_gpus": ws, "steps": args.steps,
