@@ -147,6 +147,14 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
     for (int k = tid; k < slice_words / 4; k += nthr) dst[k] = src[k];
   }
   if (tid == 0) { s_flag[0] = INT_MAX; s_flag[1] = INT_MAX; }
+  // optional per-epoch trace (snn_set_trace; tools/trace_epochs.py): per epoch parity, the latest warp exit
+  // (%globaltimer), the longest warp speculation loop (cycles) and the deepest speculation (steps)
+  unsigned long long* trace = d.trace ? d.trace + (size_t)rank * d.trace_cap * 8 : nullptr;
+  unsigned long long* s_trmax = reinterpret_cast<unsigned long long*>(s_misc + 4);    // [2]
+  unsigned long long* s_trloop = reinterpret_cast<unsigned long long*>(s_misc + 8);   // [2]
+  int* s_trdepth = s_misc + 12;                                                      // [2]
+  if (tid == 0) { s_trmax[0] = s_trmax[1] = 0ull; s_trloop[0] = s_trloop[1] = 0ull; s_trdepth[0] = s_trdepth[1] = 0; }
+  unsigned long long tg0 = 0, tg3 = 0;
   int v[CPT], cnt[CPT], lpost[CPT];
 #pragma unroll
   for (int c = 0; c < CPT; ++c) {
@@ -249,6 +257,9 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
       const int kend = kb;
       const int fp = ep & 1;
       const uint32_t flag_addr = smem_u32(&s_flag[fp]);
+      const long long tl0 = trace ? clock64() : 0ll;
+      long long c_draw = 0, c_int = 0, c_ev = 0;          // trace: cycles in LTD draws, integration+LIF, LTD events
+      if (trace && tid == 0) tg0 = globaltimer();
 
       // ---------------------------------------------------------- speculation (warp-synchronous)
       int cnt0[CPT], v1[CPT], cnt1[CPT];
@@ -298,6 +309,27 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         }
       };
 
+      // LTD events of one step (rows [a0, a1) within the drawn window, <= 32 rows), applied in row order;
+      // events of steps after k0 are logged for a possible rollback (R14: old last_post, eq.(7))
+      auto ltd_apply = [&](int kstep, int a0, int a1) {
+#pragma unroll
+        for (int c = 0; c < CPT; ++c) {
+          if (!(dmask >> c & 1u)) continue;
+          uint32_t em = (a1 > a0) ? ((evm[c] >> (a0 - dr0)) & ((a1 - a0) == 32 ? FULL : ((1u << (a1 - a0)) - 1u))) : 0u;
+          const int shc = fsh + c * Z::LW;
+          while (em) {
+            const int xr = __ffs(em) - 1;
+            em &= em - 1;
+            const int i = (int)(s_rraw[a0 + xr] & 0xFFFFu);
+            uint32_t* pw = s_w + i * wpr + wj;
+            const bool applied = ((*pw >> shc) & FMASK) != 0u;
+            if (applied) atomicSub(pw, 1u << shc);     // lanes sharing the word may decrement concurrently
+            ++ltd_events;
+            if (kstep > k0) s_log[nlog++ * nthr + tid] = lean_log_entry(kstep - k0, c, applied, i);
+          }
+        }
+      };
+
 #ifdef SNN_LEAN_DEBUG
       long long dbg_it = 0;
 #endif
@@ -319,14 +351,42 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
 #pragma unroll
         for (int c = 0; c < CPT; ++c) live |= (valid >> c & 1u) && cnt[c] == 0;
         const bool wlive = __any_sync(FULL, live);
-        if (!wlive && wdirty == 0u) {                            // held warp: skip the run in O(1)
+        if (!wlive) {                                            // held warp: skip the run
           int mc = INT_MAX;
 #pragma unroll
           for (int c = 0; c < CPT; ++c) if (valid >> c & 1u) mc = min(mc, cnt[c]);
           mc = __reduce_min_sync(FULL, mc);
           int n = min(mc, kend - kk);
           if (fl != INT_MAX) n = min(n, fl - kk + 1);
-          if (kk == k0) {
+          bool stop = false;
+          if (wdirty) {
+            // LTD-active warp: nothing integrates during the run, so only its LTD events (in step order)
+            // remain -- applied here without the per-step machinery; a step of > 32 rows ends the run
+            // (the general path handles it), a full undo log stops the speculation before that step
+            const long long tq = trace ? clock64() : 0ll;
+            int m = 0;
+            for (; m < n; ++m) {
+              const int xs = kk + m - ka;
+              const int a0 = (int)s_offs[xs], a1 = (int)s_offs[xs + 1];
+              if (a1 - a0 > 32) break;                                               // warp-uniform
+              if (a0 < dr0 || a1 > dr0 + 32) { draw(a0); dr0 = a0; }
+              const uint32_t sm = (a1 > a0) ? (((a1 - a0) == 32 ? FULL : ((1u << (a1 - a0)) - 1u)) << (a0 - dr0)) : 0u;
+              int nev = 0;
+#pragma unroll
+              for (int c = 0; c < CPT; ++c) nev += __popc(evm[c] & sm);
+              const bool full = (kk + m) > k0 && nlog + nev > logn;
+              if (__any_sync(FULL, full)) {
+                if (full) hstep = kk + m;
+                stop = true;
+                break;
+              }
+              if (dmask) ltd_apply(kk + m, a0, a1);
+            }
+            n = m;
+            if (trace) c_ev += clock64() - tq;
+          }
+          if (n == 0 && !stop) goto general_step;                                  // a big step first
+          if (n > 0 && kk == k0) {
 #pragma unroll
             for (int c = 0; c < CPT; ++c) { v1[c] = v[c]; cnt1[c] = (valid >> c & 1u) ? cnt[c] - 1 : cnt[c]; }
           }
@@ -334,13 +394,20 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           for (int c = 0; c < CPT; ++c) if (valid >> c & 1u) cnt[c] -= n;
           kk += n;
           p_done = kk - 1;
+          if (stop) break;
           continue;
         }
+      general_step:
         // ---- this step's LTD events of the warp's LTD-active pairs (draws cover 32 rows ahead)
         const bool big = (o1 - o0) > 32;
         int nev = 0;
         if (wdirty) {
-          if (!big && (o0 < dr0 || o1 > dr0 + 32)) { draw(o0); dr0 = o0; }
+          if (!big && (o0 < dr0 || o1 > dr0 + 32)) {
+            const long long tq = trace ? clock64() : 0ll;
+            draw(o0);
+            dr0 = o0;
+            if (trace) c_draw += clock64() - tq;
+          }
           if (!big) {
             const uint32_t sm = (o1 > o0) ? (((o1 - o0) == 32 ? FULL : ((1u << (o1 - o0)) - 1u)) << (o0 - dr0)) : 0u;
 #pragma unroll
@@ -357,6 +424,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         }
         // ---- (a2) eq.(3) + (a3) eqs.(1)(2): integrate the step's rows, Euler step of live columns
         uint32_t cm = 0;
+        const long long tq_int = trace ? clock64() : 0ll;
         if (wlive) {
           int S[CPT];
 #pragma unroll
@@ -385,26 +453,13 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
 #pragma unroll
           for (int c = 0; c < CPT; ++c) if ((valid >> c & 1u) && cnt[c] > 0) --cnt[c];
         }
+        if (trace) c_int += clock64() - tq_int;
+        const long long tq_ev = trace ? clock64() : 0ll;
         // ---- (a5) LTD events of the step (old last_post, R14), applied in step order
         if (wdirty && dmask) {
           const int t = tbase + kk;
           if (!big) {
-#pragma unroll
-            for (int c = 0; c < CPT; ++c) {
-              if (!(dmask >> c & 1u)) continue;
-              uint32_t em = (o1 > o0) ? ((evm[c] >> (o0 - dr0)) & ((o1 - o0) == 32 ? FULL : ((1u << (o1 - o0)) - 1u))) : 0u;
-              const int shc = fsh + c * Z::LW;
-              while (em) {
-                const int xr = __ffs(em) - 1;
-                em &= em - 1;
-                const int i = (int)(s_rraw[o0 + xr] & 0xFFFFu);
-                uint32_t* pw = s_w + i * wpr + wj;
-                const bool applied = ((*pw >> shc) & FMASK) != 0u;
-                if (applied) atomicSub(pw, 1u << shc);
-                ++ltd_events;
-                if (kk > k0) s_log[nlog++ * nthr + tid] = lean_log_entry(kk - k0, c, applied, i);
-              }
-            }
+            ltd_apply(kk, o0, o1);
           } else {
             // steps with more than 32 active rows: the lane draws its own rows serially (rare)
 #pragma unroll
@@ -429,6 +484,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
             }
           }
         }
+        if (trace) c_ev += clock64() - tq_ev;
         if (kk == k0) {
 #pragma unroll
           for (int c = 0; c < CPT; ++c) { v1[c] = v[c]; cnt1[c] = cnt[c]; }
@@ -457,6 +513,14 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           if (r != rank) red_min_cluster(&s_flag[fp], (uint32_t)r, hstep - 1);
       }
       if (valid) eng_spec += (uint32_t)(p_done - k0 + 1) * (uint32_t)__popc(valid);
+      if (trace && lane == 0) {
+        atomicMax(&s_trmax[fp], globaltimer());
+        const unsigned long long f16 = 0xFFFFull;
+        const unsigned long long loop16 = min((unsigned long long)(clock64() - tl0) >> 4, f16);
+        atomicMax(&s_trloop[fp], (loop16 << 48) | (min((unsigned long long)c_draw >> 4, f16) << 32) |
+                                 (min((unsigned long long)c_ev >> 4, f16) << 16) | min((unsigned long long)c_int >> 4, f16));
+        atomicMax(&s_trdepth[fp], p_done - k0 + 1);
+      }
 
       // ---------------------------------------------------------- CTA summary -> cluster exchange
 #ifdef SNN_LEAN_DEBUG
@@ -494,6 +558,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         if (lane == 0) s_flag[fp ^ 1] = INT_MAX;
       }
       if (cs > 1) { cluster_arrive(); cluster_wait(); } else { __syncthreads(); }   // the one cross-SM exchange
+      if (trace && tid == 0) tg3 = globaltimer();
 
       // ---------------------------------------------------------- global decision
       int P, H;
@@ -629,6 +694,16 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           }
           __syncthreads();
         }
+      }
+      if (trace && tid == 0 && ep < d.trace_cap) {
+        unsigned long long* rec = trace + (size_t)ep * 8;
+        rec[0] = ((unsigned long long)b << 32) | (unsigned)k0;
+        rec[1] = ((unsigned long long)(event ? 1 : 2) << 32) | (unsigned)P;
+        rec[2] = tg0; rec[3] = s_trmax[fp]; rec[5] = tg3;
+        rec[4] = event ? (unsigned long long)(0xFFFFFFFFu - (uint32_t)K) : 0xFFFFFFFFull;   // winner column
+        rec[6] = s_trloop[fp];   // slowest warp: loop | draws | LTD events | integration+LIF (cycles / 16, 16 bits each)
+        rec[7] = globaltimer();
+        s_trmax[fp] = 0ull; s_trloop[fp] = 0ull; s_trdepth[fp] = 0;   // reused at epoch ep + 2 (after two barriers)
       }
       k0 = k_last + 1;
       ++ep;
