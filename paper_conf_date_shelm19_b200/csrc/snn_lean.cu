@@ -25,6 +25,13 @@
 
 namespace snn {
 
+// SNN_LEAN_TRACE_CYCLES=1 (compile time) adds the per-section cycle split of the slowest warp to the epoch
+// trace (tools/trace_lean.py); off by default, so the step loop carries no clock reads.
+#ifndef SNN_LEAN_TRACE_CYCLES
+#define SNN_LEAN_TRACE_CYCLES 0
+#endif
+constexpr bool kTraceCycles = SNN_LEAN_TRACE_CYCLES != 0;
+
 namespace {
 
 template <int BITS, int CPT_> struct LSwar {
@@ -363,7 +370,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
             // LTD-active warp: nothing integrates during the run, so only its LTD events (in step order)
             // remain -- applied here without the per-step machinery; a step of > 32 rows ends the run
             // (the general path handles it), a full undo log stops the speculation before that step
-            const long long tq = trace ? clock64() : 0ll;
+            const long long tq = (kTraceCycles && trace) ? clock64() : 0ll;
             int m = 0;
             for (; m < n; ++m) {
               const int xs = kk + m - ka;
@@ -383,7 +390,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
               if (dmask) ltd_apply(kk + m, a0, a1);
             }
             n = m;
-            if (trace) c_ev += clock64() - tq;
+            if (kTraceCycles && trace) c_ev += clock64() - tq;
           }
           if (n == 0 && !stop) goto general_step;                                  // a big step first
           if (n > 0 && kk == k0) {
@@ -403,10 +410,10 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         int nev = 0;
         if (wdirty) {
           if (!big && (o0 < dr0 || o1 > dr0 + 32)) {
-            const long long tq = trace ? clock64() : 0ll;
+            const long long tq = (kTraceCycles && trace) ? clock64() : 0ll;
             draw(o0);
             dr0 = o0;
-            if (trace) c_draw += clock64() - tq;
+            if (kTraceCycles && trace) c_draw += clock64() - tq;
           }
           if (!big) {
             const uint32_t sm = (o1 > o0) ? (((o1 - o0) == 32 ? FULL : ((1u << (o1 - o0)) - 1u)) << (o0 - dr0)) : 0u;
@@ -424,7 +431,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         }
         // ---- (a2) eq.(3) + (a3) eqs.(1)(2): integrate the step's rows, Euler step of live columns
         uint32_t cm = 0;
-        const long long tq_int = trace ? clock64() : 0ll;
+        const long long tq_int = (kTraceCycles && trace) ? clock64() : 0ll;
         if (wlive) {
           int S[CPT];
 #pragma unroll
@@ -453,8 +460,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
 #pragma unroll
           for (int c = 0; c < CPT; ++c) if ((valid >> c & 1u) && cnt[c] > 0) --cnt[c];
         }
-        if (trace) c_int += clock64() - tq_int;
-        const long long tq_ev = trace ? clock64() : 0ll;
+        if (kTraceCycles && trace) c_int += clock64() - tq_int;
+        const long long tq_ev = (kTraceCycles && trace) ? clock64() : 0ll;
         // ---- (a5) LTD events of the step (old last_post, R14), applied in step order
         if (wdirty && dmask) {
           const int t = tbase + kk;
@@ -484,7 +491,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
             }
           }
         }
-        if (trace) c_ev += clock64() - tq_ev;
+        if (kTraceCycles && trace) c_ev += clock64() - tq_ev;
         if (kk == k0) {
 #pragma unroll
           for (int c = 0; c < CPT; ++c) { v1[c] = v[c]; cnt1[c] = cnt[c]; }

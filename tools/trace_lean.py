@@ -1,5 +1,5 @@
 #!/usr/bin/env python
-"""Per-CTA speculation time of the lean event kernel (snn_set_trace records), split by the CTA's role in
+"""(Cycle split columns need the library built with -DSNN_LEAN_TRACE_CYCLES=1.)  Per-CTA speculation time of the lean event kernel (snn_set_trace records), split by the CTA's role in
 the epoch: the CTA that held the previous winner (LTP at the epoch start, LTD-active column), the CTA
 holding this epoch's winner, and the others.  Usage: python tools/trace_lean.py [--images 8]"""
 import argparse
