@@ -376,7 +376,12 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
               const int xs = kk + m - ka;
               const int a0 = (int)s_offs[xs], a1 = (int)s_offs[xs + 1];
               if (a1 - a0 > 32) break;                                               // warp-uniform
-              if (a0 < dr0 || a1 > dr0 + 32) { draw(a0); dr0 = a0; }
+              if (a0 < dr0 || a1 > dr0 + 32) {
+                const long long td = (kTraceCycles && trace) ? clock64() : 0ll;
+                draw(a0);
+                dr0 = a0;
+                if (kTraceCycles && trace) { c_draw += clock64() - td; c_ev -= clock64() - td; }
+              }
               const uint32_t sm = (a1 > a0) ? (((a1 - a0) == 32 ? FULL : ((1u << (a1 - a0)) - 1u)) << (a0 - dr0)) : 0u;
               int nev = 0;
 #pragma unroll
