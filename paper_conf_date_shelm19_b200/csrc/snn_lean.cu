@@ -446,10 +446,19 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           while (q < pe) {
             const int qe = min(pe, q + Z::CHUNK);
             uint32_t acc = 0u;
-            for (; q < qe; q += 4) {
+            for (; q + 4 < qe; q += 8) {         // two padded groups per trip: both offset loads in flight
+              const uint4 m = *reinterpret_cast<const uint4*>(s_prow + q);
+              const uint4 m2 = *reinterpret_cast<const uint4*>(s_prow + q + 4);
+              acc += ((wcol[m.x] >> fsh) & Z::LMASK) + ((wcol[m.y] >> fsh) & Z::LMASK) +
+                     ((wcol[m.z] >> fsh) & Z::LMASK) + ((wcol[m.w] >> fsh) & Z::LMASK);
+              acc += ((wcol[m2.x] >> fsh) & Z::LMASK) + ((wcol[m2.y] >> fsh) & Z::LMASK) +
+                     ((wcol[m2.z] >> fsh) & Z::LMASK) + ((wcol[m2.w] >> fsh) & Z::LMASK);
+            }
+            if (q < qe) {
               const uint4 m = *reinterpret_cast<const uint4*>(s_prow + q);
               acc += ((wcol[m.x] >> fsh) & Z::LMASK) + ((wcol[m.y] >> fsh) & Z::LMASK) +
                      ((wcol[m.z] >> fsh) & Z::LMASK) + ((wcol[m.w] >> fsh) & Z::LMASK);
+              q += 4;
             }
 #pragma unroll
             for (int c = 0; c < CPT; ++c)
