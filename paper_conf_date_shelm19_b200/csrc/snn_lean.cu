@@ -337,6 +337,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         }
       };
 
+      int fl_pf = __shfl_sync(FULL, ld_volatile_shared_u32addr(flag_addr), 0);   // early-stop flag, one step ahead
 #ifdef SNN_LEAN_DEBUG
       long long dbg_it = 0;
 #endif
@@ -350,10 +351,14 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
 #endif
         // one lane's read of the early-stop flag decides for the warp (lanes that executed the load apart
         // could otherwise see different values and leave the loop apart)
-        const int fl = __shfl_sync(FULL, ld_volatile_shared_u32addr(flag_addr), 0);
+        // (the value read here is used one step later: a flag lowered meanwhile only lets the warp run one
+        // step further, which the rollback at t* covers like any other step past t*)
+        const int fl = fl_pf;
+        fl_pf = __shfl_sync(FULL, ld_volatile_shared_u32addr(flag_addr), 0);
         if (kk >= kend || kk > fl) break;                        // warp-uniform
         const int x = kk - ka;
         const int o0 = (int)s_offs[x], o1 = (int)s_offs[x + 1];
+        const int ps = (int)s_pst[x], pe = (int)s_pst[x + 1];   // padded row range (integration below)
         bool live = false;
 #pragma unroll
         for (int c = 0; c < CPT; ++c) live |= (valid >> c & 1u) && cnt[c] == 0;
@@ -441,7 +446,6 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           int S[CPT];
 #pragma unroll
           for (int c = 0; c < CPT; ++c) S[c] = 0;
-          const int ps = (int)s_pst[x], pe = (int)s_pst[x + 1];
           int q = ps;
           while (q < pe) {
             const int qe = min(pe, q + Z::CHUNK);
