@@ -94,3 +94,28 @@ def test_16bit_rejections(gpu):
         g.infer(synthdata.images(1), 10, synthdata.seeds(1))
     with pytest.raises(P.SnnError):
         P.Network(784, 640, 16, P.preset("16b"), shard=(0, 2))
+
+
+def test_table2_grid_ensemble_mixed_widths(gpu):
+    """The Table II grid (precisions x rounding x rule) as ONE snn_present_many launch on the per-step
+    engine (same cluster shape for every width, 16-bit included): every network bit-exact with its oracle."""
+    import paper_conf_date_shelm19_b200 as P
+    rows = {2: "2b", 4: "4b", 8: "8b", 16: "16b"}
+    nets, oracles, imgs, seeds = [], [], [], []
+    k = 0
+    for bits in (2, 4, 8, 16):
+        for rounding in (0, 2):
+            for stdp in (0, 1):
+                p = O.params(rows[bits], stdp_mode=stdp, rounding=rounding, membrane_mode=1, init_seed=1 + k,
+                             cluster_size=4)
+                nets.append(P.Network(784, 128, bits, P.params_from_dict(p, engine=1)))
+                oracles.append(O.OracleNet(784, 128, bits, p))
+                imgs.append(synthdata.images(2, "mnist", start=20 * k))
+                seeds.append(synthdata.seeds(2, base_seed=300 + k))
+                k += 1
+    P.present_many(nets, imgs, 100, seeds)
+    for g, o, im, sd in zip(nets, oracles, imgs, seeds):
+        for x, s in zip(im, sd):
+            o.present(x, 100, int(s))
+        assert np.array_equal(g.weights(), o.weights())
+        assert np.array_equal(g.spikes(), o.spikes())
