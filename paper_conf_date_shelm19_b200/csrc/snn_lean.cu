@@ -277,6 +277,16 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
       for (int c = 0; c < CPT; ++c)
         if ((valid >> c & 1u) && lpost[c] >= 0 && (tbase + k0 - lpost[c]) < L_dep) dmask |= 1u << c;
       const uint32_t wdirty = __ballot_sync(FULL, dmask != 0);
+      // countdowns only run down during speculation (R6, R7), so the warp's first step with a live column is
+      // k0 + the smallest countdown of its valid columns (no per-step vote needed)
+      int live_from;
+      {
+        int mc0 = INT_MAX;
+#pragma unroll
+        for (int c = 0; c < CPT; ++c) if (valid >> c & 1u) mc0 = min(mc0, cnt[c]);
+        mc0 = __reduce_min_sync(FULL, mc0);
+        live_from = mc0 == INT_MAX ? INT_MAX : k0 + mc0;
+      }
       int kk = k0;
       int p_done = k0 - 1;           // last step fully processed by this thread
       int cstep = kNoStep;           // crossing step (the warp stops right after it)
@@ -359,16 +369,9 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         const int x = kk - ka;
         const int o0 = (int)s_offs[x], o1 = (int)s_offs[x + 1];
         const int ps = (int)s_pst[x], pe = (int)s_pst[x + 1];   // padded row range (integration below)
-        bool live = false;
-#pragma unroll
-        for (int c = 0; c < CPT; ++c) live |= (valid >> c & 1u) && cnt[c] == 0;
-        const bool wlive = __any_sync(FULL, live);
+        const bool wlive = kk >= live_from;                      // warp-uniform
         if (!wlive) {                                            // held warp: skip the run
-          int mc = INT_MAX;
-#pragma unroll
-          for (int c = 0; c < CPT; ++c) if (valid >> c & 1u) mc = min(mc, cnt[c]);
-          mc = __reduce_min_sync(FULL, mc);
-          int n = min(mc, kend - kk);
+          int n = min(live_from - kk, kend - kk);
           if (fl != INT_MAX) n = min(n, fl - kk + 1);
           bool stop = false;
           if (wdirty) {
