@@ -45,6 +45,24 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   while (!mbar_test(bar, parity)) {
   }
 }
+__device__ __forceinline__ uint32_t ld_acquire_cta(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.cta.shared.u32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_cta(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.cta.shared.u32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
+}
+// named barriers among the consumer warps (the producer warp never joins them)
+__device__ __forceinline__ int bar_red_or(int id, int n, bool pred) {
+  int r;
+  asm volatile("{\n .reg .pred p, q;\n setp.ne.u32 q, %1, 0;\n bar.red.or.pred p, %2, %3, q;\n selp.s32 %0, 1, 0, p;\n}\n"
+               : "=r"(r) : "r"((uint32_t)pred), "r"(id), "r"(n) : "memory");
+  return r;
+}
+__device__ __forceinline__ void bar_sync(int id, int n) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
 // TMA bulk copy global -> shared, completion signalled on `bar` (bytes % 16 == 0, 16-byte aligned)
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
@@ -85,6 +103,8 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
   unsigned long long* s_key = reinterpret_cast<unsigned long long*>(s_base + kSR);  // [32]
   int* s_cnt = reinterpret_cast<int*>(s_key + 32);                              // [32]
   uint32_t* s_wbuf = reinterpret_cast<uint32_t*>(s_cnt + 32);                   // [2][kWB][32] producer's word prefetch
+  uint32_t* s_pub = s_wbuf + 2 * kWB * 32;   // steps whose ring records the producer has published
+  uint32_t* s_rel = s_pub + 1;               // steps the consumers have finished (their ring slots are free)
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int ncw = (d.nthr_cols + 31) >> 5;        // consumer warps
@@ -98,9 +118,12 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
 
   if (tid == 0) {
     for (int r = 0; r < d.R; ++r) mbar_init(&full[r], 1);
+    *s_pub = 0u;
+    *s_rel = 0u;
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
+  const int ncons = ncw * 32;                     // consumer threads: they alone take part in the step barriers
 
   // ---------------- producer state (producer warp, uniform across its lanes)
   long long p_step = 0;       // next step to issue
@@ -205,10 +228,23 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
   unsigned long long act_sum = 0, spikes = 0;
 
   if (is_producer) {
+    // the producer runs decoupled from the consumers' step barriers: it publishes step records (release) and
+    // reuses ring slots of steps the consumers report finished (acquire)
     if (wfast) { prefetch_batch(); prefetch_batch(); }
-    produce(2, 0);                               // steps 0 and 1 before the first barrier
+    uint32_t rel = 0;
+    while (p_step < G) {
+      const long long before = p_step;
+      produce((long long)rel + kSR - 1, (long long)rel);
+      if (p_step != before) {
+        __syncwarp();
+        if (lane == 0) st_release_cta(s_pub, (uint32_t)p_step);
+      }
+      uint32_t r2 = ld_acquire_cta(s_rel);
+      while (r2 == rel && p_step == before && p_step < G) r2 = ld_acquire_cta(s_rel);   // ring full: wait
+      rel = __shfl_sync(FULL, r2, 0);
+    }
+    return;
   }
-  __syncthreads();
 
   uint32_t* counts_img = nullptr;
   int img = 0, t = 0;
@@ -234,6 +270,7 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
         if (j0 + 32 > d.n_exc) my_min_free = j0 >= d.n_exc ? 0xFFFF : 0;
       }
     }
+    while (ld_acquire_cta(s_pub) <= (uint32_t)g) {}     // the producer published step g
     const uint32_t nr = s_nrows[g & (kSR - 1)];
     if (consumer && (int)tt >= my_min_free) {
       if (!(nr & kDirect)) {
@@ -310,9 +347,9 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
       has_cand = ncand > 0;
     }
     if (tid == 0) act_sum += nr & ~kDirect;
-    // ---- B_g: the one barrier of a step; also releases the ring slots of step g
-    const int any = __syncthreads_or(has_cand);
-    if (is_producer) produce(g + kSR - 1, g + 1);     // records of steps >= g+2 become visible at B_{g+1}
+    // ---- B_g: the one barrier of a step (consumers only); then the ring slots of step g are released
+    const int any = bar_red_or(1, ncons, has_cand);
+    if (tid == 0) st_release_cta(s_rel, (uint32_t)(g + 1));
     if (any) {
       // WTA (R7): HARD -> the largest key wins; LAYER -> every candidate spikes
       unsigned long long wb = best;
@@ -324,7 +361,7 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
         wc += __shfl_xor_sync(FULL, wc, o);
       }
       if (lane == 0) { s_key[warp] = wb; s_cnt[warp] = wc; }
-      __syncthreads();
+      bar_sync(2, ncons);
       unsigned long long kbest = 0;
       int nsp = 0;
       for (int q = 0; q < ncw; ++q) {
@@ -332,7 +369,7 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
         kbest = y > kbest ? y : kbest;
         nsp += s_cnt[q];
       }
-      __syncthreads();                                   // s_key / s_cnt reusable
+      bar_sync(2, ncons);                                // s_key / s_cnt reusable
       const int W = (int)(0xFFFFFFFFu - (uint32_t)kbest);
       if (d.wta_mode == 0) nsp = 1;
       if (consumer) {
@@ -461,7 +498,7 @@ __global__ void __launch_bounds__(kVoteWarps * 32) classify_kernel(
 
 // ---------------------------------------------------------------- host side
 size_t infer_smem_bytes(int R, int row_bytes) {
-  return (size_t)R * row_bytes + (size_t)R * 8 + 2 * kSR * 4 + 32 * 8 + 32 * 4 + 2 * kWB * 32 * 4;
+  return (size_t)R * row_bytes + (size_t)R * 8 + 2 * kSR * 4 + 32 * 8 + 32 * 4 + 2 * kWB * 32 * 4 + 16;
 }
 
 template <int BITS, bool FIXED, int MINB>
