@@ -1104,7 +1104,8 @@ namespace {
 
 // Ring geometry of the inference kernel for this handle: the largest power-of-two ring (<= 64 rows)
 // (>= 32 rows) that leaves room for three CTAs per SM, else two, else one (>= 8 rows).  r01 sweep on
-// 784->6400 2-bit: R=32 / 3 CTAs 370k images/s, R=64 / 2 CTAs 333k, R=32 / 2 CTAs 329k, R=16 / 3 CTAs 125k.
+// 784->6400 2-bit (decoupled producer): R=32 / 3 CTAs 455k images/s, R=64 / 2 CTAs 401k, R=32 / 2 CTAs 401k,
+// R=16 / 3 CTAs 133k (steps beyond R/2 rows take the direct path).
 int infer_geometry(const snn_handle* h, int* wpr, int* R, int* nthr, size_t* smem) {
   const int ncols = (h->n_exc + 31) / 32;
   *wpr = ((ncols * h->bits) + 3) & ~3;
