@@ -1102,9 +1102,9 @@ int snn_get_info(const snn_handle* h, int64_t info[SNN_NINFO]) {
 // ---------------------------------------------------------------- NEXT-1: inference, labelling, vote
 namespace {
 
-// Ring geometry of the inference kernel for this handle: the largest power-of-two ring (<= 64 rows)
-// (>= 32 rows) that leaves room for three CTAs per SM, else two, else one (>= 8 rows).  r01 sweep on
-// 784->6400 2-bit (decoupled producer): R=32 / 3 CTAs 455k images/s, R=64 / 2 CTAs 401k, R=32 / 2 CTAs 401k,
+// Ring geometry of the inference kernel for this handle: the largest ring (multiple of 8, <= 64 rows;
+// >= 32 rows) that leaves room for three CTAs per SM, else two, else one (>= 8 rows).  r01 sweep on
+// 784->6400 2-bit (decoupled producer): R=40 / 3 CTAs 468k images/s, R=32 / 3 CTAs 448-455k, R=64 / 2 CTAs 401k,
 // R=16 / 3 CTAs 133k (steps beyond R/2 rows take the direct path).
 int infer_geometry(const snn_handle* h, int* wpr, int* R, int* nthr, size_t* smem) {
   const int ncols = (h->n_exc + 31) / 32;
@@ -1112,11 +1112,11 @@ int infer_geometry(const snn_handle* h, int* wpr, int* R, int* nthr, size_t* sme
   const int row_bytes = *wpr * 4;
   *nthr = (((ncols + 31) / 32) + 1) * 32;
   int r = 64;
-  if (const char* e = std::getenv("SNN_INFER_RING"))   // experiment hook: ring rows (power of two, 8..64)
-    if (std::atoi(e) >= 8 && std::atoi(e) <= 64 && !(std::atoi(e) & (std::atoi(e) - 1))) r = std::atoi(e);
-  while (r > 32 && snn::infer_smem_bytes(r, row_bytes) > 74 * 1024) r >>= 1;   // three CTAs per SM (measured best)
-  while (r > 8 && snn::infer_smem_bytes(r, row_bytes) > 110 * 1024) r >>= 1;
-  while (r > 8 && snn::infer_smem_bytes(r, row_bytes) > 220 * 1024) r >>= 1;
+  if (const char* e = std::getenv("SNN_INFER_RING"))   // experiment hook: ring rows (multiple of 8, 8..64)
+    if (std::atoi(e) >= 8 && std::atoi(e) <= 64 && !(std::atoi(e) & 7)) r = std::atoi(e);
+  while (r > 32 && snn::infer_smem_bytes(r, row_bytes) > 74 * 1024) r -= 8;    // three CTAs per SM (measured best)
+  while (r > 8 && snn::infer_smem_bytes(r, row_bytes) > 110 * 1024) r -= 8;
+  while (r > 8 && snn::infer_smem_bytes(r, row_bytes) > 220 * 1024) r -= 8;
   if (snn::infer_smem_bytes(r, row_bytes) > 220 * 1024) return fail(SNN_ESIZE, "inference ring does not fit");
   *R = r;
   *smem = snn::infer_smem_bytes(r, row_bytes);

@@ -110,8 +110,7 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
   const int ncw = (d.nthr_cols + 31) >> 5;        // consumer warps
   const bool is_producer = warp == ncw;
   const int T = d.T;
-  const uint32_t rmask = (uint32_t)d.R - 1u;      // R is a power of two: positions are u32 and wrap freely
-  const int rlog = __ffs(d.R) - 1;
+  const uint32_t Ru = (uint32_t)d.R;               // ring slots (any R in [8, 64]); positions are u32 per CTA
   const int my_images = d.n_images > (int)blockIdx.x ? (d.n_images - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
   const long long G = (long long)my_images * T;   // steps this CTA simulates (images back to back)
   if (G == 0) return;
@@ -196,8 +195,8 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
           while (bits) {                               // rows in ascending order, one bulk copy each
             const int i = 32 * w + __ffs(bits) - 1;
             bits &= bits - 1;
-            const uint32_t slot = (uint32_t)p & rmask;
-            if (p >= d.R) mbar_wait(&full[slot], (uint32_t)(((p >> rlog) - 1) & 1));   // previous use landed
+            const uint32_t pu = (uint32_t)p, use = pu / Ru, slot = pu - use * Ru;
+            if (p >= d.R) mbar_wait(&full[slot], (use - 1u) & 1u);                  // previous use landed
             mbar_arrive_tx(&full[slot], row_bytes);
             bulk_g2s(ring + (size_t)slot * row_bytes, d.w + (size_t)i * d.wpr, row_bytes, &full[slot]);
             ++p;
@@ -277,10 +276,12 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
         uint32_t acc[SW::NACC];
 #pragma unroll
         for (int a = 0; a < SW::NACC; ++a) acc[a] = 0;
-        uint32_t pos = s_base[g & (kSR - 1)];
-        for (uint32_t r = 0; r < nr; ++r, ++pos) {
-          const uint32_t slot = pos & rmask;
-          mbar_wait(&full[slot], (pos >> rlog) & 1u);
+        const uint32_t pos0 = s_base[g & (kSR - 1)];
+        uint32_t par = pos0 / Ru;
+        uint32_t slot = pos0 - par * Ru;
+        par &= 1u;
+        for (uint32_t r = 0; r < nr; ++r) {
+          mbar_wait(&full[slot], par);
           const uint32_t* src = reinterpret_cast<const uint32_t*>(ring + (size_t)slot * d.row_bytes) + tcol * BITS;
           uint32_t w[BITS];
           if constexpr (BITS == 2) {
@@ -294,6 +295,7 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
             }
           }
           SW::add(acc, w);
+          if (++slot == Ru) { slot = 0; par ^= 1u; }
         }
         // LIF (eqs.(1)(2)) of the non-held columns; keys only if some column crossed
         bool cross = false;
