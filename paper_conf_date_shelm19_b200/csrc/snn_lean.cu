@@ -277,6 +277,11 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
       for (int c = 0; c < CPT; ++c)
         if ((valid >> c & 1u) && lpost[c] >= 0 && (tbase + k0 - lpost[c]) < L_dep) dmask |= 1u << c;
       const uint32_t wdirty = __ballot_sync(FULL, dmask != 0);
+      // A packed word belongs to TPW consecutive lanes of one warp and, during speculation, only LTD writes
+      // codes (each lane its own fields).  When no two LTD-active lanes share a word, a lane's decrement is
+      // the only write to that word: a plain read-modify-write replaces the shared-memory atomic (-7 % time).
+      const uint32_t same_word = (TPW >= 32 ? FULL : ((1u << TPW) - 1u)) << (TPW >= 32 ? 0 : (lane & ~(TPW - 1)));
+      const bool ltd_plain = !__any_sync(FULL, dmask != 0 && __popc(same_word & wdirty) > 1);
       // countdowns only run down during speculation (R6, R7), so the warp's first step with a live column is
       // k0 + the smallest countdown of its valid columns (no per-step vote needed)
       int live_from;
@@ -334,15 +339,29 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           if (!(dmask >> c & 1u)) continue;
           uint32_t em = (a1 > a0) ? ((evm[c] >> (a0 - dr0)) & ((a1 - a0) == 32 ? FULL : ((1u << (a1 - a0)) - 1u))) : 0u;
           const int shc = fsh + c * Z::LW;
-          while (em) {
-            const int xr = __ffs(em) - 1;
-            em &= em - 1;
-            const int i = (int)(s_rraw[a0 + xr] & 0xFFFFu);
-            uint32_t* pw = s_w + i * wpr + wj;
-            const bool applied = ((*pw >> shc) & FMASK) != 0u;
-            if (applied) atomicSub(pw, 1u << shc);     // lanes sharing the word may decrement concurrently
-            ++ltd_events;
-            if (kstep > k0) s_log[nlog++ * nthr + tid] = lean_log_entry(kstep - k0, c, applied, i);
+          if (ltd_plain) {                             // warp-uniform: this lane is the only writer of its words
+            while (em) {
+              const int xr = __ffs(em) - 1;
+              em &= em - 1;
+              const int i = (int)(s_rraw[a0 + xr] & 0xFFFFu);
+              uint32_t* pw = s_w + i * wpr + wj;
+              const uint32_t wv = *pw;
+              const bool applied = ((wv >> shc) & FMASK) != 0u;
+              if (applied) *pw = wv - (1u << shc);
+              ++ltd_events;
+              if (kstep > k0) s_log[nlog++ * nthr + tid] = lean_log_entry(kstep - k0, c, applied, i);
+            }
+          } else {                                     // another LTD-active lane shares a word: atomics
+            while (em) {
+              const int xr = __ffs(em) - 1;
+              em &= em - 1;
+              const int i = (int)(s_rraw[a0 + xr] & 0xFFFFu);
+              uint32_t* pw = s_w + i * wpr + wj;
+              const bool applied = ((*pw >> shc) & FMASK) != 0u;
+              if (applied) atomicSub(pw, 1u << shc);
+              ++ltd_events;
+              if (kstep > k0) s_log[nlog++ * nthr + tid] = lean_log_entry(kstep - k0, c, applied, i);
+            }
           }
         }
       };
