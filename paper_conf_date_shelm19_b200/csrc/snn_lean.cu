@@ -734,8 +734,9 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
               ++ltp_trials;
               if (pick(u, r) <= s_pot[D]) {
                 ++ltp_events;
-                uint32_t* pw = s_w + i * wpr + ww;
-                if (((*pw >> wsh) & FMASK) < (uint32_t)qmax) atomicAdd(pw, 1u << wsh);
+                uint32_t* pw = s_w + i * wpr + ww;              // row i is this thread's alone during LTP
+                const uint32_t wv = *pw;
+                if (((wv >> wsh) & FMASK) < (uint32_t)qmax) *pw = wv + (1u << wsh);
               }
             }
           }
