@@ -419,7 +419,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
                 stop = true;
                 break;
               }
-              if (dmask) ltd_apply(kk + m, a0, a1);
+              if (nev) ltd_apply(kk + m, a0, a1);                    // this lane has events in the step
             }
             n = m;
             if (kTraceCycles && trace) c_ev += clock64() - tq;
@@ -506,7 +506,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         if (wdirty && dmask) {
           const int t = tbase + kk;
           if (!big) {
-            ltd_apply(kk, o0, o1);
+            if (nev) ltd_apply(kk, o0, o1);                      // this lane has events in the step
           } else {
             // steps with more than 32 active rows: the lane draws its own rows serially (rare)
 #pragma unroll
