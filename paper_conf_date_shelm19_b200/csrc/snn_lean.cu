@@ -45,6 +45,8 @@ template <int BITS, int CPT_> struct LSwar {
   static constexpr int CHUNK = CPT_ == 1 ? (1 << 28) : (int)((((1u << (LW & 31)) - 1u) / FM) & ~3u);
 };
 
+constexpr int kDrawRows = 64;        // raw rows one LTD draw covers (two Philox blocks per lane, in flight together)
+
 struct LeanLayout {
   size_t slots, wsum, flags, misc, w, pot, dep, lpre, offs, pst, prow, rraw, log, total;
 };
@@ -64,7 +66,7 @@ __host__ __device__ inline LeanLayout lean_layout(int n_in, int slice_words, int
   L.offs = o;  o = align16(o + (size_t)(offs_cap + 1) * 4);          // raw row offset of every window step
   L.pst = o;   o = align16(o + (size_t)(offs_cap + 1) * 4);          // padded (x4) start of every window step
   L.prow = o;  o = align16(o + (size_t)(rows_cap + 3 * offs_cap + 4) * 4);   // padded word offsets row*wpr
-  L.rraw = o;  o = align16(o + (size_t)(rows_cap + 32) * 4);         // raw rows: step << 16 | row id
+  L.rraw = o;  o = align16(o + (size_t)(rows_cap + kDrawRows) * 4);         // raw rows: step << 16 | row id
   L.log = o;   o = align16(o + (size_t)logn * nthr * 4);
   L.total = o;
   return L;
@@ -258,7 +260,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           }
           for (uint32_t q = p0 + (o1 - o0); q < p1; ++q) s_prow[q] = zero_off;
         }
-        for (int x = tid; x < 32; x += nthr) s_rraw[nrows + x] = 0xFFFF0000u;   // draw pads (never an event)
+        for (int x = tid; x < kDrawRows; x += nthr) s_rraw[nrows + x] = 0xFFFF0000u;   // draw pads (never an event)
         __syncthreads();
       }
       const int kend = kb;
@@ -298,17 +300,25 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
       int hstep = kNoStep;           // undo log full: stopped before this step
       unsigned long long ckey = 0ull;
       int nlog = 0;
-      int dr0 = INT_MIN;             // warp-uniform raw start of the drawn LTD row range [dr0, dr0 + 32)
-      uint32_t evm[CPT];
+      int dr0 = INT_MIN;             // warp-uniform raw start of the drawn LTD row range [dr0, dr0 + kDrawRows)
+      unsigned long long evm[CPT];   // LTD event bits of raw rows [dr0, dr0 + 64) (owning lane)
 #pragma unroll
-      for (int c = 0; c < CPT; ++c) evm[c] = 0u;
+      for (int c = 0; c < CPT; ++c) evm[c] = 0ull;
+      // event bits of column slot c for raw rows [a0, a1) (a1 - a0 <= 32, inside the drawn range)
+      auto evbits = [&](int c, int a0, int a1) -> uint32_t {
+        const int nr = a1 - a0;
+        return nr <= 0 ? 0u : ((uint32_t)(evm[c] >> (a0 - dr0)) & (nr >= 32 ? FULL : ((1u << nr) - 1u)));
+      };
 
-      // LTD draws of every (lane, column) pair of the warp for raw rows [base, base + 32): lanes over rows
+      // LTD draws of every (lane, column) pair of the warp for raw rows [base, base + 64): lanes over rows,
+      // two rows per lane whose Philox blocks are independent (one chain's latency for 64 rows)
       auto draw = [&](int base) {
-        const uint32_t rr = s_rraw[base + lane];
-        const int t = tbase + ka + (int)(rr >> 16);
-        const uint32_t i = rr & 0xFFFFu;
-        const bool ok = (rr >> 16) != 0xFFFFu && base + lane < (int)s_offs[kend - ka];
+        const uint32_t rr0 = s_rraw[base + lane], rr1 = s_rraw[base + 32 + lane];
+        const int nrw = (int)s_offs[kend - ka];
+        const int t0 = tbase + ka + (int)(rr0 >> 16), t1 = tbase + ka + (int)(rr1 >> 16);
+        const uint32_t i0 = rr0 & 0xFFFFu, i1 = rr1 & 0xFFFFu;
+        const bool ok0 = (rr0 >> 16) != 0xFFFFu && base + lane < nrw;
+        const bool ok1 = (rr1 >> 16) != 0xFFFFu && base + 32 + lane < nrw;
 #pragma unroll 1
         for (uint32_t lm = wdirty; lm; lm &= lm - 1) {
           const int Ls = __ffs(lm) - 1;
@@ -319,14 +329,14 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
             const int jl = __shfl_sync(FULL, jcol[c], Ls);
             const int lp = __shfl_sync(FULL, lpost[c], Ls);
             const int jg = cbase + col0 + jl;
-            const int D = t - lp;
-            bool bit = false;
-            if (ok && D < L_dep) {
-              const uint4 u = philox((uint32_t)t, i, (uint32_t)(jg >> 2), TAG_LTD, seed);   // eq.(7), R13
-              bit = pick(u, jg & 3) <= s_dep[D];
-            }
-            const uint32_t m = __ballot_sync(FULL, bit);
-            if (lane == Ls) evm[c] = m;
+            const int D0 = t0 - lp, D1 = t1 - lp;
+            const uint4 u0 = philox((uint32_t)t0, i0, (uint32_t)(jg >> 2), TAG_LTD, seed);   // eq.(7), R13
+            const uint4 u1 = philox((uint32_t)t1, i1, (uint32_t)(jg >> 2), TAG_LTD, seed);
+            const bool in0 = ok0 && D0 < L_dep, in1 = ok1 && D1 < L_dep;
+            const bool bit0 = in0 && pick(u0, jg & 3) <= s_dep[in0 ? D0 : 0];
+            const bool bit1 = in1 && pick(u1, jg & 3) <= s_dep[in1 ? D1 : 0];
+            const uint32_t m0 = __ballot_sync(FULL, bit0), m1 = __ballot_sync(FULL, bit1);
+            if (lane == Ls) evm[c] = ((unsigned long long)m1 << 32) | m0;
           }
         }
       };
@@ -337,7 +347,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
 #pragma unroll
         for (int c = 0; c < CPT; ++c) {
           if (!(dmask >> c & 1u)) continue;
-          uint32_t em = (a1 > a0) ? ((evm[c] >> (a0 - dr0)) & ((a1 - a0) == 32 ? FULL : ((1u << (a1 - a0)) - 1u))) : 0u;
+          uint32_t em = evbits(c, a0, a1);
           const int shc = fsh + c * Z::LW;
           if (ltd_plain) {                             // warp-uniform: this lane is the only writer of its words
             while (em) {
@@ -403,16 +413,15 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
               const int xs = kk + m - ka;
               const int a0 = (int)s_offs[xs], a1 = (int)s_offs[xs + 1];
               if (a1 - a0 > 32) break;                                               // warp-uniform
-              if (a0 < dr0 || a1 > dr0 + 32) {
+              if (a0 < dr0 || a1 > dr0 + kDrawRows) {
                 const long long td = (kTraceCycles && trace) ? clock64() : 0ll;
                 draw(a0);
                 dr0 = a0;
                 if (kTraceCycles && trace) { c_draw += clock64() - td; c_ev -= clock64() - td; }
               }
-              const uint32_t sm = (a1 > a0) ? (((a1 - a0) == 32 ? FULL : ((1u << (a1 - a0)) - 1u)) << (a0 - dr0)) : 0u;
               int nev = 0;
 #pragma unroll
-              for (int c = 0; c < CPT; ++c) nev += __popc(evm[c] & sm);
+              for (int c = 0; c < CPT; ++c) nev += __popc(evbits(c, a0, a1));
               const bool full = (kk + m) > k0 && nlog + nev > logn;
               if (__any_sync(FULL, full)) {
                 if (full) hstep = kk + m;
@@ -441,16 +450,15 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         const bool big = (o1 - o0) > 32;
         int nev = 0;
         if (wdirty) {
-          if (!big && (o0 < dr0 || o1 > dr0 + 32)) {
+          if (!big && (o0 < dr0 || o1 > dr0 + kDrawRows)) {
             const long long tq = (kTraceCycles && trace) ? clock64() : 0ll;
             draw(o0);
             dr0 = o0;
             if (kTraceCycles && trace) c_draw += clock64() - tq;
           }
           if (!big) {
-            const uint32_t sm = (o1 > o0) ? (((o1 - o0) == 32 ? FULL : ((1u << (o1 - o0)) - 1u)) << (o0 - dr0)) : 0u;
 #pragma unroll
-            for (int c = 0; c < CPT; ++c) nev += __popc(evm[c] & sm);
+            for (int c = 0; c < CPT; ++c) nev += __popc(evbits(c, o0, o1));
           } else {
             nev = __popc(dmask) * (o1 - o0);                     // conservative bound (steps of > 32 rows)
           }
