@@ -48,7 +48,7 @@ template <int BITS, int CPT_> struct LSwar {
 constexpr int kDrawRows = 64;        // raw rows one LTD draw covers (two Philox blocks per lane, in flight together)
 
 struct LeanLayout {
-  size_t slots, wsum, flags, misc, w, pot, dep, lpre, offs, pst, prow, rraw, log, total;
+  size_t slots, wsum, flags, misc, pd, w, pot, dep, lpre, offs, pst, prow, rraw, log, total;
 };
 
 __host__ __device__ inline LeanLayout lean_layout(int n_in, int slice_words, int L_pot, int L_dep, int nthr,
@@ -59,6 +59,7 @@ __host__ __device__ inline LeanLayout lean_layout(int n_in, int slice_words, int
   L.wsum = o;  o = align16(o + 32 * 2 * 8);                  // per warp: steps, key
   L.flags = o; o = align16(o + 4 * 4);                       // early-stop flag per epoch parity
   L.misc = o;  o = align16(o + 16 * 4);
+  L.pd = o;    o = align16(o + (size_t)(nthr / 32 + 1) * 4);          // winner's pre-drawn LTD bits, per warp
   L.w = o;     o = align16(o + (size_t)slice_words * 4);
   L.pot = o;   o = align16(o + (size_t)(L_pot > 0 ? L_pot : 1) * 4);
   L.dep = o;   o = align16(o + (size_t)(L_dep > 0 ? L_dep : 1) * 4);
@@ -119,6 +120,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
   uint32_t* s_prow = reinterpret_cast<uint32_t*>(smem + L.prow);
   uint32_t* s_rraw = reinterpret_cast<uint32_t*>(smem + L.rraw);
   uint32_t* s_log = reinterpret_cast<uint32_t*>(smem + L.log);
+  uint32_t* s_pd = reinterpret_cast<uint32_t*>(smem + L.pd);
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwarps = nthr >> 5;
   const int g0 = (rank * d.ngroups) / cs, g1 = ((rank + 1) * d.ngroups) / cs;
@@ -195,6 +197,9 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
     int ka = 0, kb = 0;            // window steps [ka, kb)
     int lpre_upto = -1;            // s_lpre holds the input spike timers through window step lpre_upto
     int k0 = 0;
+    // LTD draws of the last winner of this CTA (local column Wpd) for raw rows [pd0, pd0 + nthr) of the window,
+    // taken by the whole CTA next to its LTP (s_pd); INT_MIN: none
+    int Wpd = INT_MIN, pd0 = 0;
     if (rank == 0 && tid == 0 && T > 0) act_sum += (unsigned long long)(offs_g[T] - offs_g[0]);
     __syncthreads();
 
@@ -218,6 +223,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         __syncthreads();
         ka = k0;
         lpre_upto = -1;
+        Wpd = INT_MIN;                                 // raw row numbering changes
         const int n_o = min(offs_cap, T - ka);
         const uint32_t wbase = offs_g[ka];
         for (int x = tid; x <= n_o; x += nthr) s_offs[x] = offs_g[ka + x] - wbase;
@@ -327,6 +333,13 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           for (int c = 0; c < CPT; ++c) {
             if (!(dm >> c & 1u)) continue;                 // warp-uniform
             const int jl = __shfl_sync(FULL, jcol[c], Ls);
+            if (jl == Wpd && base >= pd0 && base + 64 <= pd0 + nthr) {   // warp-uniform: drawn by the CTA
+              const int o = base - pd0, w = o >> 5, sh = o & 31;
+              const uint32_t p0 = s_pd[w], p1 = s_pd[w + 1], p2 = s_pd[w + 2 <= nwarps ? w + 2 : nwarps];
+              if (lane == Ls)
+                evm[c] = ((unsigned long long)__funnelshift_r(p1, p2, sh) << 32) | __funnelshift_r(p0, p1, sh);
+              continue;
+            }
             const int lp = __shfl_sync(FULL, lpost[c], Ls);
             const int jg = cbase + col0 + jl;
             const int D0 = t0 - lp, D1 = t1 - lp;
@@ -729,6 +742,19 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           __syncthreads();
           const int Wg = cbase + col0 + Wl;
           const int ww = Wl / CPW, wsh = (Wl % CPW) * BITS;
+          // the winner's eq.(7) LTD draws (last_post = t*) for the next raw rows, one per thread, in flight with
+          // the LTP draws below: the winner's warp then finds them in s_pd instead of drawing them itself
+          const bool pd_ok = P + 1 < kend;                                     // CTA-uniform: same window
+          const int pr0 = pd_ok ? (int)s_offs[P + 1 - ka] : 0;
+          const int nrw = (int)s_offs[kend - ka];
+          bool pbit = false;
+          if (pd_ok && pr0 + tid < nrw) {
+            const uint32_t rr = s_rraw[pr0 + tid];
+            const int t = tbase + ka + (int)(rr >> 16);
+            const int D = t - tP;
+            const uint4 u = philox((uint32_t)t, rr & 0xFFFFu, (uint32_t)(Wg >> 2), TAG_LTD, seed);
+            pbit = D < L_dep && pick(u, Wg & 3) <= s_dep[D < L_dep ? D : 0];
+          }
           for (int grp = tid; grp < nq4; grp += nthr) {
             const uint4 u = philox((uint32_t)tP, (uint32_t)Wg, (uint32_t)grp, TAG_LTP, seed);
 #pragma unroll
@@ -746,6 +772,16 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
                 const uint32_t wv = *pw;
                 if (((wv >> wsh) & FMASK) < (uint32_t)qmax) *pw = wv + (1u << wsh);
               }
+            }
+          }
+          {
+            const uint32_t m = __ballot_sync(FULL, pbit);
+            if (pd_ok) {
+              if (lane == 0) s_pd[warp] = m;
+              if (tid == 0) s_pd[nwarps] = 0u;
+              Wpd = Wl; pd0 = pr0;
+            } else {
+              Wpd = INT_MIN;
             }
           }
           __syncthreads();
