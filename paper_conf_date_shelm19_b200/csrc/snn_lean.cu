@@ -737,7 +737,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         for (int c = 0; c < CPT; ++c)
           if ((valid >> c & 1u) && jcol[c] == Wl) lpost[c] = tP;             // after LTD at t* (R14)
         if (Wl >= 0 && Wl < ncols) {                                           // CTA-uniform
-          __syncthreads();
+          // (no barrier before the catch-up: it reads only the staged window and writes only s_lpre, which
+          // nothing reads before the barrier below; the undo above and the LTP below are still separated by it)
           lpre_catch_up(P - ka);                                               // last_pre includes step t*
           __syncthreads();
           const int Wg = cbase + col0 + Wl;
