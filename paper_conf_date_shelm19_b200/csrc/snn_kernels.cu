@@ -129,6 +129,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
   }
   uint32_t ltd_trials = 0, ltd_events = 0, ltp_trials = 0, ltp_events = 0;
   unsigned long long act_sum = 0, post_sum = 0;
+  // every CTA of the cluster must have started before another addresses its shared memory (DSMEM stores below)
+  if (cs > 1) { cluster_arrive(); cluster_wait(); } else { __syncthreads(); }
 
   for (int b = 0; b < d.n_images; ++b) {
     const unsigned long long seed = d.seeds[b];

@@ -13,7 +13,14 @@
 //     summing the thread's CPT columns in SWAR lanes (eq.(3)); held (refractory / inhibited) warps skip
 //     whole runs of steps in O(1);
 //   * LTP of the winner (eq.(6)) needs last_pre only in the winner's CTA: the input spike timers are
-//     brought up to date lazily there, and nowhere else.
+//     brought up to date lazily there, and nowhere else;
+//   * the last winner of each CTA is its *deferred* column: it is LTD-active on every input spike right after
+//     its post spike (eq.(7) with small |Dt|) and used to put the longest dependent chain on one warp.  Its LTD
+//     events for the next <= 2*nthr raw rows (<= 64 steps) are drawn by the whole CTA at once, and with them its
+//     integration sums S(t) = sum_{i active at t} max(q_i - n_i(<t), 0) (n_i(<t): its events on row i at earlier
+//     table steps -- decrements clamped at 0 commute), so the owning thread reads S(t) from a table and
+//     applies no LTD in the step loop; the events of the committed steps are written back by the CTA when the
+//     table is retired (a new winner in the CTA, a rebuild, a window or image boundary).
 // Results are bit-identical to the oracle (tests/test_gpu_parity.py runs every case on this kernel and
 // on the general one).
 #include "snn_internal.h"
@@ -46,9 +53,11 @@ template <int BITS, int CPT_> struct LSwar {
 };
 
 constexpr int kDrawRows = 64;        // raw rows one LTD draw covers (two Philox blocks per lane, in flight together)
+constexpr int kDefSteps = 64;        // steps one deferred-LTD table covers at most (u64 step masks per input row)
+constexpr int kDefMargin = 16;       // a table with fewer steps left than this is rebuilt at the epoch start
 
 struct LeanLayout {
-  size_t slots, wsum, flags, misc, pd, w, pot, dep, lpre, offs, pst, prow, rraw, log, total;
+  size_t slots, wsum, flags, misc, dS, dbits, dev, w, pot, dep, lpre, offs, pst, prow, rraw, log, total;
 };
 
 __host__ __device__ inline LeanLayout lean_layout(int n_in, int slice_words, int L_pot, int L_dep, int nthr,
@@ -59,7 +68,9 @@ __host__ __device__ inline LeanLayout lean_layout(int n_in, int slice_words, int
   L.wsum = o;  o = align16(o + 32 * 2 * 8);                  // per warp: steps, key
   L.flags = o; o = align16(o + 4 * 4);                       // early-stop flag per epoch parity
   L.misc = o;  o = align16(o + 16 * 4);
-  L.pd = o;    o = align16(o + (size_t)(nthr / 32 + 1) * 4);          // winner's pre-drawn LTD bits, per warp
+  L.dS = o;    o = align16(o + (size_t)kDefSteps * 4);                // deferred column: S per table step
+  L.dbits = o; o = align16(o + (size_t)(2 * nthr / 32) * 4);          // deferred column: event bit per raw row
+  L.dev = o;   o = align16(o + (size_t)n_in * 8);                     // deferred column: event steps per input row
   L.w = o;     o = align16(o + (size_t)slice_words * 4);
   L.pot = o;   o = align16(o + (size_t)(L_pot > 0 ? L_pot : 1) * 4);
   L.dep = o;   o = align16(o + (size_t)(L_dep > 0 ? L_dep : 1) * 4);
@@ -120,7 +131,9 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
   uint32_t* s_prow = reinterpret_cast<uint32_t*>(smem + L.prow);
   uint32_t* s_rraw = reinterpret_cast<uint32_t*>(smem + L.rraw);
   uint32_t* s_log = reinterpret_cast<uint32_t*>(smem + L.log);
-  uint32_t* s_pd = reinterpret_cast<uint32_t*>(smem + L.pd);
+  int* s_dS = reinterpret_cast<int*>(smem + L.dS);
+  uint32_t* s_dbits = reinterpret_cast<uint32_t*>(smem + L.dbits);
+  unsigned long long* s_dev = reinterpret_cast<unsigned long long*>(smem + L.dev);
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwarps = nthr >> 5;
   const int g0 = (rank * d.ngroups) / cs, g1 = ((rank + 1) * d.ngroups) / cs;
@@ -158,6 +171,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
     for (int k = tid; k < slice_words / 4; k += nthr) dst[k] = src[k];
   }
   if (tid == 0) { s_flag[0] = INT_MAX; s_flag[1] = INT_MAX; }
+  for (int i = tid; i < n_in; i += nthr) s_dev[i] = 0ull;
   // optional per-epoch trace (snn_set_trace; tools/trace_epochs.py): per epoch parity, the latest warp exit
   // (%globaltimer), the longest warp speculation loop (cycles) and the deepest speculation (steps)
   unsigned long long* trace = d.trace ? d.trace + (size_t)rank * d.trace_cap * 8 : nullptr;
@@ -196,10 +210,12 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
     int img_spikes = 0;
     int ka = 0, kb = 0;            // window steps [ka, kb)
     int lpre_upto = -1;            // s_lpre holds the input spike timers through window step lpre_upto
+    int kend_w = 0;                // window end (kb) as seen by the deferred-table helpers
     int k0 = 0;
-    // LTD draws of the last winner of this CTA (local column Wpd) for raw rows [pd0, pd0 + nthr) of the window,
-    // taken by the whole CTA next to its LTP (s_pd); INT_MIN: none
-    int Wpd = INT_MIN, pd0 = 0;
+    // the CTA's deferred column (its last winner, local index Wd; -1 none) and its LTD table: steps [tk0, kcov],
+    // raw rows [tr0, tr0 + tnr) of the window; d_lp = its last post spike (absolute step).  CTA-uniform.
+    int Wd = -1, d_lp = 0, tk0 = 0, kcov = -1, tr0 = 0, tnr = 0;
+    bool tvalid = false;
     if (rank == 0 && tid == 0 && T > 0) act_sum += (unsigned long long)(offs_g[T] - offs_g[0]);
     __syncthreads();
 
@@ -215,15 +231,94 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
       }
     };
 
+    // ---- deferred column (CTA-cooperative; every thread calls these at the same point, arguments CTA-uniform)
+    // retire the table: write back the deferred column's eq.(7) events of the table steps <= kc (decrements of one
+    // row clamp at 0, so their total is applied at once by the thread holding the row's first event), count them
+    // and their trials (R20), clear the per-row event masks
+    auto dtab_commit = [&](int kc) {
+      const int ww = Wd / CPW, wsh = (Wd % CPW) * BITS;
+      const int relc = kc - tk0;
+      for (int r = tid; r < tnr; r += nthr) {
+        const uint32_t rr = s_rraw[tr0 + r];
+        const int k = ka + (int)(rr >> 16);
+        if (k > kc) continue;
+        const int i = (int)(rr & 0xFFFFu);
+        if (tbase + k - d_lp < L_dep) ++ltd_trials;
+        if (!((s_dbits[r >> 5] >> (r & 31)) & 1u)) continue;
+        ++ltd_events;
+        const unsigned long long m = s_dev[i];
+        if (__popcll(m & ((1ull << (k - tk0)) - 1ull)) != 0) continue;    // not the row's first event
+        const int n = __popcll(relc >= 63 ? m : (m & ((2ull << relc) - 1ull)));
+        // the column's field of row i is this thread's alone (other fields may be in an undo: atomic)
+        uint32_t* pw = s_w + i * wpr + ww;
+        const int dec = min(n, (int)((*pw >> wsh) & FMASK));
+        if (dec) atomicSub(pw, (uint32_t)dec << wsh);
+      }
+      __syncthreads();
+      for (int r = tid; r < tnr; r += nthr) s_dev[s_rraw[tr0 + r] & 0xFFFFu] = 0ull;
+      __syncthreads();
+      tvalid = false;
+    };
+    // build the table from window step k_start (the deferred column's codes are committed through k_start - 1):
+    // eq.(7) draws of the column for the next <= 2*nthr raw rows (whole steps, <= kDefSteps of them), one row per
+    // thread and iteration, and S(t) of every table step
+    auto dtab_build = [&](int k_start) {
+      tvalid = false;
+      if (tbase + k_start - d_lp >= L_dep) { Wd = -1; return; }          // no longer LTD-active (R10)
+      const int r0 = (int)s_offs[k_start - ka];
+      const int nrw = (int)s_offs[kend_w - ka];
+      int kc = kend_w - 1;
+      if (r0 + 2 * nthr < nrw) kc = ka + (int)(s_rraw[r0 + 2 * nthr] >> 16) - 1;   // last whole step
+      kc = min(kc, k_start + kDefSteps - 1);
+      if (kc < k_start) return;                        // a step of > 2*nthr rows: the column stays in the loop
+      const int nr = (int)s_offs[kc + 1 - ka] - r0;
+      const int Wg = cbase + col0 + Wd;
+      const int ww = Wd / CPW, wsh = (Wd % CPW) * BITS;
+      for (int k = tid; k < kDefSteps; k += nthr) s_dS[k] = 0;
+      bool ev[2];
+#pragma unroll
+      for (int it = 0; it < 2; ++it) {
+        const int r = it * nthr + tid;
+        ev[it] = false;
+        if (r < nr) {
+          const uint32_t rr = s_rraw[r0 + r];
+          const int k = ka + (int)(rr >> 16);
+          const int t = tbase + k;
+          const int D = t - d_lp;                                            // R10: Dt = -D < 0
+          if (D < L_dep) {
+            const uint4 u = philox((uint32_t)t, rr & 0xFFFFu, (uint32_t)(Wg >> 2), TAG_LTD, seed);   // eq.(7), R13
+            ev[it] = pick(u, Wg & 3) <= s_dep[D];
+          }
+          if (ev[it]) atomicOr(&s_dev[rr & 0xFFFFu], 1ull << (k - k_start));
+        }
+      }
+#pragma unroll
+      for (int it = 0; it < 2; ++it) {
+        const uint32_t m = __ballot_sync(FULL, ev[it]);
+        if (lane == 0) s_dbits[it * nwarps + warp] = m;
+      }
+      __syncthreads();
+      for (int r = tid; r < nr; r += nthr) {
+        const uint32_t rr = s_rraw[r0 + r];
+        const int rel = ka + (int)(rr >> 16) - k_start;
+        const int i = (int)(rr & 0xFFFFu);
+        const int n = __popcll(s_dev[i] & ((1ull << rel) - 1ull));          // earlier events on the row
+        const int q = (int)((s_w[i * wpr + ww] >> wsh) & FMASK);
+        if (q > n) atomicAdd(&s_dS[rel], q - n);                           // eq.(3) with the clamped codes
+      }
+      __syncthreads();
+      tk0 = k_start; kcov = kc; tr0 = r0; tnr = nr; tvalid = true;
+    };
+
     while (k0 < T) {
       // ---------------------------------------------------------- stage the active-row window
       if (k0 >= kb) {
+        if (tvalid) dtab_commit(min(k0 - 1, kcov));                 // the table indexes the old window
         __syncthreads();
         if (kb > ka) lpre_catch_up(kb - 1 - ka);                   // finish the old window's timers
         __syncthreads();
         ka = k0;
         lpre_upto = -1;
-        Wpd = INT_MIN;                                 // raw row numbering changes
         const int n_o = min(offs_cap, T - ka);
         const uint32_t wbase = offs_g[ka];
         for (int x = tid; x <= n_o; x += nthr) s_offs[x] = offs_g[ka + x] - wbase;
@@ -269,6 +364,12 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         for (int x = tid; x < kDrawRows; x += nthr) s_rraw[nrows + x] = 0xFFFF0000u;   // draw pads (never an event)
         __syncthreads();
       }
+      kend_w = kb;
+      // (re)build the deferred column's table when it is missing or covers too little of this epoch
+      if (Wd >= 0 && (!tvalid || kcov < min(k0 + kDefMargin, kb - 1))) {
+        if (tvalid) dtab_commit(k0 - 1);
+        dtab_build(k0);
+      }
       const int kend = kb;
       const int fp = ep & 1;
       const uint32_t flag_addr = smem_u32(&s_flag[fp]);
@@ -280,10 +381,17 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
       int cnt0[CPT], v1[CPT], cnt1[CPT];
 #pragma unroll
       for (int c = 0; c < CPT; ++c) { cnt0[c] = cnt[c]; v1[c] = v[c]; cnt1[c] = cnt[c]; }
+      // the deferred column (this thread's slot dslot, if any) takes S from its table and no in-loop LTD
+      int dslot = -1;
+#pragma unroll
+      for (int c = 0; c < CPT; ++c)
+        if (tvalid && (valid >> c & 1u) && jcol[c] == Wd) dslot = c;
+      // its warp stops before the first step the table does not cover (the epoch then ends there, no spike)
+      const int kstop = __any_sync(FULL, dslot >= 0) ? kcov + 1 : kend;
       uint32_t dmask = 0;                                  // LTD-active columns of this thread (R10)
 #pragma unroll
       for (int c = 0; c < CPT; ++c)
-        if ((valid >> c & 1u) && lpost[c] >= 0 && (tbase + k0 - lpost[c]) < L_dep) dmask |= 1u << c;
+        if ((valid >> c & 1u) && c != dslot && lpost[c] >= 0 && (tbase + k0 - lpost[c]) < L_dep) dmask |= 1u << c;
       const uint32_t wdirty = __ballot_sync(FULL, dmask != 0);
       // A packed word belongs to TPW consecutive lanes of one warp and, during speculation, only LTD writes
       // codes (each lane its own fields).  When no two LTD-active lanes share a word, a lane's decrement is
@@ -333,13 +441,6 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           for (int c = 0; c < CPT; ++c) {
             if (!(dm >> c & 1u)) continue;                 // warp-uniform
             const int jl = __shfl_sync(FULL, jcol[c], Ls);
-            if (jl == Wpd && base >= pd0 && base + 64 <= pd0 + nthr) {   // warp-uniform: drawn by the CTA
-              const int o = base - pd0, w = o >> 5, sh = o & 31;
-              const uint32_t p0 = s_pd[w], p1 = s_pd[w + 1], p2 = s_pd[w + 2 <= nwarps ? w + 2 : nwarps];
-              if (lane == Ls)
-                evm[c] = ((unsigned long long)__funnelshift_r(p1, p2, sh) << 32) | __funnelshift_r(p0, p1, sh);
-              continue;
-            }
             const int lp = __shfl_sync(FULL, lpost[c], Ls);
             const int jg = cbase + col0 + jl;
             const int D0 = t0 - lp, D1 = t1 - lp;
@@ -407,13 +508,16 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         // step further, which the rollback at t* covers like any other step past t*)
         const int fl = fl_pf;
         fl_pf = __shfl_sync(FULL, ld_volatile_shared_u32addr(flag_addr), 0);
-        if (kk >= kend || kk > fl) break;                        // warp-uniform
+        if (kk >= kstop || kk > fl) {                            // warp-uniform
+          if (kk < kend && kk <= fl && dslot >= 0) hstep = kk;   // beyond the deferred table: end the epoch here
+          break;
+        }
         const int x = kk - ka;
         const int o0 = (int)s_offs[x], o1 = (int)s_offs[x + 1];
         const int ps = (int)s_pst[x], pe = (int)s_pst[x + 1];   // padded row range (integration below)
         const bool wlive = kk >= live_from;                      // warp-uniform
         if (!wlive) {                                            // held warp: skip the run
-          int n = min(live_from - kk, kend - kk);
+          int n = min(live_from - kk, kstop - kk);
           if (fl != INT_MAX) n = min(n, fl - kk + 1);
           bool stop = false;
           if (wdirty) {
@@ -510,6 +614,11 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
 #pragma unroll
             for (int c = 0; c < CPT; ++c)
               S[c] += (int)(Z::LW == 32 ? acc : ((acc >> (c * Z::LW)) & ((1u << (Z::LW & 31)) - 1u)));
+          }
+          if (dslot >= 0) {                                         // the deferred column: S from its table
+            const int Sd = s_dS[kk - tk0];
+#pragma unroll
+            for (int c = 0; c < CPT; ++c) if (c == dslot) S[c] = Sd;
           }
 #pragma unroll
           for (int c = 0; c < CPT; ++c) {
@@ -697,6 +806,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
             for (int c = 0; c < CPT; ++c) S[c] += (int)((w >> (fsh + c * Z::LW)) & FMASK);
           }
 #pragma unroll
+          for (int c = 0; c < CPT; ++c) if (c == dslot) S[c] = s_dS[k2 - tk0];   // k2 <= k_last <= kcov
+#pragma unroll
           for (int c = 0; c < CPT; ++c) {
             if (!(valid >> c & 1u)) continue;
             if (cnt[c] > 0) --cnt[c]; else lif.step_t<FIXED>(v[c], S[c]);
@@ -737,25 +848,14 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         for (int c = 0; c < CPT; ++c)
           if ((valid >> c & 1u) && jcol[c] == Wl) lpost[c] = tP;             // after LTD at t* (R14)
         if (Wl >= 0 && Wl < ncols) {                                           // CTA-uniform
+          // the previous deferred column's eq.(7) events through t* (old last_post, R14) before the LTP below
+          if (tvalid) dtab_commit(P);
           // (no barrier before the catch-up: it reads only the staged window and writes only s_lpre, which
           // nothing reads before the barrier below; the undo above and the LTP below are still separated by it)
           lpre_catch_up(P - ka);                                               // last_pre includes step t*
           __syncthreads();
           const int Wg = cbase + col0 + Wl;
           const int ww = Wl / CPW, wsh = (Wl % CPW) * BITS;
-          // the winner's eq.(7) LTD draws (last_post = t*) for the next raw rows, one per thread, in flight with
-          // the LTP draws below: the winner's warp then finds them in s_pd instead of drawing them itself
-          const bool pd_ok = P + 1 < kend;                                     // CTA-uniform: same window
-          const int pr0 = pd_ok ? (int)s_offs[P + 1 - ka] : 0;
-          const int nrw = (int)s_offs[kend - ka];
-          bool pbit = false;
-          if (pd_ok && pr0 + tid < nrw) {
-            const uint32_t rr = s_rraw[pr0 + tid];
-            const int t = tbase + ka + (int)(rr >> 16);
-            const int D = t - tP;
-            const uint4 u = philox((uint32_t)t, rr & 0xFFFFu, (uint32_t)(Wg >> 2), TAG_LTD, seed);
-            pbit = D < L_dep && pick(u, Wg & 3) <= s_dep[D < L_dep ? D : 0];
-          }
           for (int grp = tid; grp < nq4; grp += nthr) {
             const uint4 u = philox((uint32_t)tP, (uint32_t)Wg, (uint32_t)grp, TAG_LTP, seed);
 #pragma unroll
@@ -775,17 +875,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
               }
             }
           }
-          {
-            const uint32_t m = __ballot_sync(FULL, pbit);
-            if (pd_ok) {
-              if (lane == 0) s_pd[warp] = m;
-              if (tid == 0) s_pd[nwarps] = 0u;
-              Wpd = Wl; pd0 = pr0;
-            } else {
-              Wpd = INT_MIN;
-            }
-          }
           __syncthreads();
+          Wd = Wl; d_lp = tP;           // the new deferred column; its table is built at the next epoch start
         }
       }
       if (trace && tid == 0 && ep < d.trace_cap) {
@@ -802,6 +893,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
       ++ep;
       ++eng_epochs;
     }  // epochs
+    if (tvalid) dtab_commit(min(T - 1, kcov));      // every table step is committed by now
 
     if (rank == 0 && tid == 0) {
       post_sum += (unsigned long long)img_spikes;

@@ -282,3 +282,56 @@ def test_undo_log_overflow_path(gpu, engine):
     _compare_presentations(g, o, synthdata.images(2, "fashion", start=3), 120, synthdata.seeds(2, 13), 784, 256, 1)
     if engine in (0, 2):
         assert int(g.stats()[9]) > 0, "undo-log overflow path not exercised"
+
+
+# ------------------------------------------------------------------ the exact benchmarked launch (bench.py)
+def _batch_vs_oracle(p, n_in, n_exc, bits, imgs, T, seeds, engine=0, expect_lean=None):
+    """One snn_present_batch launch of all images (weights resident in shared memory across the images,
+    the in-launch image-boundary reset, window re-staging and per-image pre-drawn LTD reset) against the
+    oracle presenting the same images one by one: per-image spike counts, final codes, the last image's
+    raster, the state blob and the counters."""
+    g, o = _pair(n_in, n_exc, bits, p, engine=engine)
+    if expect_lean is not None:
+        assert g.info()["lean"] == expect_lean
+    counts = np.zeros(len(imgs), np.int32)
+    g.reset_stats()
+    g.present_batch(imgs, T, seeds, counts)
+    oc, ost = [], np.zeros(6, np.int64)
+    for img, sd in zip(imgs, seeds):
+        o.present(img, T, int(sd))
+        oc.append(int(O.unpack_bits(o.spikes(), n_exc).sum()))
+        ost += o.stats()[:6].astype(np.int64)
+    assert counts.tolist() == oc, "per-image post-spike counts"
+    assert np.array_equal(g.weights(), o.weights()), "conductance codes after the batch"
+    assert np.array_equal(g.spikes(), o.spikes()), "last image's output raster"
+    assert np.array_equal(g.stats()[:6].astype(np.int64), ost), "counters summed over the batch"
+    _assert_state_equal(g, o, n_in, n_exc, p["membrane_mode"])
+    assert sum(oc) > 0
+    return g
+
+
+@pytest.mark.parametrize("mode", [0, 1])
+@pytest.mark.parametrize("engine", [0, 2])
+def test_C4_present_batch_vs_oracle(gpu, engine, mode):
+    """bench.py's launch: 784 -> 6400, 2 bit, default cluster (16 CTAs; lean <2,2,*> kernel for engine 0),
+    8 fashion images in ONE present_batch call."""
+    p = O.params("2b", membrane_mode=mode, init_seed=1)
+    g = _batch_vs_oracle(p, 784, 6400, 2, synthdata.images(8, "fashion", start=200), 350,
+                         synthdata.seeds(8, base_seed=31), engine=engine, expect_lean=int(engine == 0))
+    assert g.info()["cluster_size"] == 16
+
+
+def test_C4_hf_present_batch_vs_oracle(gpu):
+    """The 5-78 Hz "high frequency" row at T = 100, 8 images in one launch on the lean kernel."""
+    p = O.params("hf", membrane_mode=1, init_seed=1)
+    _batch_vs_oracle(p, 784, 6400, 2, synthdata.images(8, "fashion", start=300), 100,
+                     synthdata.seeds(8, base_seed=37), expect_lean=1)
+
+
+@pytest.mark.parametrize("n_exc,bits,preset,cs", [(400, 8, "8b", 0), (1600, 2, "2b", 0), (1600, 2, "2b", 2)])
+def test_C2_C3_present_batch_vs_oracle(gpu, n_exc, bits, preset, cs):
+    """Batches at the C2 / C3 shapes (other thread counts and cluster sizes than the bench's), 12 images per
+    launch: the deferred column's tables cover 2 raw rows per thread, so their extent depends on the CTA size."""
+    p = O.params(preset, membrane_mode=1, init_seed=3, cluster_size=cs)
+    _batch_vs_oracle(p, 784, n_exc, bits, synthdata.images(12, "mnist", start=50), 350,
+                     synthdata.seeds(12, base_seed=41), expect_lean=1)

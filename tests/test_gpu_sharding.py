@@ -111,8 +111,8 @@ def test_sharded_undo_log_overflow(gpu):
 
 @pytest.mark.parametrize("world", [2, 4])
 def test_sharded_C4_784x6400_2bit(gpu, world):
-    """The bench workload split over `world` shards: oracle on one image, then the unsharded CUDA
-    network on a batch (both bit-exact)."""
+    """The bench workload split over `world` shards, against the ORACLE: one image presented alone, then
+    a batch of 4 images in one launch (the oracle presents them one by one)."""
     import paper_conf_date_shelm19_b200 as P
     p = O.params("2b", membrane_mode=0, init_seed=1)
     sh = _shards(784, 6400, 2, p, world)
@@ -120,16 +120,21 @@ def test_sharded_C4_784x6400_2bit(gpu, world):
     imgs = synthdata.images(5, "fashion")
     seeds = synthdata.seeds(5, base_seed=1)
     _compare(sh, o, imgs[:1], 350, seeds[:1], 784, 6400, 0)
-    full = P.Network(784, 6400, 2, P.params_from_dict(p))
-    full.present(imgs[0], 350, int(seeds[0]))
-    counts = np.zeros(4, np.int32)
-    full.present_batch(imgs[1:], 350, seeds[1:], counts)
     for s in sh:
         s.reset_stats()
     P.present_many(sh, [imgs[1:]] * world, 350, [seeds[1:]] * world)
-    assert np.array_equal(np.concatenate([s.weights() for s in sh], axis=1), full.weights())
-    assert np.array_equal(_cat_raster(sh, 350), O.unpack_bits(full.spikes(), 6400))
-    assert all(int(s.stats()[1]) == int(counts.sum()) for s in sh)
+    post = 0
+    for img, sd in zip(imgs[1:], seeds[1:]):
+        o.present(img, 350, int(sd))
+        post += int(o.stats()[1])
+    assert np.array_equal(np.concatenate([s.weights() for s in sh], axis=1), o.weights())
+    assert np.array_equal(_cat_raster(sh, 350), O.unpack_bits(o.spikes(), 6400))
+    assert all(int(s.stats()[1]) == post for s in sh)
+    ref = O.unpack_state(o.state(), 784, 6400)
+    parts = [O.unpack_state(s.state(), 784, s.n_exc) for s in sh]
+    for k in ("cnt", "last_post"):
+        assert np.array_equal(np.concatenate([x[k] for x in parts]), ref[k]), k
+    np.testing.assert_allclose(np.concatenate([x["v"] for x in parts]), ref["v"], rtol=1e-5, atol=0)
 
 
 def test_shard_api_errors(gpu):

@@ -106,20 +106,26 @@ def exact_distribution(p, image, q0, T, wta_mode=0, inh_mode=0):
                     for i in range(n_in):
                         if lp[i] >= 0:
                             trials.append(("p", i, W, P_pot(t - lp[i])))
-                for outcome in itertools.product((0, 1), repeat=len(trials)):
-                    po = 1.0
-                    qq = list(q)
-                    for (kind, i, j, P), hit in zip(trials, outcome):
-                        po *= P if hit else 1.0 - P
-                        if hit:
-                            k = i * n_exc + j
-                            qq[k] = max(qq[k] - 1, 0) if kind == "d" else min(qq[k] + 1, qmax)
+                # every Bernoulli branch, applied in trial order; branches that reach the same codes merge
+                qd = {tuple(q): 1.0}
+                for kind, i, j, P in trials:
+                    k = i * n_exc + j
+                    nd = defaultdict(float)
+                    for qq, pq in qd.items():
+                        if P < 1.0:
+                            nd[qq] += pq * (1.0 - P)
+                        if P > 0.0:
+                            q2 = list(qq)
+                            q2[k] = max(q2[k] - 1, 0) if kind == "d" else min(q2[k] + 1, qmax)
+                            nd[tuple(q2)] += pq * P
+                    qd = nd
+                lpost = list(last_post)
+                for W in spikers:
+                    lpost[W] = t
+                for qq, po in qd.items():
                     if po == 0.0:
                         continue
-                    lpost = list(last_post)
-                    for W in spikers:
-                        lpost[W] = t
-                    key = (tuple(qq), tuple(vv), tuple(cc), tuple(lp), tuple(lpost), raster + (rbits,))
+                    key = (qq, tuple(vv), tuple(cc), tuple(lp), tuple(lpost), raster + (rbits,))
                     new[key] += pr * ps * po
         dist = new
     out = defaultdict(float)
@@ -128,8 +134,8 @@ def exact_distribution(p, image, q0, T, wta_mode=0, inh_mode=0):
     return dict(out)
 
 
-def oracle_samples(p, image, q0, T, n, wta_mode=0):
-    pp = dict(p, wta_mode=wta_mode)
+def oracle_samples(p, image, q0, T, n, wta_mode=0, inh_mode=0):
+    pp = dict(p, wta_mode=wta_mode, inh_mode=inh_mode)
     net = O.OracleNet(N_IN, N_EXC, BITS, pp)
     counts = defaultdict(int)
     for seed in range(n):
@@ -141,16 +147,23 @@ def oracle_samples(p, image, q0, T, n, wta_mode=0):
     return counts
 
 
-@pytest.mark.parametrize("wta_mode", [0, 1])
-def test_bruteforce_matches_oracle_montecarlo(wta_mode):
-    exact = exact_distribution(PARAMS, IMAGE, Q0, T, wta_mode=wta_mode)
+# HOLD inhibition (R7, "inhibitory signal ... for t inh"): an inhibited neuron keeps v.  With
+# t_inh = t_ref = 1 a neuron inhibited at t is blocked at t+1 and integrates again at t+2 < T from its HELD
+# v (HOLD) or from v_reset (RESET), so the raster law at t = 2 separates the two readings.
+PARAMS_HOLD = dict(PARAMS, t_inh_steps=1, t_ref_steps=1)
+
+
+@pytest.mark.parametrize("wta_mode,inh_mode", [(0, 0), (1, 0), (0, 1), (1, 1)])
+def test_bruteforce_matches_oracle_montecarlo(wta_mode, inh_mode):
+    prm = PARAMS if inh_mode == 0 else PARAMS_HOLD
+    exact = exact_distribution(prm, IMAGE, Q0, T, wta_mode=wta_mode, inh_mode=inh_mode)
     assert abs(sum(exact.values()) - 1.0) < 1e-9
     # the configuration must exercise the rules being pinned
     p_spike = sum(pr for (q, r), pr in exact.items() if any(r))
     p_changed = sum(pr for (q, r), pr in exact.items() if q != tuple(int(x) for x in Q0.reshape(-1)))
     assert p_spike > 0.3 and p_changed > 0.2
     n = 100_000
-    mc = oracle_samples(PARAMS, IMAGE, Q0, T, n, wta_mode=wta_mode)
+    mc = oracle_samples(prm, IMAGE, Q0, T, n, wta_mode=wta_mode, inh_mode=inh_mode)
     assert set(mc) <= set(exact), "oracle produced an outcome of probability zero"
     cats = sorted(exact, key=lambda k: -exact[k])
     big = [k for k in cats if exact[k] * n >= 5.0]
@@ -176,4 +189,15 @@ def test_bruteforce_detects_a_wrong_phase_order():
     keys = set(exact) | set(shifted)
     big = [k for k in keys if exact.get(k, 0) * n >= 5.0]
     chi2 = sum((shifted.get(k, 0) * n - exact[k] * n) ** 2 / (exact[k] * n) for k in big)
+    assert sst.chi2.sf(chi2, len(big) - 1) < 1e-6
+
+
+def test_bruteforce_separates_hold_from_reset(wta_mode=0):
+    """Power check for the HOLD rows: the exact laws under HOLD and RESET inhibition (same parameters)
+    differ enough that 10^5 samples of one reject the other (so a HOLD branch that also resets v fails)."""
+    hold = exact_distribution(PARAMS_HOLD, IMAGE, Q0, T, wta_mode=wta_mode, inh_mode=1)
+    reset = exact_distribution(PARAMS_HOLD, IMAGE, Q0, T, wta_mode=wta_mode, inh_mode=0)
+    n = 100_000
+    big = [k for k in hold if hold[k] * n >= 5.0]
+    chi2 = sum((reset.get(k, 0) * n - hold[k] * n) ** 2 / (hold[k] * n) for k in big)
     assert sst.chi2.sf(chi2, len(big) - 1) < 1e-6

@@ -384,6 +384,31 @@ def test_det_arm_hand_values_8bit():
     assert _det_run(8, 1, 128, fires)[0].tolist() == [128 + 1, 128]  # 2.56 e^{-1.5} = 0.571 -> 1; dep 0
 
 
+@pytest.mark.parametrize("t_ltp", [0, 3, 20])
+def test_det_arm_ltp_window_boundary(t_ltp):
+    """R16 window (eqs.(4)(5), Querlioz-style rule): at the post spike of W (t = P), input i takes
+    eq.(4) iff it fired and P - last_pre_i <= t_LTP, else eq.(5).  Four inputs per code value fire exactly
+    t_LTP steps before the post spike (inside: LTP), t_LTP + 1 before (outside: LTD), in the post step itself
+    (D = 0: LTP), and never (LTD).  8 bit, nearest: q = 128 -> LTP 2.56 e^{-1.5} = 0.571 -> +1, LTD 0.286 -> 0;
+    q = 240 -> LTP 2.56 e^{-2.8125} = 0.154 -> 0, LTD 1.28 e^{-0.1875} = 1.061 -> -1."""
+    P = t_ltp + 3
+    steps = [P - t_ltp, P - t_ltp - 1, P, None]
+    p = O.params("16b", stdp_mode=1, rounding=1, t_ltp_steps=t_ltp, i_ext=60.0, v_spike=1e-9,
+                 t_ref_steps=100000)
+    expect = {128: [129, 128, 129, 128], 240: [240, 239, 240, 239]}
+    for q0, want in expect.items():
+        net = O.OracleNet(4, 1, 8, p)
+        raster = np.zeros((P + 1, 1), np.uint32)
+        for i, s in enumerate(steps):
+            if s is not None:
+                raster[s, 0] |= np.uint32(1 << i)
+        net.set_weights(np.full((4, 1), q0, np.uint8))
+        _force_state(net, P)
+        net.present_raster(raster, P + 1, seed=7, keep_state=True, t0=0)
+        assert _spike_steps(net, P + 1) == [P]
+        assert net.weights()[:, 0].astype(int).tolist() == want, (q0, t_ltp)
+
+
 def test_det_arm_2bit_truncation_never_learns():
     """Q0.2: dG_p <= 0.01 = 0.04 LSB, dG_d <= 0.005 = 0.02 LSB -> truncation and nearest give 0:
     consistent with Table II Q0.2 baseline ~ chance (9.6 %)."""
