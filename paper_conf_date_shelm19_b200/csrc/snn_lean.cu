@@ -387,7 +387,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
       for (int c = 0; c < CPT; ++c)
         if (tvalid && (valid >> c & 1u) && jcol[c] == Wd) dslot = c;
       // its warp stops before the first step the table does not cover (the epoch then ends there, no spike)
-      const int kstop = __any_sync(FULL, dslot >= 0) ? kcov + 1 : kend;
+      const bool wdef = __any_sync(FULL, dslot >= 0);
+      const int kstop = wdef ? kcov + 1 : kend;
       uint32_t dmask = 0;                                  // LTD-active columns of this thread (R10)
 #pragma unroll
       for (int c = 0; c < CPT; ++c)
@@ -401,12 +402,16 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
       // countdowns only run down during speculation (R6, R7), so the warp's first step with a live column is
       // k0 + the smallest countdown of its valid columns (no per-step vote needed)
       int live_from;
+      int solo_end = INT_MIN;        // [live_from, solo_end): the deferred column is the warp's only live column
       {
-        int mc0 = INT_MAX;
+        int mc0 = INT_MAX, mnd = INT_MAX;
 #pragma unroll
-        for (int c = 0; c < CPT; ++c) if (valid >> c & 1u) mc0 = min(mc0, cnt[c]);
+        for (int c = 0; c < CPT; ++c)
+          if (valid >> c & 1u) { mc0 = min(mc0, cnt[c]); if (c != dslot) mnd = min(mnd, cnt[c]); }
         mc0 = __reduce_min_sync(FULL, mc0);
+        mnd = __reduce_min_sync(FULL, mnd);
         live_from = mc0 == INT_MAX ? INT_MAX : k0 + mc0;
+        if (wdef && !wdirty && mc0 < mnd) solo_end = mnd == INT_MAX ? kstop : min(k0 + mnd, kstop);
       }
       int kk = k0;
       int p_done = k0 - 1;           // last step fully processed by this thread
@@ -560,6 +565,42 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           kk += n;
           p_done = kk - 1;
           if (stop) break;
+          continue;
+        }
+        if (kk < solo_end && kk > k0) {                          // warp-uniform
+          // only the deferred column is live (the others are held through solo_end - 1): its lane runs the
+          // eqs.(1)(2) chain on the table sums alone, the held columns just count down
+          int n = solo_end - kk;
+          if (fl != INT_MAX) n = min(n, fl - kk + 1);
+          n = min(n, 8);                                         // re-read the early-stop flag every 8 steps
+          int m = n, crossed = 0;
+          unsigned long long key = 0ull;
+#pragma unroll
+          for (int c = 0; c < CPT; ++c) {
+            if (c != dslot) continue;
+            for (m = 0; m < n; ++m)
+              if (lif.step_t<FIXED>(v[c], s_dS[kk + m - tk0])) { crossed = 1; break; }
+            if (crossed)
+              key = ((unsigned long long)lif.ord(v[c]) << 32) | (0xFFFFFFFFu - (uint32_t)(cbase + col0 + jcol[c]));
+          }
+          const int dl = __ffs(__ballot_sync(FULL, dslot >= 0)) - 1;
+          m = __shfl_sync(FULL, m, dl);
+          crossed = __shfl_sync(FULL, crossed, dl);
+          const int steps = crossed ? m + 1 : m;
+#pragma unroll
+          for (int c = 0; c < CPT; ++c) if ((valid >> c & 1u) && c != dslot) cnt[c] -= steps;
+          kk += steps;
+          p_done = kk - 1;
+          if (crossed) {
+            const int kc = kk - 1;
+            if (dslot >= 0) {
+              cstep = kc; ckey = key;
+              atomicMin(&s_flag[fp], kc);
+              for (int r = 0; r < cs; ++r)
+                if (r != rank) red_min_cluster(&s_flag[fp], (uint32_t)r, kc);
+            }
+            break;
+          }
           continue;
         }
       general_step:

@@ -59,6 +59,7 @@ for name, x in (("prev-winner CTA", sel_p), ("other CTAs", sel_o)):
 crit = lat.argmax(axis=0)
 wp = np.array([W[e - 1] // cols if W[e - 1] != 0xFFFFFFFF else -1 for e in range(1, E)])
 print(f"critical CTA == previous winner's CTA in {np.mean(crit[1:] == wp) * 100:.0f}% of epochs")
-steps = (Pst - k0 + 1).astype(float)
+ev = (tr[0, :, 1] >> 32) == 1                  # epochs that ended with a post spike (P = t*)
+steps = (Pst[ev] - k0[ev] + 1).astype(float)
 print(f"epochs {E}, steps/epoch {steps.mean():.1f}, per-epoch: spec (global) {lat.max(axis=0).mean():.0f} ns, "
       f"exchange->end {(end.max(axis=0) - exch.min(axis=0)).mean():.0f} ns, total {(end.max(axis=0) - gstart).mean():.0f} ns")
