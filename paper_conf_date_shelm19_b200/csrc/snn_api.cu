@@ -526,13 +526,22 @@ int create_impl(int n_in, int n_exc, int bits, const snn_params* p, int col_base
     if (ev) {
       // on-chip window of active-row lists + LTD undo log: shrink until it fits
       const int plans[4][3] = {{std::max(n_in, 4096), 512, 16}, {n_in, 256, 16}, {n_in, 128, 8}, {n_in, 64, 4}};
+      // (the lean kernel, when the mode allows it, needs more: prefer the largest window that fits both)
       smem = 0;
+      int k_ev = -1, k_lean = -1;
       for (int k = 0; k < 4; ++k) {
-        rows_cap = plans[k][0]; offs_cap = plans[k][1];
-        logn = p->stdp_mode == SNN_STDP_STOCH ? plans[k][2] : 1;
-        smem = snn::event_smem_bytes(n_in, sw, h->L_pot, h->L_dep, h->q_max, nthr, rows_cap, offs_cap, logn);
-        if (smem <= (size_t)smem_optin) break;
+        const int lg = p->stdp_mode == SNN_STDP_STOCH ? plans[k][2] : 1;
+        const size_t se = snn::event_smem_bytes(n_in, sw, h->L_pot, h->L_dep, h->q_max, nthr, plans[k][0], plans[k][1], lg);
+        if (se > (size_t)smem_optin) continue;
+        if (k_ev < 0) k_ev = k;
+        if (lean_mode && k_lean < 0 &&
+            snn::lean_smem_bytes(n_in, sw, h->L_pot, h->L_dep, nthr, plans[k][0], plans[k][1], lg) <= (size_t)smem_optin)
+          k_lean = k;
       }
+      const int kp = k_lean >= 0 ? k_lean : (k_ev >= 0 ? k_ev : 3);
+      rows_cap = plans[kp][0]; offs_cap = plans[kp][1];
+      logn = p->stdp_mode == SNN_STDP_STOCH ? plans[kp][2] : 1;
+      smem = snn::event_smem_bytes(n_in, sw, h->L_pot, h->L_dep, h->q_max, nthr, rows_cap, offs_cap, logn);
     } else {
       smem = snn::present_smem_bytes(n_in, sw, h->L_pot, h->L_dep, h->q_max, nthr);
     }

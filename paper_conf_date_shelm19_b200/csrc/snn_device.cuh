@@ -138,6 +138,32 @@ struct Lif {
       return vn > vthf;
     }
   }
+  // step_t split in two: the part of eq.(1) that does not depend on v (computable ahead for a block of steps)
+  // and the v-dependent rest; post_t(v, pre_t(S)) performs exactly the operations of step_t(v, S) (the integer
+  // recipe's int64 sum is reassociated, which is exact)
+  template <bool FIXED>
+  __device__ __forceinline__ int pre_t(int S) const {
+    if constexpr (FIXED) {
+      return (int)(A + ((C * (long long)S + (1LL << 15)) >> 16) + E);
+    } else {
+      const float I = __fmul_rn(__int2float_rn(S), kI);
+      return __float_as_int(__fmaf_rn(cf, __fadd_rn(I, ief), af));
+    }
+  }
+  template <bool FIXED>
+  __device__ __forceinline__ bool post_t(int& v, int y) const {
+    if constexpr (FIXED) {
+      const long long x = v;
+      v = (int)(x + (long long)y + ((B * x + (1LL << 31)) >> 32));
+      return v > Vth;
+    } else {
+      const float vf = __int_as_float(v);
+      const float dv = __fmaf_rn(bf, vf, __int_as_float(y));
+      const float vn = __fmaf_rn(dtf, dv, vf);
+      v = __float_as_int(vn);
+      return vn > vthf;
+    }
+  }
   __device__ __forceinline__ uint32_t ord(int v) const {
     return fixed ? ((uint32_t)v ^ 0x80000000u) : float_ord((uint32_t)v);
   }

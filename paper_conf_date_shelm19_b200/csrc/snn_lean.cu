@@ -16,7 +16,7 @@
 //     brought up to date lazily there, and nowhere else;
 //   * the last winner of each CTA is its *deferred* column: it is LTD-active on every input spike right after
 //     its post spike (eq.(7) with small |Dt|) and used to put the longest dependent chain on one warp.  Its LTD
-//     events for the next <= 2*nthr raw rows (<= 64 steps) are drawn by the whole CTA at once, and with them its
+//     events for the next <= nthr raw rows (<= 64 steps) are drawn by the whole CTA at once, and with them its
 //     integration sums S(t) = sum_{i active at t} max(q_i - n_i(<t), 0) (n_i(<t): its events on row i at earlier
 //     table steps -- decrements clamped at 0 commute), so the owning thread reads S(t) from a table and
 //     applies no LTD in the step loop; the events of the committed steps are written back by the CTA when the
@@ -55,9 +55,12 @@ template <int BITS, int CPT_> struct LSwar {
 constexpr int kDrawRows = 64;        // raw rows one LTD draw covers (two Philox blocks per lane, in flight together)
 constexpr int kDefSteps = 64;        // steps one deferred-LTD table covers at most (u64 step masks per input row)
 constexpr int kDefMargin = 16;       // a table with fewer steps left than this is rebuilt at the epoch start
+constexpr int kDefRowsPerThr = 1;    // raw rows a table draws per thread (an epoch spans ~15 steps of ~6 rows)
+constexpr int kSlots = 8;            // fixed row slots per step (steps with more active rows take the general path)
+constexpr int kBlk = 4;              // steps one block integrates before running the LIF chains through them
 
 struct LeanLayout {
-  size_t slots, wsum, flags, misc, dS, dbits, dev, w, pot, dep, lpre, offs, pst, prow, rraw, log, total;
+  size_t slots, wsum, flags, misc, dS, dbits, dev, w, pot, dep, lpre, offs, pst, prow, p8, run, rraw, log, total;
 };
 
 __host__ __device__ inline LeanLayout lean_layout(int n_in, int slice_words, int L_pot, int L_dep, int nthr,
@@ -67,10 +70,10 @@ __host__ __device__ inline LeanLayout lean_layout(int n_in, int slice_words, int
   L.slots = o; o = align16(o + 2 * kMaxCluster * 2 * 8);     // [parity][rank][2] u64: steps, key
   L.wsum = o;  o = align16(o + 32 * 2 * 8);                  // per warp: steps, key
   L.flags = o; o = align16(o + 4 * 4);                       // early-stop flag per epoch parity
-  L.misc = o;  o = align16(o + 16 * 4);
+  L.misc = o;  o = align16(o + 32 * 4);
   L.dS = o;    o = align16(o + (size_t)kDefSteps * 4);                // deferred column: S per table step
-  L.dbits = o; o = align16(o + (size_t)(2 * nthr / 32) * 4);          // deferred column: event bit per raw row
-  L.dev = o;   o = align16(o + (size_t)n_in * 8);                     // deferred column: event steps per input row
+  L.dbits = o; o = align16(o + (size_t)(kDefRowsPerThr * nthr / 32) * 4);   // deferred column: event bit per raw row
+  L.dev = o;   o = align16(o + (size_t)n_in * 8 * 2);                 // deferred column: event steps per input row (x2)
   L.w = o;     o = align16(o + (size_t)slice_words * 4);
   L.pot = o;   o = align16(o + (size_t)(L_pot > 0 ? L_pot : 1) * 4);
   L.dep = o;   o = align16(o + (size_t)(L_dep > 0 ? L_dep : 1) * 4);
@@ -78,6 +81,8 @@ __host__ __device__ inline LeanLayout lean_layout(int n_in, int slice_words, int
   L.offs = o;  o = align16(o + (size_t)(offs_cap + 1) * 4);          // raw row offset of every window step
   L.pst = o;   o = align16(o + (size_t)(offs_cap + 1) * 4);          // padded (x4) start of every window step
   L.prow = o;  o = align16(o + (size_t)(rows_cap + 3 * offs_cap + 4) * 4);   // padded word offsets row*wpr
+  L.p8 = o;    o = align16(o + (size_t)(offs_cap + kBlk) * kSlots * 4);   // first kSlots row byte offsets of each step
+  L.run = o;   o = align16(o + (size_t)(offs_cap + 1));                   // small steps (<= kSlots rows) from here, <= kBlk
   L.rraw = o;  o = align16(o + (size_t)(rows_cap + kDrawRows) * 4);         // raw rows: step << 16 | row id
   L.log = o;   o = align16(o + (size_t)logn * nthr * 4);
   L.total = o;
@@ -129,6 +134,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
   uint32_t* s_offs = reinterpret_cast<uint32_t*>(smem + L.offs);
   uint32_t* s_pst = reinterpret_cast<uint32_t*>(smem + L.pst);
   uint32_t* s_prow = reinterpret_cast<uint32_t*>(smem + L.prow);
+  uint32_t* s_p8 = reinterpret_cast<uint32_t*>(smem + L.p8);
+  uint8_t* s_run = reinterpret_cast<uint8_t*>(smem + L.run);
   uint32_t* s_rraw = reinterpret_cast<uint32_t*>(smem + L.rraw);
   uint32_t* s_log = reinterpret_cast<uint32_t*>(smem + L.log);
   int* s_dS = reinterpret_cast<int*>(smem + L.dS);
@@ -171,15 +178,21 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
     for (int k = tid; k < slice_words / 4; k += nthr) dst[k] = src[k];
   }
   if (tid == 0) { s_flag[0] = INT_MAX; s_flag[1] = INT_MAX; }
-  for (int i = tid; i < n_in; i += nthr) s_dev[i] = 0ull;
+  for (int i = tid; i < 2 * n_in; i += nthr) s_dev[i] = 0ull;
   // optional per-epoch trace (snn_set_trace; tools/trace_epochs.py): per epoch parity, the latest warp exit
   // (%globaltimer), the longest warp speculation loop (cycles) and the deepest speculation (steps)
   unsigned long long* trace = d.trace ? d.trace + (size_t)rank * d.trace_cap * 8 : nullptr;
   unsigned long long* s_trmax = reinterpret_cast<unsigned long long*>(s_misc + 4);    // [2]
   unsigned long long* s_trloop = reinterpret_cast<unsigned long long*>(s_misc + 8);   // [2]
   int* s_trdepth = s_misc + 12;                                                      // [2]
-  if (tid == 0) { s_trmax[0] = s_trmax[1] = 0ull; s_trloop[0] = s_trloop[1] = 0ull; s_trdepth[0] = s_trdepth[1] = 0; }
-  unsigned long long tg0 = 0, tg3 = 0;
+  unsigned long long* s_trcross = reinterpret_cast<unsigned long long*>(s_misc + 16);  // [2] first crossing (ns)
+  if (tid == 0) {
+    s_trmax[0] = s_trmax[1] = 0ull; s_trloop[0] = s_trloop[1] = 0ull; s_trdepth[0] = s_trdepth[1] = 0;
+    s_trcross[0] = s_trcross[1] = ~0ull;
+    for (int q = 24; q < 30; ++q) s_misc[q] = 0;
+  }
+  int* s_trsteps = s_misc + 24;      // [parity][3]: warp-steps taken by block, general and solo paths (trace)
+  unsigned long long tg0 = 0, tg3 = 0, tc3 = 0, tph[5] = {0ull, 0ull, 0ull, 0ull, 0ull};
   int v[CPT], cnt[CPT], lpost[CPT];
 #pragma unroll
   for (int c = 0; c < CPT; ++c) {
@@ -214,8 +227,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
     int k0 = 0;
     // the CTA's deferred column (its last winner, local index Wd; -1 none) and its LTD table: steps [tk0, kcov],
     // raw rows [tr0, tr0 + tnr) of the window; d_lp = its last post spike (absolute step).  CTA-uniform.
-    int Wd = -1, d_lp = 0, tk0 = 0, kcov = -1, tr0 = 0, tnr = 0;
-    bool tvalid = false;
+    int Wd = -1, d_lp = 0, tk0 = 0, kcov = -1, tr0 = 0, tnr = 0, dbuf = 0;
+    bool tvalid = false, pclear = false;
     if (rank == 0 && tid == 0 && T > 0) act_sum += (unsigned long long)(offs_g[T] - offs_g[0]);
     __syncthreads();
 
@@ -231,11 +244,13 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
       }
     };
 
-    // ---- deferred column (CTA-cooperative; every thread calls these at the same point, arguments CTA-uniform)
-    // retire the table: write back the deferred column's eq.(7) events of the table steps <= kc (decrements of one
-    // row clamp at 0, so their total is applied at once by the thread holding the row's first event), count them
-    // and their trials (R20), clear the per-row event masks
-    auto dtab_commit = [&](int kc) {
+    // ---- deferred column (CTA-cooperative; every thread calls these at the same point, arguments CTA-uniform).
+    // The per-row event masks are double-buffered (s_dev + dbuf * n_in), so clearing a retired table's masks and
+    // drawing the next table share one barrier phase.  Phases: apply | clear + draw | sums.
+    // apply: write back the table's eq.(7) events of the steps <= kc (decrements of one row clamp at 0, so their
+    // total is applied at once by the thread holding the row's first event), count them and their trials (R20)
+    auto dtab_apply = [&](int kc) {
+      const unsigned long long* dev = s_dev + dbuf * n_in;
       const int ww = Wd / CPW, wsh = (Wd % CPW) * BITS;
       const int relc = kc - tk0;
       for (int r = tid; r < tnr; r += nthr) {
@@ -246,7 +261,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         if (tbase + k - d_lp < L_dep) ++ltd_trials;
         if (!((s_dbits[r >> 5] >> (r & 31)) & 1u)) continue;
         ++ltd_events;
-        const unsigned long long m = s_dev[i];
+        const unsigned long long m = dev[i];
         if (__popcll(m & ((1ull << (k - tk0)) - 1ull)) != 0) continue;    // not the row's first event
         const int n = __popcll(relc >= 63 ? m : (m & ((2ull << relc) - 1ull)));
         // the column's field of row i is this thread's alone (other fields may be in an undo: atomic)
@@ -254,30 +269,35 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         const int dec = min(n, (int)((*pw >> wsh) & FMASK));
         if (dec) atomicSub(pw, (uint32_t)dec << wsh);
       }
-      __syncthreads();
-      for (int r = tid; r < tnr; r += nthr) s_dev[s_rraw[tr0 + r] & 0xFFFFu] = 0ull;
-      __syncthreads();
       tvalid = false;
+      pclear = true;                                   // its masks are cleared in the next phase
     };
-    // build the table from window step k_start (the deferred column's codes are committed through k_start - 1):
-    // eq.(7) draws of the column for the next <= 2*nthr raw rows (whole steps, <= kDefSteps of them), one row per
-    // thread and iteration, and S(t) of every table step
-    auto dtab_build = [&](int k_start) {
-      tvalid = false;
-      if (tbase + k_start - d_lp >= L_dep) { Wd = -1; return; }          // no longer LTD-active (R10)
+    auto dtab_clear = [&]() {
+      if (!pclear) return;
+      unsigned long long* dev = s_dev + dbuf * n_in;
+      for (int r = tid; r < tnr; r += nthr) dev[s_rraw[tr0 + r] & 0xFFFFu] = 0ull;
+      pclear = false;
+    };
+    // draw: the next table from window step k_start (the column's codes are committed through k_start - 1 by the
+    // end of this phase): eq.(7) draws of the column for the next <= kDefRowsPerThr*nthr raw rows (whole steps, <= kDefSteps
+    // of them), one row per thread and iteration, into the other mask buffer.  Returns false (no table) when the
+    // column is no longer LTD-active or the next step alone has more rows than a table covers.
+    int nt_r0 = 0, nt_nr = 0, nt_kc = -1;
+    auto dtab_draw = [&](int k_start) -> bool {
+      if (tbase + k_start - d_lp >= L_dep) { Wd = -1; return false; }   // no longer LTD-active (R10)
       const int r0 = (int)s_offs[k_start - ka];
       const int nrw = (int)s_offs[kend_w - ka];
       int kc = kend_w - 1;
-      if (r0 + 2 * nthr < nrw) kc = ka + (int)(s_rraw[r0 + 2 * nthr] >> 16) - 1;   // last whole step
+      if (r0 + kDefRowsPerThr * nthr < nrw) kc = ka + (int)(s_rraw[r0 + kDefRowsPerThr * nthr] >> 16) - 1;
       kc = min(kc, k_start + kDefSteps - 1);
-      if (kc < k_start) return;                        // a step of > 2*nthr rows: the column stays in the loop
+      if (kc < k_start) return false;                  // a step of more rows than a table: the column stays in the loop
       const int nr = (int)s_offs[kc + 1 - ka] - r0;
       const int Wg = cbase + col0 + Wd;
-      const int ww = Wd / CPW, wsh = (Wd % CPW) * BITS;
+      unsigned long long* dev = s_dev + (dbuf ^ 1) * n_in;
       for (int k = tid; k < kDefSteps; k += nthr) s_dS[k] = 0;
-      bool ev[2];
+      bool ev[kDefRowsPerThr];
 #pragma unroll
-      for (int it = 0; it < 2; ++it) {
+      for (int it = 0; it < kDefRowsPerThr; ++it) {
         const int r = it * nthr + tid;
         ev[it] = false;
         if (r < nr) {
@@ -289,31 +309,54 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
             const uint4 u = philox((uint32_t)t, rr & 0xFFFFu, (uint32_t)(Wg >> 2), TAG_LTD, seed);   // eq.(7), R13
             ev[it] = pick(u, Wg & 3) <= s_dep[D];
           }
-          if (ev[it]) atomicOr(&s_dev[rr & 0xFFFFu], 1ull << (k - k_start));
+          if (ev[it]) atomicOr(&dev[rr & 0xFFFFu], 1ull << (k - k_start));
         }
       }
 #pragma unroll
-      for (int it = 0; it < 2; ++it) {
+      for (int it = 0; it < kDefRowsPerThr; ++it) {
         const uint32_t m = __ballot_sync(FULL, ev[it]);
         if (lane == 0) s_dbits[it * nwarps + warp] = m;
       }
-      __syncthreads();
-      for (int r = tid; r < nr; r += nthr) {
-        const uint32_t rr = s_rraw[r0 + r];
-        const int rel = ka + (int)(rr >> 16) - k_start;
+      nt_r0 = r0; nt_nr = nr; nt_kc = kc;
+      tk0 = k_start;
+      return true;
+    };
+    // sums (after a barrier): S(t) of every table step from the clamped codes; the table goes live
+    auto dtab_sums = [&]() {
+      dbuf ^= 1;
+      const unsigned long long* dev = s_dev + dbuf * n_in;
+      const int ww = Wd / CPW, wsh = (Wd % CPW) * BITS;
+      for (int r = tid; r < nt_nr; r += nthr) {
+        const uint32_t rr = s_rraw[nt_r0 + r];
+        const int rel = ka + (int)(rr >> 16) - tk0;
         const int i = (int)(rr & 0xFFFFu);
-        const int n = __popcll(s_dev[i] & ((1ull << rel) - 1ull));          // earlier events on the row
+        const int n = __popcll(dev[i] & ((1ull << rel) - 1ull));            // earlier events on the row
         const int q = (int)((s_w[i * wpr + ww] >> wsh) & FMASK);
         if (q > n) atomicAdd(&s_dS[rel], q - n);                           // eq.(3) with the clamped codes
       }
+      kcov = nt_kc; tr0 = nt_r0; tnr = nt_nr; tvalid = true;
+    };
+    // retire the table completely (window / image end)
+    auto dtab_retire = [&](int kc) {
+      dtab_apply(kc);
       __syncthreads();
-      tk0 = k_start; kcov = kc; tr0 = r0; tnr = nr; tvalid = true;
+      dtab_clear();
+      __syncthreads();
+    };
+    // (re)build from k_start, retiring the current table (if any) through k_start - 1
+    auto dtab_rebuild = [&](int k_start) {
+      if (tvalid) { dtab_apply(k_start - 1); __syncthreads(); }
+      dtab_clear();
+      const bool ok = dtab_draw(k_start);
+      __syncthreads();
+      if (ok) { dtab_sums(); __syncthreads(); }
     };
 
     while (k0 < T) {
       // ---------------------------------------------------------- stage the active-row window
       if (k0 >= kb) {
-        if (tvalid) dtab_commit(min(k0 - 1, kcov));                 // the table indexes the old window
+        if (tvalid) dtab_retire(min(k0 - 1, kcov));                 // the table indexes the old window
+        else if (pclear) { dtab_clear(); __syncthreads(); }
         __syncthreads();
         if (kb > ka) lpre_catch_up(kb - 1 - ka);                   // finish the old window's timers
         __syncthreads();
@@ -360,21 +403,30 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
             s_prow[p0 + (r - o0)] = i * (uint32_t)wpr;
           }
           for (uint32_t q = p0 + (o1 - o0); q < p1; ++q) s_prow[q] = zero_off;
+#pragma unroll
+          for (int j = 0; j < kSlots; ++j) s_p8[kSlots * x + j] = 4u * ((uint32_t)j < o1 - o0 ? s_prow[p0 + j] : zero_off);
         }
+        for (int x = nsteps * kSlots + tid; x < (nsteps + kBlk) * kSlots; x += nthr) s_p8[x] = 4u * zero_off;
         for (int x = tid; x < kDrawRows; x += nthr) s_rraw[nrows + x] = 0xFFFF0000u;   // draw pads (never an event)
+        for (int x = tid; x < nsteps; x += nthr) {
+          int run = 0;
+          while (run < kBlk && x + run < nsteps && s_offs[x + run + 1] - s_offs[x + run] <= (uint32_t)kSlots) ++run;
+          s_run[x] = (uint8_t)run;
+        }
         __syncthreads();
       }
       kend_w = kb;
       // (re)build the deferred column's table when it is missing or covers too little of this epoch
       if (Wd >= 0 && (!tvalid || kcov < min(k0 + kDefMargin, kb - 1))) {
-        if (tvalid) dtab_commit(k0 - 1);
-        dtab_build(k0);
+        dtab_rebuild(k0);
       }
       const int kend = kb;
       const int fp = ep & 1;
       const uint32_t flag_addr = smem_u32(&s_flag[fp]);
       const long long tl0 = trace ? clock64() : 0ll;
-      long long c_draw = 0, c_int = 0, c_ev = 0;          // trace: cycles in LTD draws, integration+LIF, LTD events
+      // trace (SNN_LEAN_TRACE_CYCLES builds): cycles of the warp in held runs, block steps, general steps
+      long long c_held = 0, c_blk = 0, c_gen = 0, t_it = 0;
+#define LEAN_CYC(acc) do { if (kTraceCycles && trace) (acc) += clock64() - t_it; } while (0)
       if (trace && tid == 0) tg0 = globaltimer();
 
       // ---------------------------------------------------------- speculation (warp-synchronous)
@@ -427,6 +479,15 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
       auto evbits = [&](int c, int a0, int a1) -> uint32_t {
         const int nr = a1 - a0;
         return nr <= 0 ? 0u : ((uint32_t)(evm[c] >> (a0 - dr0)) & (nr >= 32 ? FULL : ((1u << nr) - 1u)));
+      };
+
+      // a crossing at window step kc: lower the early-stop flag of every CTA of the cluster (lane r -> CTA r)
+      auto signal_cross = [&](int kc) {
+        if (trace && lane == 0) atomicMin(&s_trcross[fp], globaltimer());
+        if (lane < cs) {
+          if (lane == rank) atomicMin(&s_flag[fp], kc);
+          else red_min_cluster(&s_flag[fp], (uint32_t)lane, kc);
+        }
       };
 
       // LTD draws of every (lane, column) pair of the warp for raw rows [base, base + 64): lanes over rows,
@@ -517,6 +578,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           if (kk < kend && kk <= fl && dslot >= 0) hstep = kk;   // beyond the deferred table: end the epoch here
           break;
         }
+        if (kTraceCycles && trace) t_it = clock64();
         const int x = kk - ka;
         const int o0 = (int)s_offs[x], o1 = (int)s_offs[x + 1];
         const int ps = (int)s_pst[x], pe = (int)s_pst[x + 1];   // padded row range (integration below)
@@ -539,7 +601,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
                 const long long td = (kTraceCycles && trace) ? clock64() : 0ll;
                 draw(a0);
                 dr0 = a0;
-                if (kTraceCycles && trace) { c_draw += clock64() - td; c_ev -= clock64() - td; }
+                (void)td;
               }
               int nev = 0;
 #pragma unroll
@@ -553,7 +615,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
               if (nev) ltd_apply(kk + m, a0, a1);                    // this lane has events in the step
             }
             n = m;
-            if (kTraceCycles && trace) c_ev += clock64() - tq;
+            (void)tq;
           }
           if (n == 0 && !stop) goto general_step;                                  // a big step first
           if (n > 0 && kk == k0) {
@@ -564,6 +626,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           for (int c = 0; c < CPT; ++c) if (valid >> c & 1u) cnt[c] -= n;
           kk += n;
           p_done = kk - 1;
+          LEAN_CYC(c_held);
           if (stop) break;
           continue;
         }
@@ -591,17 +654,82 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           for (int c = 0; c < CPT; ++c) if ((valid >> c & 1u) && c != dslot) cnt[c] -= steps;
           kk += steps;
           p_done = kk - 1;
+          LEAN_CYC(c_held);
+          if (trace && lane == 0) atomicAdd(&s_trsteps[fp * 3 + 2], steps);
           if (crossed) {
             const int kc = kk - 1;
-            if (dslot >= 0) {
-              cstep = kc; ckey = key;
-              atomicMin(&s_flag[fp], kc);
-              for (int r = 0; r < cs; ++r)
-                if (r != rank) red_min_cluster(&s_flag[fp], (uint32_t)r, kc);
-            }
+            if (dslot >= 0) { cstep = kc; ckey = key; }
+            signal_cross(kc);
             break;
           }
           continue;
+        }
+        if (!wdirty && kk > k0) {                                // warp-uniform
+          // a block of up to kBlk steps of <= kSlots rows: every sum first (independent loads), then the
+          // eqs.(1)(2) chains through them; a crossing ends the block (the sums after it are discarded)
+          int nbs = min((int)s_run[x], kstop - kk);
+          if (fl != INT_MAX) nbs = min(nbs, fl - kk + 1);
+          if (nbs > 0) {
+            // sums of the block's steps and the v-independent part of eq.(1) (ahead of the chains); every step of the
+            // block is summed unconditionally (branch-free, so all loads are in flight together; s_p8 is padded with
+            // the zero row past the window), sums past nbs are discarded
+            const char* const wb = reinterpret_cast<const char*>(wcol);
+            auto ldw = [&](uint32_t off) { return (*reinterpret_cast<const uint32_t*>(wb + off) >> fsh) & Z::LMASK; };
+            uint32_t acc[kBlk];
+#pragma unroll
+            for (int j = 0; j < kBlk; ++j) {
+              const uint4 m = *reinterpret_cast<const uint4*>(s_p8 + kSlots * (x + j));
+              const uint4 m2 = *reinterpret_cast<const uint4*>(s_p8 + kSlots * (x + j) + 4);
+              acc[j] = ((ldw(m.x) + ldw(m.y)) + (ldw(m.z) + ldw(m.w))) + ((ldw(m2.x) + ldw(m2.y)) + (ldw(m2.z) + ldw(m2.w)));
+            }
+            int yv[kBlk][CPT];
+#pragma unroll
+            for (int j = 0; j < kBlk; ++j) {
+              const int Sd = (dslot >= 0 && j < nbs) ? s_dS[kk + j - tk0] : 0;
+#pragma unroll
+              for (int c = 0; c < CPT; ++c) {
+                const int Sc = c == dslot ? Sd
+                                          : (int)(Z::LW == 32 ? acc[j] : ((acc[j] >> (c * Z::LW)) & ((1u << (Z::LW & 31)) - 1u)));
+                yv[j][c] = lif.pre_t<FIXED>(Sc);
+              }
+            }
+            // the chains: eqs.(1)(2) step by step; a crossing ends the block (the sums after it are discarded)
+            uint32_t cmb = 0;
+            int jb = 0;
+#pragma unroll
+            for (int j = 0; j < kBlk; ++j) {
+              if (j >= nbs || cmb) continue;                     // warp-uniform
+              jb = j;
+              uint32_t cm = 0;
+#pragma unroll
+              for (int c = 0; c < CPT; ++c) {
+                if (!(valid >> c & 1u)) continue;
+                if (cnt[c] > 0) { --cnt[c]; continue; }             // refractory / inhibited: hold v (R6, R7)
+                if (lif.post_t<FIXED>(v[c], yv[j][c])) cm |= 1u << c;   // eq.(2): v > v_th
+              }
+              if (cm) {
+                cstep = kk + j;
+#pragma unroll
+                for (int c = 0; c < CPT; ++c) {
+                  if (!(cm >> c & 1u)) continue;
+                  const unsigned long long key = ((unsigned long long)lif.ord(v[c]) << 32) |
+                                                 (0xFFFFFFFFu - (uint32_t)(cbase + col0 + jcol[c]));
+                  ckey = key > ckey ? key : ckey;
+                }
+              }
+              cmb = __any_sync(FULL, cm != 0) ? 1u : 0u;
+            }
+            LEAN_CYC(c_blk);
+            if (trace && lane == 0) atomicAdd(&s_trsteps[fp * 3 + 0], cmb ? jb + 1 : nbs);
+            if (cmb) {
+              p_done = kk + jb;
+              signal_cross(kk + jb);
+              break;
+            }
+            kk += nbs;
+            p_done = kk - 1;
+            continue;
+          }
         }
       general_step:
         // ---- this step's LTD events of the warp's LTD-active pairs (draws cover 32 rows ahead)
@@ -612,7 +740,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
             const long long tq = (kTraceCycles && trace) ? clock64() : 0ll;
             draw(o0);
             dr0 = o0;
-            if (kTraceCycles && trace) c_draw += clock64() - tq;
+            (void)tq;
           }
           if (!big) {
 #pragma unroll
@@ -671,7 +799,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
 #pragma unroll
           for (int c = 0; c < CPT; ++c) if ((valid >> c & 1u) && cnt[c] > 0) --cnt[c];
         }
-        if (kTraceCycles && trace) c_int += clock64() - tq_int;
+        (void)tq_int;
         const long long tq_ev = (kTraceCycles && trace) ? clock64() : 0ll;
         // ---- (a5) LTD events of the step (old last_post, R14), applied in step order
         if (wdirty && dmask) {
@@ -702,7 +830,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
             }
           }
         }
-        if (kTraceCycles && trace) c_ev += clock64() - tq_ev;
+        (void)tq_ev;
         if (kk == k0) {
 #pragma unroll
           for (int c = 0; c < CPT; ++c) { v1[c] = v[c]; cnt1[c] = cnt[c]; }
@@ -717,11 +845,10 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
                                            (0xFFFFFFFFu - (uint32_t)(cbase + col0 + jcol[c]));
             ckey = key > ckey ? key : ckey;
           }
-          atomicMin(&s_flag[fp], kk);
-          for (int r = 0; r < cs; ++r)
-            if (r != rank) red_min_cluster(&s_flag[fp], (uint32_t)r, kk);
         }
-        if (__any_sync(FULL, cm != 0)) break;
+        LEAN_CYC(c_gen);
+        if (trace && lane == 0) atomicAdd(&s_trsteps[fp * 3 + 1], 1);
+        if (__any_sync(FULL, cm != 0)) { signal_cross(kk); break; }
         ++kk;
       }
       if (hstep != kNoStep) {                                    // tell the cluster where to stop
@@ -735,8 +862,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         atomicMax(&s_trmax[fp], globaltimer());
         const unsigned long long f16 = 0xFFFFull;
         const unsigned long long loop16 = min((unsigned long long)(clock64() - tl0) >> 4, f16);
-        atomicMax(&s_trloop[fp], (loop16 << 48) | (min((unsigned long long)c_draw >> 4, f16) << 32) |
-                                 (min((unsigned long long)c_ev >> 4, f16) << 16) | min((unsigned long long)c_int >> 4, f16));
+        atomicMax(&s_trloop[fp], (loop16 << 48) | (min((unsigned long long)c_held >> 4, f16) << 32) |
+                                 (min((unsigned long long)c_blk >> 4, f16) << 16) | min((unsigned long long)c_gen >> 4, f16));
         atomicMax(&s_trdepth[fp], p_done - k0 + 1);
       }
 
@@ -776,7 +903,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         if (lane == 0) s_flag[fp ^ 1] = INT_MAX;
       }
       if (cs > 1) { cluster_arrive(); cluster_wait(); } else { __syncthreads(); }   // the one cross-SM exchange
-      if (trace && tid == 0) tg3 = globaltimer();
+      if (trace && tid == 0) { tg3 = globaltimer(); tc3 = clock64(); }
 
       // ---------------------------------------------------------- global decision
       int P, H;
@@ -889,12 +1016,19 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         for (int c = 0; c < CPT; ++c)
           if ((valid >> c & 1u) && jcol[c] == Wl) lpost[c] = tP;             // after LTD at t* (R14)
         if (Wl >= 0 && Wl < ncols) {                                           // CTA-uniform
-          // the previous deferred column's eq.(7) events through t* (old last_post, R14) before the LTP below
-          if (tvalid) dtab_commit(P);
-          // (no barrier before the catch-up: it reads only the staged window and writes only s_lpre, which
-          // nothing reads before the barrier below; the undo above and the LTP below are still separated by it)
+          // phase 1: the previous deferred column's eq.(7) events through t* (old last_post, R14) and the input
+          // spike timers through t* (no barrier before: the catch-up reads only the staged window and writes only
+          // s_lpre; the table write-back touches only the deferred column's fields, atomically)
+          if (tvalid) dtab_apply(P);
           lpre_catch_up(P - ka);                                               // last_pre includes step t*
           __syncthreads();
+          if (trace && tid == 0) tph[0] = clock64();
+          // phase 2: LTP of the winner (eq.(6)) next to the eq.(7) draws of its table (it is the new deferred
+          // column, last_post = t*) and the clearing of the retired table's masks
+          dtab_clear();
+          Wd = Wl; d_lp = tP;
+          const bool tab = P + 1 < kend && dtab_draw(P + 1);
+          if (trace && tid == 0) tph[1] = clock64();
           const int Wg = cbase + col0 + Wl;
           const int ww = Wl / CPW, wsh = (Wl % CPW) * BITS;
           for (int grp = tid; grp < nq4; grp += nthr) {
@@ -916,25 +1050,38 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
               }
             }
           }
+          if (trace && tid == 0) tph[2] = clock64();
           __syncthreads();
-          Wd = Wl; d_lp = tP;           // the new deferred column; its table is built at the next epoch start
+          if (trace && tid == 0) tph[3] = clock64();
+          if (tab) { dtab_sums(); __syncthreads(); }   // phase 3: the table's sums read the codes after LTP
+          if (trace && tid == 0) tph[4] = clock64();
         }
       }
       if (trace && tid == 0 && ep < d.trace_cap) {
         unsigned long long* rec = trace + (size_t)ep * 8;
-        rec[0] = ((unsigned long long)b << 32) | (unsigned)k0;
-        rec[1] = ((unsigned long long)(event ? 1 : 2) << 32) | (unsigned)P;
+        rec[0] = ((unsigned long long)b << 32) | (unsigned)k0 | ((unsigned long long)min(s_trsteps[fp * 3], 0xFFFF) << 48);
+        rec[1] = ((unsigned long long)(event ? 1 : 2) << 32) | (unsigned)P |
+                 ((unsigned long long)min(s_trsteps[fp * 3 + 1], 0xFFFF) << 48);
         rec[2] = tg0; rec[3] = s_trmax[fp]; rec[5] = tg3;
-        rec[4] = event ? (unsigned long long)(0xFFFFFFFFu - (uint32_t)K) : 0xFFFFFFFFull;   // winner column
+        rec[4] = (event ? (unsigned long long)(0xFFFFFFFFu - (uint32_t)K) : 0xFFFFFFFFull) |   // winner column
+                 ((unsigned long long)min(s_trsteps[fp * 3 + 2], 0xFFFF) << 48);
         rec[6] = s_trloop[fp];   // slowest warp: loop | draws | LTD events | integration+LIF (cycles / 16, 16 bits each)
+        if (!kTraceCycles) {     // winner's CTA: the three phases after the exchange (cycles / 8 after it, 16 bits each)
+          rec[6] = 0ull;
+          if (tph[0] > tc3)
+            for (int q = 0; q < 4; ++q) rec[6] |= min((tph[q + 1] - tph[q]) >> 3, 0xFFFFull) << (48 - 16 * q);
+        }
+        s_trcross[fp] = ~0ull;
+        tph[0] = tph[1] = tph[2] = tph[3] = tph[4] = 0ull;
         rec[7] = globaltimer();
-        s_trmax[fp] = 0ull; s_trloop[fp] = 0ull; s_trdepth[fp] = 0;   // reused at epoch ep + 2 (after two barriers)
+        s_trmax[fp] = 0ull; s_trloop[fp] = 0ull; s_trdepth[fp] = 0;
+        s_trsteps[fp * 3] = s_trsteps[fp * 3 + 1] = s_trsteps[fp * 3 + 2] = 0;   // reused at epoch ep + 2 (after two barriers)
       }
       k0 = k_last + 1;
       ++ep;
       ++eng_epochs;
     }  // epochs
-    if (tvalid) dtab_commit(min(T - 1, kcov));      // every table step is committed by now
+    if (tvalid) dtab_retire(min(T - 1, kcov));      // every table step is committed by now
 
     if (rank == 0 && tid == 0) {
       post_sum += (unsigned long long)img_spikes;

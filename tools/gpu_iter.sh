@@ -8,3 +8,4 @@ python -c "
 import json
 d=json.load(open('gpurun_out/bench.json')); print('bench', d['value'], d['e2e']['value'], 'epochs', d['secondary']['epochs_per_image'], 'resim', d['secondary']['resims_per_image'], 'hz', d['secondary']['log_stops_per_image'], d['clocks']['sm_mhz'], d['clocks']['reasons'])
 "; tail -2 gpurun_out/bench.err; cat gpurun_out/trace_lean.txt
+SNN_LIB_PATH=exp_libs/libsnn_cyc.so timeout 120 python tools/trace_lean.py --images 8 > gpurun_out/trace_lean_cyc.txt 2>&1; grep "cycles/epoch\|warp-steps" gpurun_out/trace_lean_cyc.txt

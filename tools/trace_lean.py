@@ -29,6 +29,10 @@ tr = tr[:, valid]
 E = tr.shape[1]
 cols = 6400 // cs
 start, end_spec, exch, end = tr[:, :, 2], tr[:, :, 3], tr[:, :, 5], tr[:, :, 7]
+nblk, ngen, nsolo = tr[:, :, 0] >> 48, tr[:, :, 1] >> 48, tr[:, :, 4] >> 48
+tr[:, :, 0] &= 0xFFFFFFFFFFFF
+tr[:, :, 1] &= 0xFFFFFFFFFFFF
+tr[:, :, 4] &= 0xFFFFFFFFFFFF
 W = tr[0, :, 4]
 k0 = tr[0, :, 0] & 0xFFFFFFFF
 Pst = tr[0, :, 1] & 0xFFFFFFFF
@@ -54,8 +58,8 @@ pw = [W[e - 1] // cols if W[e - 1] != 0xFFFFFFFF else -1 for e in range(1, E)]
 sel_p = np.array([split[pw[e - 1], e] for e in range(1, E) if pw[e - 1] >= 0])
 sel_o = np.array([split[r, e] for e in range(1, E) for r in range(cs) if r != pw[e - 1]])
 for name, x in (("prev-winner CTA", sel_p), ("other CTAs", sel_o)):
-    print(f"{name:16s} slowest warp cycles/epoch: loop {x[:, 0].mean():7.0f}  draws {x[:, 1].mean():6.0f}  "
-          f"LTD events {x[:, 2].mean():6.0f}  integration+LIF {x[:, 3].mean():6.0f}")
+    print(f"{name:16s} slowest warp cycles/epoch: loop {x[:, 0].mean():7.0f}  held+solo {x[:, 1].mean():6.0f}  "
+          f"block {x[:, 2].mean():6.0f}  general {x[:, 3].mean():6.0f}")
 crit = lat.argmax(axis=0)
 wp = np.array([W[e - 1] // cols if W[e - 1] != 0xFFFFFFFF else -1 for e in range(1, E)])
 print(f"critical CTA == previous winner's CTA in {np.mean(crit[1:] == wp) * 100:.0f}% of epochs")
@@ -63,3 +67,12 @@ ev = (tr[0, :, 1] >> 32) == 1                  # epochs that ended with a post s
 steps = (Pst[ev] - k0[ev] + 1).astype(float)
 print(f"epochs {E}, steps/epoch {steps.mean():.1f}, per-epoch: spec (global) {lat.max(axis=0).mean():.0f} ns, "
       f"exchange->end {(end.max(axis=0) - exch.min(axis=0)).mean():.0f} ns, total {(end.max(axis=0) - gstart).mean():.0f} ns")
+ph = tr[:, :, 6]
+win = [(e, W[e] // cols) for e in range(E) if W[e] != 0xFFFFFFFF]     # the winner's CTA runs the phases
+if win:
+    x = np.array([[(ph[r, e] >> (48 - 16 * q)) & 0xFFFF for q in range(4)] for e, r in win], dtype=np.float64) * 8
+    x = x[x.sum(axis=1) > 0]
+    if len(x):
+        print(f"winner CTA after the exchange (cycles, phase-stamp build): draw {x[:, 0].mean():.0f}, LTP {x[:, 1].mean():.0f}, "
+              f"barrier {x[:, 2].mean():.0f}, sums {x[:, 3].mean():.0f}")
+print(f"warp-steps per CTA per epoch: block {nblk.mean():.1f}  general {ngen.mean():.1f}  solo {nsolo.mean():.1f}")
