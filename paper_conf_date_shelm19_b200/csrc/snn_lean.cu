@@ -453,17 +453,16 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
       const bool ltd_plain = !__any_sync(FULL, dmask != 0 && __popc(same_word & wdirty) > 1);
       // countdowns only run down during speculation (R6, R7), so the warp's first step with a live column is
       // k0 + the smallest countdown of its valid columns (no per-step vote needed)
+      // the deferred column runs ahead on its own (below); the step loop handles the other columns (lvalid)
+      const uint32_t lvalid = valid & ~(dslot >= 0 ? (1u << dslot) : 0u);
       int live_from;
-      int solo_end = INT_MIN;        // [live_from, solo_end): the deferred column is the warp's only live column
       {
-        int mc0 = INT_MAX, mnd = INT_MAX;
+        int mnd = INT_MAX;
 #pragma unroll
         for (int c = 0; c < CPT; ++c)
-          if (valid >> c & 1u) { mc0 = min(mc0, cnt[c]); if (c != dslot) mnd = min(mnd, cnt[c]); }
-        mc0 = __reduce_min_sync(FULL, mc0);
+          if (lvalid >> c & 1u) mnd = min(mnd, cnt[c]);
         mnd = __reduce_min_sync(FULL, mnd);
-        live_from = mc0 == INT_MAX ? INT_MAX : k0 + mc0;
-        if (wdef && !wdirty && mc0 < mnd) solo_end = mnd == INT_MAX ? kstop : min(k0 + mnd, kstop);
+        live_from = mnd == INT_MAX ? INT_MAX : k0 + mnd;
       }
       int kk = k0;
       int p_done = k0 - 1;           // last step fully processed by this thread
@@ -556,6 +555,47 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         }
       };
 
+      // ---- the deferred column runs ahead alone: its S(t) comes from the table and it has no in-loop LTD, so its
+      // lane walks its eqs.(1)(2) chain to its first crossing (or the table's end, or a crossing already reported)
+      // at once and lowers the early-stop flag; the step loop below then handles only the warp's other columns.
+      // Past t* nothing it computed is kept (RESET: every column restarts from its countdown), so running ahead
+      // is exact; for a replay (no spike) it leaves its state after step k0 in v1/cnt1 like every column.
+      int p_look = k0 - 1;
+      if (wdef) {                                                  // warp-uniform
+        int cd = kNoStep, last = k0 - 1;
+        unsigned long long keyd = 0ull;
+        const int fl0 = ld_volatile_shared_u32addr(flag_addr);
+        const int lim = fl0 == INT_MAX ? kstop : min(kstop, fl0 + 1);
+#pragma unroll
+        for (int c = 0; c < CPT; ++c) {
+          if (c != dslot) continue;
+          int m = k0;
+          const int nh = min(cnt[c], max(lim - k0, 0));          // held steps: the countdown runs down (R6, R7)
+          cnt[c] -= nh;
+          m += nh;
+          if (nh > 0) { v1[c] = v[c]; cnt1[c] = cnt0[c] - 1; }   // state after step k0 (held at k0)
+          for (; m < lim; ++m) {
+            const bool cr = lif.post_t<FIXED>(v[c], lif.pre_t<FIXED>(s_dS[m - tk0]));   // eqs.(1)(2), eq.(3) from the table
+            if (m == k0) { v1[c] = v[c]; cnt1[c] = 0; }
+            if (cr) {
+              cd = m;
+              keyd = ((unsigned long long)lif.ord(v[c]) << 32) | (0xFFFFFFFFu - (uint32_t)(cbase + col0 + jcol[c]));
+              break;
+            }
+          }
+          last = cd != kNoStep ? cd : m - 1;
+        }
+        const int dl = __ffs(__ballot_sync(FULL, dslot >= 0)) - 1;
+        const int cdw = __shfl_sync(FULL, cd, dl);
+        const int lastw = __shfl_sync(FULL, last, dl);
+        if (dslot >= 0) { p_look = last; if (cd != kNoStep) { cstep = cd; ckey = keyd; } }
+        if (cdw != kNoStep) {
+          signal_cross(cdw);
+        } else if (lastw == kstop - 1 && kstop < kend) {          // the table ends first: the epoch ends there
+          if (dslot >= 0) hstep = kstop;
+          signal_cross(kstop - 1);
+        }
+      }
       int fl_pf = __shfl_sync(FULL, ld_volatile_shared_u32addr(flag_addr), 0);   // early-stop flag, one step ahead
 #ifdef SNN_LEAN_DEBUG
       long long dbg_it = 0;
@@ -574,10 +614,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         // step further, which the rollback at t* covers like any other step past t*)
         const int fl = fl_pf;
         fl_pf = __shfl_sync(FULL, ld_volatile_shared_u32addr(flag_addr), 0);
-        if (kk >= kstop || kk > fl) {                            // warp-uniform
-          if (kk < kend && kk <= fl && dslot >= 0) hstep = kk;   // beyond the deferred table: end the epoch here
-          break;
-        }
+        if (kk >= kstop || kk > fl) break;                       // warp-uniform
         if (kTraceCycles && trace) t_it = clock64();
         const int x = kk - ka;
         const int o0 = (int)s_offs[x], o1 = (int)s_offs[x + 1];
@@ -620,48 +657,14 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           if (n == 0 && !stop) goto general_step;                                  // a big step first
           if (n > 0 && kk == k0) {
 #pragma unroll
-            for (int c = 0; c < CPT; ++c) { v1[c] = v[c]; cnt1[c] = (valid >> c & 1u) ? cnt[c] - 1 : cnt[c]; }
+            for (int c = 0; c < CPT; ++c) if (lvalid >> c & 1u) { v1[c] = v[c]; cnt1[c] = cnt[c] - 1; }
           }
 #pragma unroll
-          for (int c = 0; c < CPT; ++c) if (valid >> c & 1u) cnt[c] -= n;
+          for (int c = 0; c < CPT; ++c) if (lvalid >> c & 1u) cnt[c] -= n;
           kk += n;
           p_done = kk - 1;
           LEAN_CYC(c_held);
           if (stop) break;
-          continue;
-        }
-        if (kk < solo_end && kk > k0) {                          // warp-uniform
-          // only the deferred column is live (the others are held through solo_end - 1): its lane runs the
-          // eqs.(1)(2) chain on the table sums alone, the held columns just count down
-          int n = solo_end - kk;
-          if (fl != INT_MAX) n = min(n, fl - kk + 1);
-          n = min(n, 8);                                         // re-read the early-stop flag every 8 steps
-          int m = n, crossed = 0;
-          unsigned long long key = 0ull;
-#pragma unroll
-          for (int c = 0; c < CPT; ++c) {
-            if (c != dslot) continue;
-            for (m = 0; m < n; ++m)
-              if (lif.step_t<FIXED>(v[c], s_dS[kk + m - tk0])) { crossed = 1; break; }
-            if (crossed)
-              key = ((unsigned long long)lif.ord(v[c]) << 32) | (0xFFFFFFFFu - (uint32_t)(cbase + col0 + jcol[c]));
-          }
-          const int dl = __ffs(__ballot_sync(FULL, dslot >= 0)) - 1;
-          m = __shfl_sync(FULL, m, dl);
-          crossed = __shfl_sync(FULL, crossed, dl);
-          const int steps = crossed ? m + 1 : m;
-#pragma unroll
-          for (int c = 0; c < CPT; ++c) if ((valid >> c & 1u) && c != dslot) cnt[c] -= steps;
-          kk += steps;
-          p_done = kk - 1;
-          LEAN_CYC(c_held);
-          if (trace && lane == 0) atomicAdd(&s_trsteps[fp * 3 + 2], steps);
-          if (crossed) {
-            const int kc = kk - 1;
-            if (dslot >= 0) { cstep = kc; ckey = key; }
-            signal_cross(kc);
-            break;
-          }
           continue;
         }
         if (!wdirty && kk > k0) {                                // warp-uniform
@@ -703,7 +706,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
               uint32_t cm = 0;
 #pragma unroll
               for (int c = 0; c < CPT; ++c) {
-                if (!(valid >> c & 1u)) continue;
+                if (!(lvalid >> c & 1u)) continue;
                 if (cnt[c] > 0) { --cnt[c]; continue; }             // refractory / inhibited: hold v (R6, R7)
                 if (lif.post_t<FIXED>(v[c], yv[j][c])) cm |= 1u << c;   // eq.(2): v > v_th
               }
@@ -791,13 +794,13 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           }
 #pragma unroll
           for (int c = 0; c < CPT; ++c) {
-            if (!(valid >> c & 1u)) continue;
+            if (!(lvalid >> c & 1u)) continue;
             if (cnt[c] > 0) { --cnt[c]; continue; }                 // refractory / inhibited: hold v (R6, R7)
             if (lif.step_t<FIXED>(v[c], S[c])) cm |= 1u << c;       // eq.(2): v > v_th
           }
         } else {
 #pragma unroll
-          for (int c = 0; c < CPT; ++c) if ((valid >> c & 1u) && cnt[c] > 0) --cnt[c];
+          for (int c = 0; c < CPT; ++c) if ((lvalid >> c & 1u) && cnt[c] > 0) --cnt[c];
         }
         (void)tq_int;
         const long long tq_ev = (kTraceCycles && trace) ? clock64() : 0ll;
@@ -833,7 +836,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         (void)tq_ev;
         if (kk == k0) {
 #pragma unroll
-          for (int c = 0; c < CPT; ++c) { v1[c] = v[c]; cnt1[c] = cnt[c]; }
+          for (int c = 0; c < CPT; ++c) if (lvalid >> c & 1u) { v1[c] = v[c]; cnt1[c] = cnt[c]; }
         }
         p_done = kk;
         if (cm) {                                                // crossing: the WTA key (R7)
@@ -857,6 +860,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         for (int r = 0; r < cs; ++r)
           if (r != rank) red_min_cluster(&s_flag[fp], (uint32_t)r, hstep - 1);
       }
+      p_done = max(p_done, p_look);
       if (valid) eng_spec += (uint32_t)(p_done - k0 + 1) * (uint32_t)__popc(valid);
       if (trace && lane == 0) {
         atomicMax(&s_trmax[fp], globaltimer());
