@@ -596,7 +596,6 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           signal_cross(kstop - 1);
         }
       }
-      int fl_pf = __shfl_sync(FULL, ld_volatile_shared_u32addr(flag_addr), 0);   // early-stop flag, one step ahead
 #ifdef SNN_LEAN_DEBUG
       long long dbg_it = 0;
 #endif
@@ -609,11 +608,9 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         }
 #endif
         // one lane's read of the early-stop flag decides for the warp (lanes that executed the load apart
-        // could otherwise see different values and leave the loop apart)
-        // (the value read here is used one step later: a flag lowered meanwhile only lets the warp run one
-        // step further, which the rollback at t* covers like any other step past t*)
-        const int fl = fl_pf;
-        fl_pf = __shfl_sync(FULL, ld_volatile_shared_u32addr(flag_addr), 0);
+        // could otherwise see different values and leave the loop apart); read fresh every iteration: an
+        // iteration may be a block of steps, so a stale value would let the warp overrun t* by a whole block
+        const int fl = __shfl_sync(FULL, ld_volatile_shared_u32addr(flag_addr), 0);
         if (kk >= kstop || kk > fl) break;                       // warp-uniform
         if (kTraceCycles && trace) t_it = clock64();
         const int x = kk - ka;
