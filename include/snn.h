@@ -25,6 +25,18 @@
  *    Handles are not thread-safe; distinct handles may be used from distinct threads.
  *  - Weights persist across presentations (online learning).  v, refractory counters and
  *    spike timers are reset at the start of each presentation unless SNN_KEEP_STATE (R5).
+ *
+ * Differences from the call list of SURVEY.md §8(b) (which this header otherwise follows):
+ *  - snn_present_many takes an n_images argument: each handle presents a batch of images in the one
+ *    launch (the ensemble C5 runs 8 networks x B images per call), not one image per handle.
+ *  - snn_create_sharded(..., nccl_unique_id) became snn_create_shard + snn_shard_ipc_handle /
+ *    snn_shard_connect (multi-process) or snn_shard_link (one process): the exchange step is a
+ *    16-byte per-epoch summary written by the kernel itself into every rank's device mailbox
+ *    (NVLink peer stores), so there is no NCCL communicator to bootstrap.  The only
+ *    host-side collective is the caller's all_gather of the 64-byte IPC handles.  SNN_ENCCL is kept
+ *    (reserved) so that the error-code values of §8(b) do not shift.
+ *  - Added beyond §8(b): snn_present_batch / snn_present_ex (batches, raster input, KEEP_STATE),
+ *    state/trace/info accessors, and the NEXT-1 / NEXT-4 entry points below.
  */
 #ifndef SNN_H
 #define SNN_H
@@ -39,7 +51,7 @@ extern "C" {
 #define SNN_EINVAL  (-1)   /* invalid argument or parameter                       */
 #define SNN_ENOMEM  (-2)   /* host or device allocation failed                    */
 #define SNN_ECUDA   (-3)   /* CUDA runtime error (message in snn_last_error)      */
-#define SNN_ENCCL   (-4)   /* NCCL error (sharded handles)                        */
+#define SNN_ENCCL   (-4)   /* reserved (never returned): the shard exchange uses no NCCL, see below */
 #define SNN_ESIZE   (-5)   /* caller buffer too small, or network exceeds the on-chip capacity */
 #define SNN_ECOOP   (-6)   /* cluster / co-residency launch not possible          */
 

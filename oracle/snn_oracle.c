@@ -246,6 +246,9 @@ int oracle_present(oracle_net* n, const uint8_t* image, int T, uint64_t seed) {
 
 int oracle_present_ex(oracle_net* n, const void* input, int T, uint64_t seed, int flags, int t0) {
   if (!n || T < 0 || t0 < 0 || (T > 0 && !input)) return E_INVAL;
+  /* continuing a presentation may not step back in time: every stored timer is below t_next <= t0, so
+   * Dt = t - last >= 1 indexes the eqs.(6)(7) tables (input validation, not part of the method) */
+  if ((flags & ORACLE_KEEP_STATE) && t0 < n->t_next) return E_INVAL;
   const oracle_params* p = &n->p;
   const int n_in = n->n_in, n_exc = n->n_exc;
   const int wi = (n_in + 31) / 32, we = (n_exc + 31) / 32;
@@ -470,6 +473,15 @@ int oracle_set_state(oracle_net* n, const void* buf, size_t sz) {
   if (sz < oracle_state_bytes(n)) return E_SIZE;
   const int32_t* w = (const int32_t*)buf;
   if (w[0] != n->n_in || w[1] != n->n_exc || w[3] != n->p.membrane_mode || w[2] < 0) return E_INVAL;
+  /* countdowns >= 0; spike timers NEVER or before t_next (input validation) */
+  for (int j = 0; j < n->n_exc; ++j) {
+    const int32_t c = w[4 + n->n_exc + j], lp = w[4 + 2 * n->n_exc + j];
+    if (c < 0 || lp < NEVER || lp >= w[2]) return E_INVAL;
+  }
+  for (int i = 0; i < n->n_in; ++i) {
+    const int32_t lp = w[4 + 3 * n->n_exc + i];
+    if (lp < NEVER || lp >= w[2]) return E_INVAL;
+  }
   n->t_next = w[2];
   const int32_t* v = w + 4;
   for (int j = 0; j < n->n_exc; ++j) {

@@ -309,6 +309,9 @@ int present_impl(snn_handle* h, const void* input, int n_images, int T, const ui
   if ((flags & SNN_KEEP_STATE) && n_images > 1) return fail(SNN_EINVAL, "SNN_KEEP_STATE needs n_images == 1");
   if ((flags & SNN_RASTER_INPUT) && n_images > 1) return fail(SNN_EINVAL, "SNN_RASTER_INPUT needs n_images == 1");
   if (!(flags & SNN_KEEP_STATE) && t0 != 0) return fail(SNN_EINVAL, "t0 != 0 requires SNN_KEEP_STATE");
+  // continuing may not step back in time: stored timers are < t_next <= t0, so every Dt >= 1 indexes the tables
+  if ((flags & SNN_KEEP_STATE) && t0 < h->t_next)
+    return fail(SNN_EINVAL, "SNN_KEEP_STATE with t0 = %d before the stored state's next step %d", t0, h->t_next);
   const bool ev = h->engine == SNN_ENGINE_EVENT;
   if (ev && T > snn::kEvMaxT) return fail(SNN_EINVAL, "T=%d exceeds %d for the event engine", T, snn::kEvMaxT);
   if (ev && (flags & SNN_FLOOR_PROBE)) return fail(SNN_EINVAL, "SNN_FLOOR_PROBE applies to the per-step engine");
@@ -1036,6 +1039,14 @@ int snn_set_state(snn_handle* h, const void* buf, size_t n) {
   const int32_t* w = static_cast<const int32_t*>(buf);
   if (w[0] != h->n_in || w[1] != h->n_exc || w[3] != h->p.membrane_mode || w[2] < 0)
     return fail(SNN_EINVAL, "state header does not match this handle");
+  for (int j = 0; j < h->n_exc; ++j) {           // countdowns >= 0, spike timers NEVER or before t_next
+    const int32_t c = w[4 + h->n_exc + j], lp = w[4 + 2 * h->n_exc + j];
+    if (c < 0 || lp < snn::kNever || lp >= w[2]) return fail(SNN_EINVAL, "state: column %d has cnt %d / last_post %d", j, c, lp);
+  }
+  for (int i = 0; i < h->n_in; ++i) {
+    const int32_t lp = w[4 + 3 * h->n_exc + i];
+    if (lp < snn::kNever || lp >= w[2]) return fail(SNN_EINVAL, "state: input %d has last_pre %d (t_next %d)", i, lp, w[2]);
+  }
   DevGuard g(h->dev);
   const size_t ne = (size_t)h->n_exc;
   CUDA_TRY(cudaMemcpyAsync(h->d_v, w + 4, ne * 4, cudaMemcpyHostToDevice, h->stream));

@@ -335,3 +335,25 @@ def test_C2_C3_present_batch_vs_oracle(gpu, n_exc, bits, preset, cs):
     p = O.params(preset, membrane_mode=1, init_seed=3, cluster_size=cs)
     _batch_vs_oracle(p, 784, n_exc, bits, synthdata.images(12, "mnist", start=50), 350,
                      synthdata.seeds(12, base_seed=41), expect_lean=1)
+
+
+def test_state_validation_matches_oracle(gpu):
+    """Both sides reject a continuation that steps back in time and a state blob with timers at or after its
+    t_next or negative countdowns, and accept the same valid blob."""
+    import paper_conf_date_shelm19_b200 as P
+    p = O.params("8b", membrane_mode=1)
+    g, o = _pair(16, 4, 8, p)
+    img = np.full(16, 200, np.uint8)
+    g.present(img, 10, 3)
+    o.present(img, 10, 3)
+    with pytest.raises(P.SnnError) as e:
+        g.present_ex(img, 5, 3, flags=P.SNN_KEEP_STATE, t0=9)
+    assert e.value.rc == -1
+    st = o.state()
+    assert np.array_equal(g.state(), st)
+    for bad_index, bad_value in ((4 + 4 + 0, -1), (4 + 8 + 1, int(st[2])), (4 + 12 + 3, int(st[2]) + 5)):
+        b = st.copy()
+        b[bad_index] = bad_value
+        with pytest.raises(P.SnnError):
+            g.set_state(b)
+    g.set_state(st)

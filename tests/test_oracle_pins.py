@@ -492,3 +492,22 @@ def test_invalid_params_rejected(bad):
 def test_invalid_bits_rejected(bits):
     with pytest.raises(O.OracleError):
         O.OracleNet(784, 10, bits, O.params("8b"))
+
+
+def test_state_validation_rejects_timers_from_the_future():
+    """Input validation: a continued presentation may not start before the stored state's next
+    step, and a state blob whose spike timers are not before its t_next (or whose countdowns are negative)
+    is rejected, so Dt = t - last >= 1 always indexes the eqs.(6)(7) tables."""
+    p = O.params("8b")
+    net = O.OracleNet(16, 4, 8, p)
+    net.present(np.full(16, 200, np.uint8), 10, seed=3)
+    with pytest.raises(O.OracleError):
+        net.present_ex(np.full(16, 200, np.uint8), 5, 3, flags=O.ORACLE_KEEP_STATE, t0=9)
+    net.present_ex(np.full(16, 200, np.uint8), 5, 3, flags=O.ORACLE_KEEP_STATE, t0=10)   # t0 == t_next is fine
+    st = net.state()
+    for bad_index, bad_value in ((4 + 4 + 0, -1), (4 + 8 + 1, int(st[2])), (4 + 12 + 3, int(st[2]) + 5)):
+        b = st.copy()
+        b[bad_index] = bad_value
+        with pytest.raises(O.OracleError):
+            net.set_state(b)
+    net.set_state(st)
