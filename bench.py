@@ -129,18 +129,95 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
-def cpu_baseline(n_images: int) -> dict:
+def cpu_info() -> dict:
+    """CPU model and core counts of the host the oracle runs on (lscpu, else /proc/cpuinfo)."""
+    info = {"model": None, "logical_cpus": os.cpu_count(), "usable_cpus": len(os.sched_getaffinity(0))}
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            k, _, v = line.partition(":")
+            if k.strip() == "Model name":
+                info["model"] = v.strip()
+            elif k.strip() in ("Socket(s)", "Core(s) per socket", "Thread(s) per core"):
+                info[k.strip().lower().replace("(s)", "s").replace(" ", "_")] = v.strip()
+    except Exception:
+        pass
+    if info["model"] is None:
+        try:
+            for line in open("/proc/cpuinfo"):
+                if line.startswith("model name"):
+                    info["model"] = line.split(":", 1)[1].strip()
+                    break
+        except OSError:
+            pass
+    return info
+
+
+def _oracle_images(mode: int, n_images: int) -> float:
+    """Seconds for the oracle to present n_images C4 images (784->6400, 2-bit, T=350) in membrane mode `mode`."""
     from oracle import oracle as O
-    p = O.params("2b", membrane_mode=0, init_seed=1)
+    p = O.params("2b", membrane_mode=mode, init_seed=1)
     net = O.OracleNet(N_IN, N_EXC, BITS, p)
     imgs = synthdata.images(n_images, "fashion", start=1000)
     seeds = synthdata.seeds(n_images, base_seed=3)
     t0 = time.perf_counter()
     for k in range(n_images):
         net.present(imgs[k], T_STEPS, int(seeds[k]))
-    dt = time.perf_counter() - t0
-    return {"value": n_images / dt, "unit": "images/s", "cores": 1, "kind": "oracle",
-            "sample": f"{n_images} fashion images of C4 (784->6400, 2-bit, T=350) via oracle_present, 1 thread"}
+    return time.perf_counter() - t0
+
+
+def _c5_pinned(args):
+    k, cpu = args
+    os.sched_setaffinity(0, {cpu})
+    return _c5_worker_unpinned(k)
+
+
+def _c5_worker_unpinned(k: int) -> float:
+    """One C5 network (784->400, bits {2,4,8}[k % 3], its Table I row, seed k) presenting 2 MNIST-shaped
+    images; returns the seconds it took."""
+    from oracle import oracle as O
+    bits = (2, 4, 8)[k % 3]
+    net = O.OracleNet(N_IN, 400, bits, O.params({2: "2b", 4: "4b", 8: "8b"}[bits], init_seed=1 + k))
+    imgs = synthdata.images(2, "mnist", start=10 * k)
+    seeds = synthdata.seeds(2, base_seed=100 + k)
+    t0 = time.perf_counter()
+    for x, sd in zip(imgs, seeds):
+        net.present(x, T_STEPS, int(sd))
+    return time.perf_counter() - t0
+
+
+def cpu_baseline(n_images: int) -> dict:
+    """The oracle as it stands (never tuned), on the host: C4 on ONE pinned core in both membrane modes (the
+    line's value is the fp32 mode, the bench's), plus the all-cores C5 ensemble figure: one
+    784->400 network per core, min(64, cores) networks in parallel."""
+    cpus = sorted(os.sched_getaffinity(0))
+    old = set(cpus)
+    os.sched_setaffinity(0, {cpus[0]})                  # taskset -c <first usable core>
+    try:
+        t_fp32 = _oracle_images(0, n_images)
+        t_fixed = _oracle_images(1, n_images)
+    finally:
+        os.sched_setaffinity(0, old)
+    out = {"value": n_images / t_fp32, "unit": "images/s", "cores": 1, "kind": "oracle",
+           "sample": f"{n_images} fashion images of C4 (784->6400, 2-bit, T=350) via oracle_present, fp32 membranes, "
+                     f"pinned to core {cpus[0]}",
+           "fixed_q15_16": {"value": n_images / t_fixed, "unit": "images/s", "cores": 1},
+           "cpu": cpu_info()}
+    try:
+        import multiprocessing as mp
+        n = min(64, len(cpus))
+        ctx = mp.get_context("spawn")
+        t0 = time.perf_counter()
+        with ctx.Pool(n) as pool:
+            secs = pool.map(_c5_pinned, [(k, cpus[k % len(cpus)]) for k in range(n)])
+        wall = time.perf_counter() - t0
+        out["c5_all_cores"] = {"value": 2 * n / max(secs), "unit": "images/s", "cores": n, "networks": n,
+                               "sample": f"{n} C5 networks (784->400, bits (2,4,8)[k%3], Table I rows), one per "
+                                         f"pinned core, 2 MNIST-shaped images each, T=350; value = images / slowest "
+                                         f"network's time", "wall_s_incl_spawn": wall}
+    except Exception as e:                              # noqa: BLE001 -- a missing pool must not sink the bench
+        out["c5_all_cores"] = {"unavailable": str(e)[:200]}
+    return out
 
 
 def main():
@@ -241,6 +318,10 @@ def main():
     for n in nets:
         n.reset_stats()
     launches0 = sum(n.info()["launches"] for n in nets)
+    profiled = K == 1                                 # single-handle presentations record kernel events
+    if profiled:
+        net0 = nets[0]
+        net0.set_profile(True)
 
     # ---- timed region: device time per step (CUDA events on the launching stream), L2 flushed between steps
     sampler = ClockSampler(local)
@@ -260,6 +341,9 @@ def main():
         dist.barrier()
     clocks = sampler.stop()
     step_ms = [a.elapsed_time(b) for a, b in ev]
+    kern_ms, kern_n = nets[0].profile() if profiled else (None, 0)
+    if profiled:
+        nets[0].set_profile(False)
     dev_s = sum(step_ms) / 1e3
     stats = net.stats()
     for n in nets[1:]:                 # per-shard trial / event counters add up; [0], [1], [6..8] are network-wide
@@ -279,20 +363,22 @@ def main():
     value = images / dev_s
     ev_rate = events / dev_s
 
-    # ---- latency floor.  Event engine: the path needs one cluster exchange per epoch (post spike), so
-    # its synchronisation floor is epochs x the measured barrier.cluster cost at this cluster size
-    # (profiles/r01_sync_probe.txt, 128 threads); per-step engine: measured live with SNN_FLOOR_PROBE.
+    # ---- latency floor: the same launch shape (B images, same cluster) doing only the
+    # synchronisation skeleton of the path -- per epoch (lean kernel: the handle's measured epochs per image) --
+    # timed live with CUDA events around the kernel on its stream; frac = t_floor / t_kernel per image
     floor = None
-    if args.engine == 0:
-        probe_ns = {1: 380.7, 2: 444.0, 4: 485.5, 8: 572.6, 16: 760.9}
-        cs = info["cluster_size"]
-        key = min(probe_ns, key=lambda k: abs(k - cs))
-        per_image_us = 1e3 * (sum(step_ms) / args.steps) / B
-        ep = int(stats[8]) / (B * args.steps)
-        floor = {"kind": "event engine: epochs x cluster-exchange cost",
-                 "epochs_per_image": ep, "exchange_ns": probe_ns[key],
-                 "t_floor_us_per_image": ep * probe_ns[key] / 1e3, "t_image_us": per_image_us,
-                 "frac": ep * probe_ns[key] / 1e3 / per_image_us}
+    if not args.no_floor and args.engine == 0 and info.get("lean") and profiled and kern_n:
+        net.set_profile(True)
+        for i in range(3):
+            step(args.warmup + i, flags=P.snn.SNN_FLOOR_PROBE)
+        fl_ms, fl_n = net.profile()
+        net.set_profile(False)
+        t_img = 1e3 * (kern_ms / kern_n) / B
+        t_fl = 1e3 * (fl_ms / fl_n) / B
+        floor = {"kind": "lean kernel, same launch shape: per epoch only the early-stop signal, warp/CTA summaries, "
+                         "DSMEM stores, cluster barrier and decision (SNN_FLOOR_PROBE), measured live",
+                 "epochs_per_image": int(stats[8]) / (B * args.steps), "t_floor_us_per_image": t_fl,
+                 "t_kernel_us_per_image": t_img, "frac": t_fl / t_img}
     if not args.no_floor and args.engine == 1:
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
@@ -339,8 +425,11 @@ def main():
     alg_bytes = (int(stats[0]) * N_EXC * bits_b                       # integration reads (a2)
                  + (int(stats[2]) + int(stats[4])) * bits_b           # LTD/LTP trial reads (a5)
                  + (int(stats[3]) + int(stats[5])) * bits_b)          # conditional writes (a5)
-    per_launch_bytes = alg_bytes / max(1, launches)
-    per_launch_s = dev_s / max(1, launches) if not dist else (sum(step_ms) / 1e3) / max(1, launches)
+    # dominant kernel = the presentation kernel (one launch per step); its time comes from the CUDA events the
+    # library records around it on the launching stream (snn_set_profile), else the whole step
+    n_main = kern_n if (profiled and kern_n) else args.steps
+    per_launch_bytes = alg_bytes / max(1, n_main)
+    per_launch_s = (kern_ms / 1e3 / kern_n) if (profiled and kern_n) else (sum(step_ms) / 1e3) / args.steps
     smclk = (clocks.get("sm_max_mhz") or 1965.0)
     peak_smem = SMEM_BYTES_PER_CLK_PER_SM * N_SM * smclk * 1e6 / 1e9   # GB/s, whole chip
     achieved = per_launch_bytes / per_launch_s / 1e9
@@ -356,6 +445,9 @@ def main():
                 "traffic": traffic, "traffic_source": traffic_src,
                 "peak_source": f"derived: 128 B/clk/SM (B300_MICROARCH smem crossbar) x {N_SM} SMs x {smclk:.0f} MHz",
                 "alg_bytes_per_launch": per_launch_bytes,
+                "kernel": "present_lean_kernel" if info.get("lean") else "present_event_kernel",
+                "kernel_ms_per_launch": 1e3 * per_launch_s,
+                "kernel_share_of_step": (kern_ms / sum(step_ms)) if (profiled and kern_n) else None,
                 "note": "latency-bound step loop; see latency_roofline"}
 
     # ---- NEXT-1: inference with the learned weights frozen, images independent.  Device-timed
@@ -387,11 +479,12 @@ def main():
             t = torch.tensor([its], device=coll_dev, dtype=torch.float64)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             its = float(t.item())
-            tot = torch.tensor([float(ist[0]), float(ist[1]), float(n_inf)], device=coll_dev, dtype=torch.float64)
+            tot = torch.tensor([float(ist[0]), float(ist[1]), float(ist[2]), float(n_inf)], device=coll_dev,
+                               dtype=torch.float64)
             dist.all_reduce(tot, op=dist.ReduceOp.SUM)
-            ist = np.array([tot[0].item(), tot[1].item()])
-            n_inf = int(tot[2].item())
-        lane_ops = 7.0 * N_EXC * T_STEPS * n_inf + float(ist[0]) * N_EXC
+            ist = np.array([tot[0].item(), tot[1].item(), tot[2].item()])
+            n_inf = int(tot[3].item())
+        lane_ops = 7.0 * float(ist[2]) + float(ist[0]) * N_EXC
         smclk_i = (clocks.get("sm_max_mhz") or 1965.0)
         peak_ops = ws * N_SM * 128 * smclk_i * 1e6 / 1e12
         inference = {"metric": "inference images/s (learned weights frozen, P:88 labelling/inference protocol)",
@@ -401,7 +494,9 @@ def main():
                      "post_spikes_per_image": float(ist[1]) / n_inf,
                      "roofline": {"bound": "alu", "achieved": lane_ops / its / 1e12, "peak": peak_ops,
                                   "unit": "Tlane-op/s", "frac": lane_ops / its / 1e12 / peak_ops,
-                                  "work": "7 lane-ops per column-step (LIF recipe) + 1 per synaptic event",
+                                  "work": "7 lane-ops per column-step that ran the LIF recipe (not refractory or "
+                                          "inhibited; counted by the kernel) + 1 per synaptic event",
+                                  "lif_column_steps_per_image": float(ist[2]) / n_inf,
                                   "peak_source": f"derived: {ws} GPU(s) x 148 SMs x 128 FP32/INT lanes x {smclk_i:.0f} MHz"}}
 
     line = {

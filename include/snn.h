@@ -132,7 +132,9 @@ int snn_synchronize(snn_handle* h);
 #define SNN_KEEP_STATE    2   /* keep v / counters / timers; steps are numbered t0 .. t0+T-1              */
 #define SNN_RECORD_INPUT  4   /* also record the input raster of the last image (snn_get_input_raster)    */
 #define SNN_ASYNC         8   /* return after enqueueing; host buffers must stay valid until synchronize  */
-#define SNN_FLOOR_PROBE  16   /* benchmark probe: same launch shape, per-step barriers/exchange only, no work */
+#define SNN_FLOOR_PROBE  16   /* benchmark probe (results are discarded, weights untouched): the same launch
+                                 shape doing only the synchronisation skeleton -- per step (per-step engine)
+                                 or per epoch, with the handle's mean epochs per image so far (lean kernel) */
 
 /* Present one image (n_in bytes, host or device) for T steps with learning on ("Each image is
  * presented to the network for t_learn ms").  `seed` keys every random draw of the presentation. */
@@ -176,6 +178,12 @@ int snn_set_state(snn_handle* h, const void* buf, size_t n);
  * [6] images presented, [7] steps simulated; event engine only: [8] epochs
  * (cluster exchanges), [9] speculation stops on a full undo log, [10] re-simulations,
  * [11] speculated column-steps, [12] undone LTD events; [13..15] reserved (0). */
+/* Kernel timing (bench.py roofline): with profiling on, every presentation records CUDA events on the
+ * handle's stream immediately before and after its presentation kernel (the pre-pass kernels of the
+ * event engine are outside the pair).  snn_get_profile synchronises the stream and returns the summed
+ * kernel milliseconds and the number of kernels since the last call (or snn_set_profile), then resets. */
+int snn_set_profile(snn_handle* h, int on);
+int snn_get_profile(snn_handle* h, double* kernel_ms, int64_t* kernels);
 #define SNN_NSTATS 16
 int snn_get_stats(snn_handle* h, uint64_t stats[SNN_NSTATS]);
 int snn_reset_stats(snn_handle* h);
@@ -238,8 +246,9 @@ int snn_shard_link(snn_handle* const* hs, int world);
  * not updated either (inference counters: snn_get_infer_stats).  All pointers host or device (the call
  * stages host buffers); SNN_ASYNC returns after enqueueing.  T <= 65535; n_exc <= 7168;
  * unsharded handles only.  Errors: SNN_EINVAL (arguments), SNN_ESIZE (n_exc too large), SNN_ECUDA.
- * snn_get_infer_stats: [0] sum over images and steps of active input rows, [1] post spikes, since
- * the handle was created.
+ * snn_get_infer_stats: [0] sum over images and steps of active input rows, [1] post spikes, [2] column-
+ * steps that ran the eqs.(1)(2) update (neither refractory nor inhibited: the LIF work that cannot be
+ * skipped), since the handle was created.
  *
  * snn_label (R22): labels[j] (n_exc int32) = the class c maximising the MEAN count of neuron j over
  * the labelling images of class c (counts: n_images x n_exc u32, classes: n_images int32 in
@@ -249,7 +258,7 @@ int snn_shard_link(snn_handle* const* hs, int world);
  * exactly (integer cross products).  Pointers host or device; synchronous. */
 int snn_infer(snn_handle* h, const uint8_t* images, int n_images, int T, const uint64_t* seeds, uint32_t* counts,
               int flags);
-int snn_get_infer_stats(snn_handle* h, uint64_t stats[2]);
+int snn_get_infer_stats(snn_handle* h, uint64_t stats[3]);
 int snn_label(snn_handle* h, const uint32_t* counts, int n_images, const int32_t* classes, int n_classes,
               int32_t* labels);
 int snn_classify(snn_handle* h, const uint32_t* counts, int n_images, const int32_t* labels, int n_classes,

@@ -96,6 +96,10 @@ struct snn_handle {
   bool last_recorded = false;
   int t_next = 0;
   long long launches = 0;
+  // snn_set_profile: CUDA events recorded on the handle's stream around every presentation kernel
+  bool prof = false;
+  std::vector<cudaEvent_t> prof_ev;    // pairs (start, stop)
+  size_t prof_used = 0;
   // event engine
   int engine = SNN_ENGINE_EVENT;
   int rows_cap = 0, offs_cap = 0, logn = 0;
@@ -220,6 +224,8 @@ void free_all(snn_handle* h) {
                   h->d_lab, h->d_istats, h->d_soff, h->d_stgt, h->d_sq, h->d_scounts, h->d_sraster,
                   h->d_sstats};
   for (void* q : ptrs) if (q) cudaFree(q);
+  for (cudaEvent_t e : h->prof_ev) cudaEventDestroy(e);
+  h->prof_ev.clear();
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
 }
 
@@ -300,6 +306,18 @@ int event_prepass(snn_handle* h, NetDesc& d, const uint8_t* images, const uint32
   return SNN_OK;
 }
 
+// snn_set_profile: record an event on the launching stream (pairs around each presentation kernel)
+constexpr size_t kProfMaxEvents = 8192;
+void prof_mark(snn_handle* h) {
+  if (!h->prof || h->prof_used >= kProfMaxEvents) return;
+  if (h->prof_used == h->prof_ev.size()) {
+    cudaEvent_t e;
+    if (cudaEventCreate(&e) != cudaSuccess) { cudaGetLastError(); h->prof = false; return; }
+    h->prof_ev.push_back(e);
+  }
+  cudaEventRecord(h->prof_ev[h->prof_used++], h->stream);
+}
+
 // Common path of every single-handle presentation.
 int present_impl(snn_handle* h, const void* input, int n_images, int T, const uint64_t* seeds, int32_t* counts,
                  int flags, int t0) {
@@ -314,7 +332,8 @@ int present_impl(snn_handle* h, const void* input, int n_images, int T, const ui
     return fail(SNN_EINVAL, "SNN_KEEP_STATE with t0 = %d before the stored state's next step %d", t0, h->t_next);
   const bool ev = h->engine == SNN_ENGINE_EVENT;
   if (ev && T > snn::kEvMaxT) return fail(SNN_EINVAL, "T=%d exceeds %d for the event engine", T, snn::kEvMaxT);
-  if (ev && (flags & SNN_FLOOR_PROBE)) return fail(SNN_EINVAL, "SNN_FLOOR_PROBE applies to the per-step engine");
+  if (ev && (flags & SNN_FLOOR_PROBE) && !h->lean)
+    return fail(SNN_EINVAL, "SNN_FLOOR_PROBE applies to the per-step engine and the lean event kernel");
   if (n_images == 0) {   // nothing to present (a T == 0 presentation still runs: it resets the state, R5)
     h->last_T = 0;
     return SNN_OK;
@@ -366,16 +385,27 @@ int present_impl(snn_handle* h, const void* input, int n_images, int T, const ui
     rc = event_prepass(h, d, img, rin, n_images, T, (flags & SNN_KEEP_STATE) ? t0 : 0, sd);
     if (rc) return rc;
     if ((rc = shard_arm(h, d))) return rc;
+    if (flags & SNN_FLOOR_PROBE) {       // the handle's mean epochs per image so far (stats [8] / [6])
+      unsigned long long st[SNN_NSTATS];
+      CUDA_TRY(cudaMemcpyAsync(st, h->d_stats, sizeof(st), cudaMemcpyDeviceToHost, h->stream));
+      CUDA_TRY(cudaStreamSynchronize(h->stream));
+      if (st[6] == 0) return fail(SNN_EINVAL, "SNN_FLOOR_PROBE needs learning presentations first (epochs per image)");
+      d.floor_epochs = (int)((st[8] + st[6] / 2) / st[6]);
+    }
     lp.single = d;
+    prof_mark(h);
     if (h->lean)
       CUDA_TRY(snn::launch_present_lean(lp, 1, h->cs, h->nthr, h->smem_lean, h->bits, h->cpt, h->p.membrane_mode,
                                         h->stream));
     else
       CUDA_TRY(snn::launch_present_event_mode(lp, 1, h->cs, h->nthr, h->smem, h->bits, h->cpt, h->p.membrane_mode,
                                               h->stream));
+    prof_mark(h);
   } else {
     lp.single = d;
+    prof_mark(h);
     CUDA_TRY(snn::launch_present(lp, 1, h->cs, h->nthr, h->smem, h->stream));
+    prof_mark(h);
   }
   h->launches++;
   if (counts && !counts_dev)
@@ -1068,6 +1098,32 @@ int snn_get_stats(snn_handle* h, uint64_t stats[SNN_NSTATS]) {
   return SNN_OK;
 }
 
+int snn_set_profile(snn_handle* h, int on) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  h->prof = on != 0;
+  h->prof_used = 0;
+  return SNN_OK;
+}
+
+int snn_get_profile(snn_handle* h, double* kernel_ms, int64_t* kernels) {
+  int rc = check_handle(h);
+  if (rc) return rc;
+  if (!kernel_ms || !kernels) return fail(SNN_EINVAL, "kernel_ms / kernels is NULL");
+  DevGuard g(h->dev);
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  double ms = 0.0;
+  for (size_t k = 0; k + 1 < h->prof_used; k += 2) {
+    float x = 0.f;
+    CUDA_TRY(cudaEventElapsedTime(&x, h->prof_ev[k], h->prof_ev[k + 1]));
+    ms += x;
+  }
+  *kernel_ms = ms;
+  *kernels = (int64_t)(h->prof_used / 2);
+  h->prof_used = 0;
+  return SNN_OK;
+}
+
 int snn_reset_stats(snn_handle* h) {
   int rc = check_handle(h);
   if (rc) return rc;
@@ -1178,8 +1234,8 @@ int snn_infer(snn_handle* h, const uint8_t* images, int n_images, int T, const u
   if ((rc = infer_geometry(h, &wpr, &R, &nthr, &smem))) return rc;
   if ((rc = infer_weights(h, wpr))) return rc;
   if (!h->d_istats) {
-    CUDA_TRY(dalloc(&h->d_istats, 2));
-    CUDA_TRY(cudaMemsetAsync(h->d_istats, 0, 2 * sizeof(unsigned long long), h->stream));
+    CUDA_TRY(dalloc(&h->d_istats, 3));
+    CUDA_TRY(cudaMemsetAsync(h->d_istats, 0, 3 * sizeof(unsigned long long), h->stream));
   }
   const uint8_t* img = nullptr;
   if ((rc = stage(h, images, (size_t)n_images * h->n_in, &h->d_img, &h->img_cap, &img))) return rc;
@@ -1237,14 +1293,14 @@ int snn_infer(snn_handle* h, const uint8_t* images, int n_images, int T, const u
   return finish(h, flags);
 }
 
-int snn_get_infer_stats(snn_handle* h, uint64_t stats[2]) {
+int snn_get_infer_stats(snn_handle* h, uint64_t stats[3]) {
   int rc = check_handle(h);
   if (rc) return rc;
   if (!stats) return fail(SNN_EINVAL, "stats is NULL");
-  stats[0] = stats[1] = 0;
+  stats[0] = stats[1] = stats[2] = 0;
   if (!h->d_istats) return SNN_OK;
   DevGuard g(h->dev);
-  CUDA_TRY(cudaMemcpyAsync(stats, h->d_istats, 2 * sizeof(uint64_t), cudaMemcpyDeviceToHost, h->stream));
+  CUDA_TRY(cudaMemcpyAsync(stats, h->d_istats, 3 * sizeof(uint64_t), cudaMemcpyDeviceToHost, h->stream));
   CUDA_TRY(cudaStreamSynchronize(h->stream));
   return SNN_OK;
 }

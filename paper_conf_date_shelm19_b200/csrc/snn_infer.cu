@@ -224,7 +224,7 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
   lif.af = d.af; lif.bf = d.bf; lif.cf = d.cf; lif.dtf = d.dtf; lif.kI = d.kI; lif.ief = d.ief; lif.vthf = d.vthf;
   lif.A = d.A; lif.B = d.B; lif.C = d.C; lif.E = d.E; lif.Vth = d.Vth; lif.fixed = FIXED;
   const bool consumer = !is_producer && tcol < d.nthr_cols;
-  unsigned long long act_sum = 0, spikes = 0;
+  unsigned long long act_sum = 0, spikes = 0, lif_cs = 0;   // lif_cs: column-steps that ran eqs.(1)(2)
 
   if (is_producer) {
     // the producer runs decoupled from the consumers' step barriers: it publishes step records (release) and
@@ -302,11 +302,12 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
         if ((int)tt >= my_max_free) {                             // no column of this thread is held
 #pragma unroll
           for (int c = 0; c < 32; ++c) cross |= lif.step_t<FIXED>(v[c], SW::get(acc, c));
+          lif_cs += 32;
         } else {
 #pragma unroll
           for (int c = 0; c < 32; ++c) {
             const uint32_t f = (fr[c >> 1] >> ((c & 1) * 16)) & 0xFFFFu;
-            if (tt >= f) cross |= lif.step_t<FIXED>(v[c], SW::get(acc, c));   // held: keep v (R6, R7)
+            if (tt >= f) { cross |= lif.step_t<FIXED>(v[c], SW::get(acc, c)); ++lif_cs; }   // held: keep v (R6, R7)
           }
         }
         if (cross) {
@@ -339,6 +340,7 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
               S += (int)((__ldg(&d.w[(size_t)i * d.wpr + tcol * BITS + kw]) >> sh) & ((1u << BITS) - 1u));
             }
           }
+          ++lif_cs;
           if (lif.step_t<FIXED>(v[c], S)) {
             const unsigned long long key = ((unsigned long long)lif.ord(v[c]) << 32) | (0xFFFFFFFFu - (uint32_t)(j0 + c));
             best = key > best ? key : best;
@@ -415,6 +417,7 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
     atomicAdd(&d.stats[0], act_sum);
   }
   if (d.stats && consumer && spikes) atomicAdd(&d.stats[1], spikes);
+  if (d.stats && consumer && lif_cs) atomicAdd(&d.stats[2], lif_cs);
 }
 
 // Pack u8 codes [n_in][n_exc] into the inference layout: row i, word q = column-thread q / BITS ...

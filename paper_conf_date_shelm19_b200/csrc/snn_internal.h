@@ -62,6 +62,7 @@ struct NetDesc {
   const uint16_t* ev_rows16;           // [n_images][T][kPadRows] first kPadRows rows of each step, padded with n_in
   long long rows_stride;
   int rows_cap, offs_cap, logn;        // on-chip window of the lists, per-thread LTD undo-log entries
+  int floor_epochs;                    // SNN_FLOOR_PROBE on the lean kernel: skeleton epochs per image
   // optional per-epoch trace: [cs][trace_cap][8] u64 (%globaltimer ns)
   unsigned long long* trace;
   int trace_cap;
@@ -140,7 +141,7 @@ struct InferDesc {
   const uint32_t* w;                 // [n_in][wpr] codes, column j at word j / (32/bits), bits (j % (32/bits)) * bits
   const uint32_t* words;             // [n_images][T][nwi] encoded input spikes
   uint32_t* counts;                  // [n_images][n_exc] spike counts (zeroed by the caller)
-  unsigned long long* stats;         // [2] += sum_t act(t), post spikes (may be null)
+  unsigned long long* stats;         // [3] += sum_t act(t), post spikes, LIF column-steps run (may be null)
 };
 size_t infer_smem_bytes(int R, int row_bytes);
 cudaError_t infer_occupancy(int bits, int fixed, int minb, int nthr, size_t smem, int* out);

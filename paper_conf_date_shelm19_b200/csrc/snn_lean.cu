@@ -209,6 +209,50 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
   if (cs > 1) { cluster_arrive(); cluster_wait(); } else { __syncthreads(); }
 
   int ep = 0;
+  if (flags & FLAG_FLOOR) {
+    // latency floor probe (SNN_FLOOR_PROBE, bench.py latency_roofline): the same launch shape runs, per image,
+    // d.floor_epochs epochs of the synchronisation skeleton alone -- the early-stop signal to every CTA, the
+    // warp and CTA summaries, the DSMEM summary stores, the cluster barrier and the decision -- with no
+    // integration, LIF or STDP
+    unsigned long long chk = 0ull;
+    for (int b = 0; b < n_images; ++b) {
+      for (int e = 0; e < d.floor_epochs; ++e, ++ep) {
+        const int fp = ep & 1;
+        const int cst = (rank == (e % cs) && warp == 0) ? e : kNoStep;
+        if (rank == (e % cs) && warp == 0 && lane < cs) {
+          if (lane == rank) atomicMin(&s_flag[fp], e);
+          else red_min_cluster(&s_flag[fp], (uint32_t)lane, e);
+        }
+        const int wc = __reduce_min_sync(FULL, cst);
+        const uint32_t kh = __reduce_max_sync(FULL, (uint32_t)(tid + e));
+        if (lane == 0) { s_wsum[2 * warp] = ((unsigned long long)(uint32_t)wc << 32) | (uint32_t)kNoStep; s_wsum[2 * warp + 1] = kh; }
+        __syncthreads();
+        if (warp == 0) {
+          const unsigned long long a = lane < nwarps ? s_wsum[2 * lane] : ~0ull;
+          const unsigned long long k = lane < nwarps ? s_wsum[2 * lane + 1] : 0ull;
+          const int C = __reduce_min_sync(FULL, (int)(a >> 32));
+          const uint32_t K2 = __reduce_max_sync(FULL, (uint32_t)k);
+          unsigned long long* slot = s_slots + (size_t)(fp * kMaxCluster + rank) * 2;
+          const unsigned long long A = ((unsigned long long)(uint32_t)C << 32) | (uint32_t)kNoStep;
+          if (cs == 1) {
+            if (lane == 0) { slot[0] = A; slot[1] = K2; }
+          } else if (lane < cs) {
+            st_cluster_u64(slot, (uint32_t)lane, A);
+            st_cluster_u64(slot + 1, (uint32_t)lane, K2);
+          }
+          if (lane == 0) s_flag[fp ^ 1] = INT_MAX;
+        }
+        if (cs > 1) { cluster_arrive(); cluster_wait(); } else { __syncthreads(); }
+        const unsigned long long A = lane < cs ? s_slots[(size_t)(fp * kMaxCluster + lane) * 2] : ~0ull;
+        const int Pf = __reduce_min_sync(FULL, (int)(A >> 32));
+        chk += (unsigned long long)Pf;
+      }
+      if (rank == 0 && tid == 0 && d.spike_counts) d.spike_counts[b] = 0;
+    }
+    if (tid == 0 && chk == 0xFFFFFFFFFFFFFFFFull) d.stats[15] = chk;   // keeps the skeleton's results live
+    if (cs > 1) { cluster_arrive(); cluster_wait(); }
+    return;
+  }
   for (int b = 0; b < n_images; ++b) {
     const unsigned long long seed = d.seeds[b];
     if (!keep) {

@@ -22,7 +22,7 @@ EXPORTS = [
     "snn_present", "snn_present_batch", "snn_present_ex", "snn_present_raster", "snn_present_many",
     "snn_get_weights", "snn_set_weights", "snn_get_spikes", "snn_get_input_raster",
     "snn_state_bytes", "snn_get_state", "snn_set_state", "snn_get_stats", "snn_reset_stats",
-    "snn_get_info", "snn_set_trace", "snn_get_trace", "snn_last_error",
+    "snn_get_info", "snn_set_trace", "snn_get_trace", "snn_set_profile", "snn_get_profile", "snn_last_error",
     "snn_create_shard", "snn_shard_ipc_handle", "snn_shard_connect", "snn_shard_link",
     "snn_infer", "snn_get_infer_stats", "snn_label", "snn_classify",
     "snn_sparse_run", "snn_get_sparse_stats",
@@ -91,6 +91,8 @@ def lib():
             "snn_get_info": ([vp, vp], i32),
             "snn_set_trace": ([vp, i32], i32),
             "snn_get_trace": ([vp, vp, sz], i32),
+            "snn_set_profile": ([vp, i32], i32),
+            "snn_get_profile": ([vp, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_int64)], i32),
             "snn_last_error": ([], ctypes.c_char_p),
             "snn_create_shard": ([i32, i32, i32, pp, i32, i32, ctypes.POINTER(vp)], i32),
             "snn_shard_ipc_handle": ([vp, vp, sz], i32),
@@ -285,6 +287,16 @@ class Network:
     def reset_stats(self):
         _check(lib().snn_reset_stats(self._h), "snn_reset_stats")
 
+    def set_profile(self, on: bool = True):
+        """CUDA events around every presentation kernel on the handle's stream (include/snn.h)."""
+        _check(lib().snn_set_profile(self._h, 1 if on else 0), "snn_set_profile")
+
+    def profile(self):
+        """-> (summed presentation-kernel milliseconds, kernels) since the last call; resets."""
+        ms, n = ctypes.c_double(0.0), ctypes.c_int64(0)
+        _check(lib().snn_get_profile(self._h, ctypes.byref(ms), ctypes.byref(n)), "snn_get_profile")
+        return ms.value, n.value
+
     # ---- NEXT-1: inference with frozen weights, labelling, vote (include/snn.h, DESIGN.md §4.6)
     def infer(self, images, T: int, seeds, counts=None, flags: int = 0):
         """Spike counts (n_images, n_exc) u32 of each image presented with frozen weights.  images/seeds/
@@ -296,7 +308,8 @@ class Network:
         return counts
 
     def infer_stats(self) -> np.ndarray:
-        out = np.zeros(2, dtype=np.uint64)
+        """[active input rows, post spikes, LIF column-steps run] summed over every inference call."""
+        out = np.zeros(3, dtype=np.uint64)
         _check(lib().snn_get_infer_stats(self._h, _ptr(out)), "snn_get_infer_stats")
         return out
 
