@@ -396,7 +396,7 @@ int present_impl(snn_handle* h, const void* input, int n_images, int T, const ui
     prof_mark(h);
     if (h->lean)
       CUDA_TRY(snn::launch_present_lean(lp, 1, h->cs, h->nthr, h->smem_lean, h->bits, h->cpt, h->p.membrane_mode,
-                                        h->stream));
+                                        h->world > 1, h->stream));
     else
       CUDA_TRY(snn::launch_present_event_mode(lp, 1, h->cs, h->nthr, h->smem, h->bits, h->cpt, h->p.membrane_mode,
                                               h->stream));
@@ -526,7 +526,7 @@ int create_impl(int n_in, int n_exc, int bits, const snn_params* p, int col_base
   h->engine = (p->engine == SNN_ENGINE_STEP || bits > 8) ? SNN_ENGINE_STEP : SNN_ENGINE_EVENT;
   // the lean kernel covers the paper's default learning mode; SNN_NO_LEAN=1 disables it
   const bool lean_mode = p->engine == SNN_ENGINE_EVENT && bits <= 8 && p->wta_mode == SNN_WTA_HARD &&
-                         p->inh_mode == SNN_INH_RESET && p->stdp_mode == SNN_STDP_STOCH && world == 1 &&
+                         p->inh_mode == SNN_INH_RESET && p->stdp_mode == SNN_STDP_STOCH &&
                          !(getenv("SNN_NO_LEAN") && atoi(getenv("SNN_NO_LEAN")) != 0);
   int chosen = 0;
   const bool ev = h->engine == SNN_ENGINE_EVENT;
@@ -948,7 +948,7 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
       if (hs[k]->cpt != hs[g[0]]->cpt) { e = cudaErrorInvalidValue; break; }
     if (e != cudaSuccess) break;
     e = lean ? snn::launch_present_lean(lp, (int)g.size(), h0->cs, hs[g[0]]->nthr, smem, hs[g[0]]->bits,
-                                        hs[g[0]]->cpt, h0->p.membrane_mode, st)
+                                        hs[g[0]]->cpt, h0->p.membrane_mode, hs[g[0]]->world > 1, st)
         : ev ? snn::launch_present_event_mode(lp, (int)g.size(), h0->cs, hs[g[0]]->nthr, smem, hs[g[0]]->bits,
                                               hs[g[0]]->cpt, h0->p.membrane_mode, st)
              : snn::launch_present(lp, (int)g.size(), h0->cs, h0->nthr, smem, st);

@@ -70,7 +70,7 @@ __host__ __device__ inline LeanLayout lean_layout(int n_in, int slice_words, int
   L.slots = o; o = align16(o + 2 * kMaxCluster * 2 * 8);     // [parity][rank][2] u64: steps, key
   L.wsum = o;  o = align16(o + 32 * 2 * 8);                  // per warp: steps, key
   L.flags = o; o = align16(o + 4 * 4);                       // early-stop flag per epoch parity
-  L.misc = o;  o = align16(o + 32 * 4);
+  L.misc = o;  o = align16(o + 40 * 4);
   L.dS = o;    o = align16(o + (size_t)kDefSteps * 4);                // deferred column: S per table step
   L.dbits = o; o = align16(o + (size_t)(kDefRowsPerThr * nthr / 32) * 4);   // deferred column: event bit per raw row
   L.dev = o;   o = align16(o + (size_t)n_in * 8 * 2);                 // deferred column: event steps per input row (x2)
@@ -103,7 +103,8 @@ size_t lean_smem_bytes(int n_in, int slice_words, int L_pot, int L_dep, int nthr
   return lean_layout(n_in, slice_words, L_pot, L_dep, nthr, rows_cap, offs_cap, logn).total;
 }
 
-template <int BITS, int CPT_, bool FIXED>
+// SH: compiled with the cross-rank (column-sharded) exchange; the unsharded instance carries none of it
+template <int BITS, int CPT_, bool FIXED, bool SH>
 __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __grid_constant__ LaunchParams lp) {
   using Z = LSwar<BITS, CPT_>;
   constexpr int CPT = Z::CPT;
@@ -209,6 +210,11 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
   if (cs > 1) { cluster_arrive(); cluster_wait(); } else { __syncthreads(); }
 
   int ep = 0;
+  // column sharding: this cluster holds columns [cbase, cbase + n_exc) of a network split over
+  // `world` ranks; per epoch the cluster summaries meet in every rank's device mailbox
+  const int world = d.world;
+  const bool sharded = SH && world > 1;
+  const uint32_t seq0 = sharded ? (uint32_t)ld_relaxed_sys_s32(reinterpret_cast<const int*>(&d.mbox->seq)) : 0u;
   if (flags & FLAG_FLOOR) {
     // latency floor probe (SNN_FLOOR_PROBE, bench.py latency_roofline): the same launch shape runs, per image,
     // d.floor_epochs epochs of the synchronisation skeleton alone -- the early-stop signal to every CTA, the
@@ -525,12 +531,15 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
       };
 
       // a crossing at window step kc: lower the early-stop flag of every CTA of the cluster (lane r -> CTA r)
+      const uint32_t cur = seq0 + (uint32_t)ep + 1u;        // shard-exchange epoch number (never 0 in use)
       auto signal_cross = [&](int kc) {
         if (trace && lane == 0) atomicMin(&s_trcross[fp], globaltimer());
         if (lane < cs) {
           if (lane == rank) atomicMin(&s_flag[fp], kc);
           else red_min_cluster(&s_flag[fp], (uint32_t)lane, kc);
         }
+        if (sharded && lane < world && lane != d.shard)      // lane r -> rank r (NVLink peer reduction)
+          red_max_sys_u64(&d.peers[lane]->flag, ((unsigned long long)cur << 32) | (0xFFFFFFFFu - (uint32_t)kc));
       };
 
       // LTD draws of every (lane, column) pair of the warp for raw rows [base, base + 64): lanes over rows,
@@ -654,6 +663,10 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         // one lane's read of the early-stop flag decides for the warp (lanes that executed the load apart
         // could otherwise see different values and leave the loop apart); read fresh every iteration: an
         // iteration may be a block of steps, so a stale value would let the warp overrun t* by a whole block
+        if (sharded && lane == 0) {        // the other ranks' early-stop signals for this epoch
+          const unsigned long long gf = ld_relaxed_sys_u64(&d.mbox->flag);
+          if ((uint32_t)(gf >> 32) == cur) atomicMin(&s_flag[fp], (int)(0xFFFFFFFFu - (uint32_t)gf));
+        }
         const int fl = __shfl_sync(FULL, ld_volatile_shared_u32addr(flag_addr), 0);
         if (kk >= kstop || kk > fl) break;                       // warp-uniform
         if (kTraceCycles && trace) t_it = clock64();
@@ -895,11 +908,10 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         if (__any_sync(FULL, cm != 0)) { signal_cross(kk); break; }
         ++kk;
       }
-      if (hstep != kNoStep) {                                    // tell the cluster where to stop
-        ++eng_hz;
-        atomicMin(&s_flag[fp], hstep - 1);
-        for (int r = 0; r < cs; ++r)
-          if (r != rank) red_min_cluster(&s_flag[fp], (uint32_t)r, hstep - 1);
+      {                                                          // tell the cluster (and the ranks) where to stop
+        const int hw = __reduce_min_sync(FULL, hstep);
+        if (hstep != kNoStep) ++eng_hz;
+        if (hw != kNoStep) signal_cross(hw - 1);
       }
       p_done = max(p_done, p_look);
       if (valid) eng_spec += (uint32_t)(p_done - k0 + 1) * (uint32_t)__popc(valid);
@@ -963,6 +975,54 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         const uint32_t kh = __reduce_max_sync(FULL, c == P ? (uint32_t)(Kr >> 32) : 0u);
         const uint32_t kl = __reduce_max_sync(FULL, (c == P && (uint32_t)(Kr >> 32) == kh) ? (uint32_t)Kr : 0u);
         K = ((unsigned long long)kh << 32) | kl;
+      }
+      if (sharded) {
+        // the cluster's summary {P, H, K} goes to slot [cur & 1][shard] of every rank's mailbox as four LL words
+        // (NVLink peer stores, no fence); warp 0 of every CTA polls its own mailbox for the world's summaries and
+        // applies the same reduction as the cluster exchange
+        const int mp = (int)(cur & 1u);
+        const unsigned long long tag = (unsigned long long)cur << 32;
+        if (rank == 0 && warp == 0 && lane < world) {
+          unsigned long long* sl = d.peers[lane]->slot[mp][d.shard];
+          st_relaxed_sys_u64(sl, tag | (uint32_t)P);
+          st_relaxed_sys_u64(sl + 1, tag | (uint32_t)H);
+          st_relaxed_sys_u64(sl + 2, tag | (uint32_t)(K >> 32));
+          st_relaxed_sys_u64(sl + 3, tag | (uint32_t)K);
+        }
+        if (warp == 0) {
+          int c = kNoStep, h = kNoStep;
+          unsigned long long Kr = 0ull;
+          if (lane < world) {
+            const unsigned long long* sl = d.mbox->slot[mp][lane];
+            const unsigned long long t_start = globaltimer();
+            unsigned long long w0, w1, w2, w3;
+            while (true) {
+              w0 = ld_relaxed_sys_u64(sl); w1 = ld_relaxed_sys_u64(sl + 1);
+              w2 = ld_relaxed_sys_u64(sl + 2); w3 = ld_relaxed_sys_u64(sl + 3);
+              if ((uint32_t)(w0 >> 32) == cur && (uint32_t)(w1 >> 32) == cur && (uint32_t)(w2 >> 32) == cur &&
+                  (uint32_t)(w3 >> 32) == cur) break;
+              if (globaltimer() - t_start > kShardTimeoutNs) __trap();   // a rank is gone: fail, never hang
+            }
+            c = (int)(uint32_t)w0; h = (int)(uint32_t)w1;
+            Kr = ((unsigned long long)(uint32_t)w2 << 32) | (uint32_t)w3;
+          }
+          const int Pg = __reduce_min_sync(FULL, c);
+          const int Hg = __reduce_min_sync(FULL, h);
+          const uint32_t kh = __reduce_max_sync(FULL, c == Pg ? (uint32_t)(Kr >> 32) : 0u);
+          const uint32_t kl = __reduce_max_sync(FULL, (c == Pg && (uint32_t)(Kr >> 32) == kh) ? (uint32_t)Kr : 0u);
+          // (own words: the next write comes after the next cluster barrier, which every thread reaches after
+          // reading these)
+          unsigned long long* s_world = reinterpret_cast<unsigned long long*>(s_misc + 32);
+          if (lane == 0) {
+            s_world[0] = ((unsigned long long)(uint32_t)Pg << 32) | (uint32_t)Hg;
+            s_world[1] = ((unsigned long long)kh << 32) | kl;
+          }
+        }
+        __syncthreads();
+        const unsigned long long* s_world = reinterpret_cast<const unsigned long long*>(s_misc + 32);
+        P = (int)(s_world[0] >> 32);
+        H = (int)(uint32_t)s_world[0];
+        K = s_world[1];
       }
       const bool event = P < kend && P < H;          // a post spike at t* = P
 #ifdef SNN_LEAN_DEBUG
@@ -1190,18 +1250,19 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
 #ifdef SNN_LEAN_DEBUG
   if (tid == 0) printf("END r %d\n", rank);
 #endif
+  if (sharded && rank == 0 && tid == 0) d.mbox->seq = seq0 + (uint32_t)ep;   // every CTA read seq0 long ago
   if (cs > 1) { cluster_arrive(); cluster_wait(); }
 }
 
 // ====================================================================== host launchers
-template <int BITS, int CPT, bool FIXED>
+template <int BITS, int CPT, bool FIXED, bool SH>
 static cudaError_t lean_launch_t(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, cudaStream_t s,
                                  int* occupancy_out) {
-  cudaError_t e = cudaFuncSetAttribute(present_lean_kernel<BITS, CPT, FIXED>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)smem);
+  auto* kern = present_lean_kernel<BITS, CPT, FIXED, SH>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   if (cs > 8) {
-    e = cudaFuncSetAttribute(present_lean_kernel<BITS, CPT, FIXED>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+    e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
     if (e != cudaSuccess) return e;
   }
   cudaLaunchConfig_t cfg = {};
@@ -1220,41 +1281,44 @@ static cudaError_t lean_launch_t(const LaunchParams& lp, int n_nets, int cs, int
     cfg.numAttrs = 1;
   }
   if (occupancy_out) {
-    if (cs == 1) return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occupancy_out, present_lean_kernel<BITS, CPT, FIXED>, nthr, smem);
-    return cudaOccupancyMaxActiveClusters(occupancy_out, present_lean_kernel<BITS, CPT, FIXED>, &cfg);
+    if (cs == 1) return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occupancy_out, kern, nthr, smem);
+    return cudaOccupancyMaxActiveClusters(occupancy_out, kern, &cfg);
   }
-  return cudaLaunchKernelEx(&cfg, present_lean_kernel<BITS, CPT, FIXED>, lp);
+  return cudaLaunchKernelEx(&cfg, kern, lp);
 }
 
 template <int BITS, int CPT>
-static cudaError_t lean_dispatch_f(int fixed, const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem,
+static cudaError_t lean_dispatch_f(int fixed, int sh, const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem,
                                    cudaStream_t s, int* occ) {
-  return fixed ? lean_launch_t<BITS, CPT, true>(lp, n_nets, cs, nthr, smem, s, occ)
-               : lean_launch_t<BITS, CPT, false>(lp, n_nets, cs, nthr, smem, s, occ);
+  if (sh)
+    return fixed ? lean_launch_t<BITS, CPT, true, true>(lp, n_nets, cs, nthr, smem, s, occ)
+                 : lean_launch_t<BITS, CPT, false, true>(lp, n_nets, cs, nthr, smem, s, occ);
+  return fixed ? lean_launch_t<BITS, CPT, true, false>(lp, n_nets, cs, nthr, smem, s, occ)
+               : lean_launch_t<BITS, CPT, false, false>(lp, n_nets, cs, nthr, smem, s, occ);
 }
 
-static cudaError_t lean_dispatch(int bits, int cpt, int fixed, const LaunchParams& lp, int n_nets, int cs, int nthr,
-                                 size_t smem, cudaStream_t s, int* occ) {
+static cudaError_t lean_dispatch(int bits, int cpt, int fixed, int sh, const LaunchParams& lp, int n_nets, int cs,
+                                 int nthr, size_t smem, cudaStream_t s, int* occ) {
   if (bits == 2) {
-    if (cpt == 4) return lean_dispatch_f<2, 4>(fixed, lp, n_nets, cs, nthr, smem, s, occ);
-    if (cpt == 1) return lean_dispatch_f<2, 1>(fixed, lp, n_nets, cs, nthr, smem, s, occ);
-    return lean_dispatch_f<2, 2>(fixed, lp, n_nets, cs, nthr, smem, s, occ);
+    if (cpt == 4) return lean_dispatch_f<2, 4>(fixed, sh, lp, n_nets, cs, nthr, smem, s, occ);
+    if (cpt == 1) return lean_dispatch_f<2, 1>(fixed, sh, lp, n_nets, cs, nthr, smem, s, occ);
+    return lean_dispatch_f<2, 2>(fixed, sh, lp, n_nets, cs, nthr, smem, s, occ);
   }
   if (bits == 4) {
-    if (cpt == 1) return lean_dispatch_f<4, 1>(fixed, lp, n_nets, cs, nthr, smem, s, occ);
-    return lean_dispatch_f<4, 2>(fixed, lp, n_nets, cs, nthr, smem, s, occ);
+    if (cpt == 1) return lean_dispatch_f<4, 1>(fixed, sh, lp, n_nets, cs, nthr, smem, s, occ);
+    return lean_dispatch_f<4, 2>(fixed, sh, lp, n_nets, cs, nthr, smem, s, occ);
   }
-  return lean_dispatch_f<8, 1>(fixed, lp, n_nets, cs, nthr, smem, s, occ);
+  return lean_dispatch_f<8, 1>(fixed, sh, lp, n_nets, cs, nthr, smem, s, occ);
 }
 
 cudaError_t query_max_clusters_lean(int bits, int cpt, int fixed, int cs, int nthr, size_t smem, int* out) {
   LaunchParams lp{};
-  return lean_dispatch(bits, cpt, fixed, lp, 1, cs, nthr, smem, 0, out);
+  return lean_dispatch(bits, cpt, fixed, 0, lp, 1, cs, nthr, smem, 0, out);
 }
 
 cudaError_t launch_present_lean(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, int bits, int cpt,
-                                int fixed, cudaStream_t s) {
-  return lean_dispatch(bits, cpt, fixed, lp, n_nets, cs, nthr, smem, s, nullptr);
+                                int fixed, int sharded, cudaStream_t s) {
+  return lean_dispatch(bits, cpt, fixed, sharded, lp, n_nets, cs, nthr, smem, s, nullptr);
 }
 
 }  // namespace snn
