@@ -12,7 +12,10 @@ Multi-GPU (torchrun, N > 1), --mode:
   replicas (default): one independent network per GPU, no data-path collective ("scaling": "weak");
   shard: ONE network whose 6400 columns are split over the N GPUs (include/snn.h snn_create_shard):
          per post-spike epoch the shards exchange 16-byte summaries through CUDA-IPC mailboxes over
-         NVLink ("scaling": "strong": every rank presents the same images).
+         NVLink ("scaling": "strong": every rank presents the same images);
+  shard-weak: one network of 6400*N columns, 6400 per GPU, same exchange ("scaling": "weak");
+  ensemble: C5, --nets independent 784->400 networks per GPU (bits (2,4,8)[k%3]) presented with one
+         snn_present_many per step, replicas across GPUs (its own metric line).
 --local-shards K (N = 1): the one network split into K shards on this GPU, presented in one launch
 (K clusters exchanging through L2 mailboxes) -- more SMs per network.
 
@@ -220,6 +223,86 @@ def cpu_baseline(n_images: int) -> dict:
     return out
 
 
+def run_ensemble(args):
+    """C5: an ensemble of independent 784 -> 400 networks, --nets per GPU (bit widths (2,4,8)[k%3],
+    each with its Table I row, seed = global network index), MNIST-shaped images, T = 350.  Every rank presents
+    its own group with one snn_present_many per step (one launch per bit width); replicas across ranks with no
+    data-path collective ("scaling": "weak").  Device time (CUDA events on the launching stream), max over
+    ranks; value = images of all networks of all ranks / that time."""
+    import torch
+    import paper_conf_date_shelm19_b200 as P
+    ws, rank, local = _dist_env()
+    dev = torch.device("cuda", local % max(1, torch.cuda.device_count()))
+    torch.cuda.set_device(dev)
+    dist = None
+    if ws > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl" if torch.cuda.device_count() >= ws else "gloo",
+                                **({"device_id": dev} if torch.cuda.device_count() >= ws else {}))
+    stream = torch.cuda.Stream(dev)
+    torch.cuda.set_stream(stream)
+    B, NE = args.images_per_step, 400
+    nets, imgs, seeds = [], [], []
+    for k in range(args.nets):
+        g = rank * args.nets + k
+        bits = (2, 4, 8)[g % 3]
+        n = P.Network(N_IN, NE, bits, P.preset({2: "2b", 4: "4b", 8: "8b"}[bits], init_seed=1 + g, cluster_size=2))
+        n.set_stream(stream.cuda_stream)
+        nets.append(n)
+        tot = B * (args.warmup + args.steps)
+        imgs.append(torch.from_numpy(synthdata.images(tot, "mnist", start=10000 * g)).to(dev))
+        seeds.append(torch.from_numpy(synthdata.seeds(tot, base_seed=200 + g).view(np.int64)).to(dev))
+    flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=dev)
+    sl = lambda s: slice(s * B, (s + 1) * B)  # noqa: E731
+    for s in range(args.warmup):
+        P.present_many(nets, [x[sl(s)] for x in imgs], T_STEPS, [x[sl(s)] for x in seeds])
+    torch.cuda.synchronize()
+    for n in nets:
+        n.reset_stats()
+    sampler = ClockSampler(local)
+    sampler.start()
+    time.sleep(0.15)
+    if dist:
+        dist.barrier()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    for i in range(args.steps):
+        flush.fill_(i & 0xFF)
+        s = args.warmup + i
+        ev[i][0].record(stream)
+        P.present_many(nets, [x[sl(s)] for x in imgs], T_STEPS, [x[sl(s)] for x in seeds])
+        ev[i][1].record(stream)
+    torch.cuda.synchronize()
+    if dist:
+        dist.barrier()
+    clocks = sampler.stop()
+    dev_s = sum(a.elapsed_time(b) for a, b in ev) / 1e3
+    images = args.nets * B * args.steps
+    events = sum(int(n.stats()[0]) for n in nets) * NE
+    if dist:
+        t = torch.tensor([dev_s], dtype=torch.float64, device=dev if torch.cuda.device_count() >= ws else "cpu")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dev_s = float(t.item())
+        tot = torch.tensor([images, events], dtype=torch.float64, device=t.device)
+        dist.all_reduce(tot, op=dist.ReduceOp.SUM)
+        images, events = int(tot[0].item()), int(tot[1].item())
+    if rank == 0:
+        print(json.dumps({
+            "metric": "C5 ensemble training images/s (784->400, bits {2,4,8})", "value": images / dev_s,
+            "unit": "images/s", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1e3 * dev_s / args.steps, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f32/u2-u8", "data": "synthetic",
+            "config": {"workload": "C5: independent 784->400 networks, bits (2,4,8)[k%3], Table I rows, MNIST-shaped, "
+                                   "T=350", "nets_per_gpu": args.nets, "images_per_net_per_step": B,
+                       "parallelism": f"{args.nets} networks per GPU x {ws} GPU(s), replicas",
+                       "l2": "flushed between timed steps (256 MiB write)"},
+            "secondary": {"synaptic_events_per_s": events / dev_s, "per_net_images_per_s": images / dev_s /
+                          (args.nets * ws)},
+            "clocks": clocks}), flush=True)
+    if dist:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -232,7 +315,11 @@ def main():
     ap.add_argument("--cpu-images", type=int, default=10, help="oracle images for cpu_baseline (0 = skip)")
     ap.add_argument("--no-floor", action="store_true")
     ap.add_argument("--engine", type=int, default=0, help="0 event-driven epochs, 1 per-step exchange")
-    ap.add_argument("--mode", default="replicas", choices=["replicas", "shard"], help="N > 1 layout")
+    ap.add_argument("--mode", default="replicas", choices=["replicas", "shard", "shard-weak", "ensemble"],
+                    help="replicas: one C4 network per GPU; shard: ONE C4 network's 6400 columns split over the GPUs "
+                         "(strong); shard-weak: a 6400*N-column network, 6400 columns per GPU (weak); ensemble: C5, "
+                         "--nets 784->400 networks per GPU")
+    ap.add_argument("--nets", type=int, default=8, help="ensemble mode: networks per GPU")
     ap.add_argument("--local-shards", type=int, default=1, help="shards of the network on this GPU (N = 1)")
     ap.add_argument("--no-infer", action="store_true", help="skip the NEXT-1 inference measurement")
     ap.add_argument("--infer-images", type=int, default=4096, help="images per inference call")
@@ -241,6 +328,8 @@ def main():
         args.warmup = 3
     if args.impl == "reference":
         return run_reference(args)
+    if args.mode == "ensemble":
+        return run_ensemble(args)
 
     import torch
     import paper_conf_date_shelm19_b200 as P
@@ -264,7 +353,8 @@ def main():
     torch.cuda.set_stream(stream)
 
     B = args.images_per_step
-    sharded = ws > 1 and args.mode == "shard"
+    sharded = ws > 1 and args.mode in ("shard", "shard-weak")
+    n_exc_net = N_EXC * ws if (sharded and args.mode == "shard-weak") else N_EXC   # columns of the whole network
     K = args.local_shards if ws == 1 else 1
     net_rank = 0 if sharded else rank           # shards of one network share seeds and images
 
@@ -273,7 +363,7 @@ def main():
         params = P.preset("2b", membrane_mode=args.membrane, init_seed=1 + net_rank,
                           cluster_size=args.cluster_size, engine=args.engine)
         if sharded:
-            n = P.Network(N_IN, N_EXC, BITS, params, shard=(rank, ws))
+            n = P.Network(N_IN, n_exc_net, BITS, params, shard=(rank, ws))
             n.set_stream(stream.cuda_stream)
             hs = [None] * ws
             dist.all_gather_object(hs, n.ipc_handle())
@@ -350,7 +440,7 @@ def main():
         stats[2:6] += n.stats()[2:6]
     launches = sum(n.info()["launches"] for n in nets) - launches0
     images = B * args.steps
-    events = int(stats[0]) * N_EXC
+    events = int(stats[0]) * n_exc_net                 # every column of the network (all shards)
     # max over ranks of the device time
     if dist:
         t = torch.tensor([dev_s], device=coll_dev, dtype=torch.float64)
@@ -422,7 +512,8 @@ def main():
 
     # ---- roofline of the dominant kernel (present_kernel; one launch per step)
     bits_b = BITS / 8.0
-    alg_bytes = (int(stats[0]) * N_EXC * bits_b                       # integration reads (a2)
+    cols_here = n_exc_net // ws if sharded else N_EXC                  # columns this rank's kernel integrates
+    alg_bytes = (int(stats[0]) * cols_here * bits_b                   # integration reads (a2)
                  + (int(stats[2]) + int(stats[4])) * bits_b           # LTD/LTP trial reads (a5)
                  + (int(stats[3]) + int(stats[5])) * bits_b)          # conditional writes (a5)
     # dominant kernel = the presentation kernel (one launch per step); its time comes from the CUDA events the
@@ -502,10 +593,11 @@ def main():
     line = {
         "metric": METRIC, "value": value, "unit": "images/s", "n_gpus": ws, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": 1e3 * dev_s / args.steps, "higher_is_better": True,
-        "scaling": "strong" if sharded else "weak", "vs_baseline": None, "dtype": "f32/u2", "data": "synthetic",
-        "config": {"workload": WORKLOAD, "n_in": N_IN, "n_exc": N_EXC, "bits": BITS, "T": T_STEPS,
+        "scaling": "strong" if (sharded and args.mode == "shard") else "weak", "vs_baseline": None, "dtype": "f32/u2", "data": "synthetic",
+        "config": {"workload": WORKLOAD, "n_in": N_IN, "n_exc": n_exc_net, "bits": BITS, "T": T_STEPS,
                    "images_per_step": B,
-                   "parallelism": (f"1 network column-sharded over {ws} GPUs" if sharded else
+                   "parallelism": (f"1 network of {n_exc_net} columns, {n_exc_net // ws} per GPU over {ws} GPUs"
+                                   if sharded else
                                    f"replicas x{ws}" if ws > 1 else
                                    f"1 network in {K} shards on 1 GPU" if K > 1 else "1 network / 1 GPU"),
                    "cluster_size": info["cluster_size"], "threads_per_cta": info["threads"],
