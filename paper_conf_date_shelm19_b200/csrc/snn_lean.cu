@@ -735,9 +735,16 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
             uint32_t acc[kBlk];
 #pragma unroll
             for (int j = 0; j < kBlk; ++j) {
-              const uint4 m = *reinterpret_cast<const uint4*>(s_p8 + kSlots * (x + j));
-              const uint4 m2 = *reinterpret_cast<const uint4*>(s_p8 + kSlots * (x + j) + 4);
-              acc[j] = ((ldw(m.x) + ldw(m.y)) + (ldw(m.z) + ldw(m.w))) + ((ldw(m2.x) + ldw(m2.y)) + (ldw(m2.z) + ldw(m2.w)));
+              uint32_t a4[kSlots / 4];
+#pragma unroll
+              for (int g = 0; g < kSlots / 4; ++g) {
+                const uint4 m = *reinterpret_cast<const uint4*>(s_p8 + kSlots * (x + j) + 4 * g);
+                a4[g] = (ldw(m.x) + ldw(m.y)) + (ldw(m.z) + ldw(m.w));
+              }
+              uint32_t a = a4[0];
+#pragma unroll
+              for (int g = 1; g < kSlots / 4; ++g) a += a4[g];
+              acc[j] = a;
             }
             int yv[kBlk][CPT];
 #pragma unroll
