@@ -772,7 +772,9 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
                 if (lif.post_t<FIXED>(v[c], yv[j][c])) cm |= 1u << c;   // eq.(2): v > v_th
               }
               if (cm) {
-                cstep = kk + j;
+                // (the thread's deferred column may have reported a LATER crossing in its run ahead: an earlier
+                // one replaces its key, an equal one competes with it)
+                if (kk + j < cstep) { cstep = kk + j; ckey = 0ull; }
 #pragma unroll
                 for (int c = 0; c < CPT; ++c) {
                   if (!(cm >> c & 1u)) continue;
@@ -901,7 +903,7 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         }
         p_done = kk;
         if (cm) {                                                // crossing: the WTA key (R7)
-          cstep = kk;
+          if (kk < cstep) { cstep = kk; ckey = 0ull; }          // (see the block path)
 #pragma unroll
           for (int c = 0; c < CPT; ++c) {
             if (!(cm >> c & 1u)) continue;

@@ -357,3 +357,50 @@ def test_state_validation_matches_oracle(gpu):
         with pytest.raises(P.SnnError):
             g.set_state(b)
     g.set_state(st)
+
+
+def test_floor_probe_and_profile_leave_learning_untouched(gpu):
+    """bench.py's instruments: SNN_FLOOR_PROBE (the lean kernel's per-epoch synchronisation skeleton) changes no
+    code, state or learning counter, and profiling (CUDA events around the presentation kernel) does not change
+    results; the profile reports one kernel per presentation."""
+    import paper_conf_date_shelm19_b200 as P
+    p = O.params("2b", membrane_mode=1, init_seed=1)
+    g, o = _pair(784, 512, 2, p)
+    imgs, seeds = synthdata.images(6, "fashion", start=400), synthdata.seeds(6, base_seed=43)
+    g.set_profile(True)
+    g.present_batch(imgs[:3], 150, seeds[:3])
+    ms, n = g.profile()
+    assert n == 1 and ms > 0.0
+    w0, st0, s0 = g.weights(), g.state(), g.stats()[:13].copy()
+    counts = np.full(3, -1, np.int32)
+    g.present_batch(imgs[3:], 150, seeds[3:], counts, flags=P.snn.SNN_FLOOR_PROBE)
+    assert counts.tolist() == [0, 0, 0]
+    assert np.array_equal(g.weights(), w0) and np.array_equal(g.state(), st0)
+    assert np.array_equal(g.stats()[:13], s0)
+    g.set_profile(False)
+    for img, sd in zip(imgs[:3], seeds[:3]):
+        o.present(img, 150, int(sd))
+    assert np.array_equal(w0, o.weights())
+
+
+@pytest.mark.parametrize("mode", [0, 1])
+@pytest.mark.parametrize("start,base", [(400, 43), (0, 1), (123, 7), (777, 99), (2024, 5)])
+def test_lean_short_tables_shared_thread(gpu, mode, start, base):
+    """784 -> 512 at 2 bits on 16 CTAs of ONE warp: the deferred column's tables cover only ~5 steps (32 raw
+    rows), so epochs end at table ends, re-simulations are frequent, and the deferred column often shares its
+    thread with the next winner (regression: a later crossing reported by the deferred column's run ahead must
+    not lend its key to an earlier crossing of the thread's other column)."""
+    p = O.params("2b", membrane_mode=mode, init_seed=1)
+    g, o = _pair(784, 512, 2, p)
+    assert g.info()["threads"] == 32 and g.info()["lean"] == 1
+    imgs, seeds = synthdata.images(4, "fashion", start=start), synthdata.seeds(4, base_seed=base)
+    counts = np.zeros(4, np.int32)
+    g.present_batch(imgs, 144, seeds, counts)
+    oc = []
+    for x, s in zip(imgs, seeds):
+        o.present(x, 144, int(s))
+        oc.append(int(O.unpack_bits(o.spikes(), 512).sum()))
+    assert counts.tolist() == oc
+    assert np.array_equal(g.weights(), o.weights())
+    assert np.array_equal(g.spikes(), o.spikes())
+    _assert_state_equal(g, o, 784, 512, mode)
