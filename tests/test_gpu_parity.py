@@ -404,3 +404,40 @@ def test_lean_short_tables_shared_thread(gpu, mode, start, base):
     assert np.array_equal(g.weights(), o.weights())
     assert np.array_equal(g.spikes(), o.spikes())
     _assert_state_equal(g, o, 784, 512, mode)
+
+
+def _fuzz_case(k):
+    rng = np.random.default_rng(1000 + k)
+    bits = int(rng.choice([2, 4, 8]))
+    n_exc = int(rng.choice([33, 100, 256, 512, 1024]))
+    fmin, fmax = [(1.0, 22.0), (5.0, 78.0), (10.0, 156.0)][int(rng.integers(3))]
+    p = O.params({2: "2b", 4: "4b", 8: "8b"}[bits], membrane_mode=int(rng.integers(2)), init_seed=int(rng.integers(1, 99)),
+                 f_min_hz=fmin, f_max_hz=fmax, t_ref_steps=int(rng.choice([1, 2, 5, 10])),
+                 t_inh_steps=int(rng.choice([3, 5, 10])), v_spike=float(rng.choice([1.0, 2.0, 4.0])),
+                 cluster_size=min(int(rng.choice([0, 0, 1, 2, 4])), (n_exc + 31) // 32))
+    return p, bits, n_exc, int(rng.choice([60, 150, 350])), str(rng.choice(["mnist", "fashion"])), int(rng.integers(10000))
+
+
+@pytest.mark.parametrize("k", range(48))
+def test_lean_fuzz_vs_oracle(gpu, k):
+    """Randomised configurations of the paper's default mode (the lean kernel): widths, column counts, cluster
+    sizes (one to many warps per CTA), input rates, refractory / inhibition lengths, current scale, membrane
+    mode; 3 images per launch against the oracle presenting them one by one."""
+    import paper_conf_date_shelm19_b200 as P
+    p, bits, n_exc, T, kind, start = _fuzz_case(k)
+    try:
+        g, o = _pair(784, n_exc, bits, p)
+    except P.SnnError as e:                       # a cluster size too small for the network's codes
+        assert e.rc == -5
+        pytest.skip("network does not fit the requested cluster")
+    imgs, seeds = synthdata.images(3, kind, start=start), synthdata.seeds(3, base_seed=k + 1)
+    counts = np.zeros(3, np.int32)
+    g.present_batch(imgs, T, seeds, counts)
+    oc = []
+    for x, s in zip(imgs, seeds):
+        o.present(x, T, int(s))
+        oc.append(int(O.unpack_bits(o.spikes(), n_exc).sum()))
+    assert counts.tolist() == oc
+    assert np.array_equal(g.weights(), o.weights())
+    assert np.array_equal(g.spikes(), o.spikes())
+    _assert_state_equal(g, o, 784, n_exc, p["membrane_mode"])
