@@ -207,3 +207,23 @@ def test_sharded_two_processes_ipc(gpu, tmp_path):
     assert np.array_equal(w, o.weights())
     for r in range(2):
         assert np.load(tmp_path / f"c{r}.npy").tolist() == oc
+
+
+@pytest.mark.parametrize("k", range(12))
+def test_sharded_lean_fuzz(gpu, k):
+    """Randomised column-sharded networks on the lean kernel (the paper's default mode): world 2-4, widths,
+    column counts, rates and refractory/inhibition lengths; the union of the shards against the oracle."""
+    rng = np.random.default_rng(500 + k)
+    bits = int(rng.choice([2, 4, 8]))
+    world = int(rng.choice([2, 3, 4]))
+    n_exc = 32 * world * int(rng.integers(1, 5))
+    fmin, fmax = [(1.0, 22.0), (5.0, 78.0)][int(rng.integers(2))]
+    p = O.params({2: "2b", 4: "4b", 8: "8b"}[bits], membrane_mode=int(rng.integers(2)), init_seed=int(rng.integers(1, 99)),
+                 f_min_hz=fmin, f_max_hz=fmax, t_ref_steps=int(rng.choice([2, 5, 10])), t_inh_steps=int(rng.choice([3, 10])),
+                 v_spike=float(rng.choice([2.0, 4.0])))
+    sh = _shards(784, n_exc, bits, p, world)
+    assert all(s.info()["lean"] == 1 for s in sh)
+    o = O.OracleNet(784, n_exc, bits, p)
+    kind = str(rng.choice(["mnist", "fashion"]))
+    _compare(sh, o, synthdata.images(2, kind, start=int(rng.integers(5000))), 150, synthdata.seeds(2, k + 3), 784, n_exc,
+             p["membrane_mode"])
