@@ -20,7 +20,14 @@ def main():
     ap.add_argument("--eval-every", type=int, default=250)
     ap.add_argument("--n-label", type=int, default=1000)
     ap.add_argument("--n-eval", type=int, default=2000)
+    ap.add_argument("--t-ref", type=int, default=None, help="reading R6b: e.g. --t-ref 10 --t-inh 10")
+    ap.add_argument("--t-inh", type=int, default=None)
     a = ap.parse_args()
+    common = {}
+    if a.t_ref is not None:
+        common["t_ref_steps"] = a.t_ref
+    if a.t_inh is not None:
+        common["t_inh_steps"] = a.t_inh
     import torch
     from paper_conf_date_shelm19_b200 import schedule as S
     torch.cuda.set_device(0)
@@ -41,10 +48,10 @@ def main():
     }
     for name, phases in schedules.items():
         curve, net = S.run_schedule(784, a.n_exc, a.bits, phases, tr, trs, li, lc, ls, ei, ec, es,
-                                    eval_every=a.eval_every, eval_T=350)
+                                    eval_every=a.eval_every, eval_T=350, common=common)
         pts = [dict(images=p.images, sim_s=p.sim_ms / 1e3, device_s=p.device_s, error=p.error, phase=p.phase)
                for p in curve]
-        print(json.dumps({"schedule": name, "n_exc": a.n_exc, "bits": a.bits, "train_images": a.train,
+        print(json.dumps({"schedule": name, "n_exc": a.n_exc, "bits": a.bits, "train_images": a.train, **common,
                           "train_images_per_s": a.train / curve[-1].device_s, "final_error": curve[-1].error,
                           "curve": pts}), flush=True)
         net.close()
