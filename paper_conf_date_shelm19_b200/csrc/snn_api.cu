@@ -396,7 +396,7 @@ int present_impl(snn_handle* h, const void* input, int n_images, int T, const ui
     prof_mark(h);
     if (h->lean)
       CUDA_TRY(snn::launch_present_lean(lp, 1, h->cs, h->nthr, h->smem_lean, h->bits, h->cpt, h->p.membrane_mode,
-                                        h->world > 1, h->stream));
+                                        h->world > 1, h->p.wta_mode == SNN_WTA_LAYER, h->stream));
     else
       CUDA_TRY(snn::launch_present_event_mode(lp, 1, h->cs, h->nthr, h->smem, h->bits, h->cpt, h->p.membrane_mode,
                                               h->stream));
@@ -525,7 +525,9 @@ int create_impl(int n_in, int n_exc, int bits, const snn_params* p, int col_base
   // 16-bit codes (NEXT-2, R27) run on the per-step engine: the event kernels pack <= 8-bit codes in SWAR lanes
   h->engine = (p->engine == SNN_ENGINE_STEP || bits > 8) ? SNN_ENGINE_STEP : SNN_ENGINE_EVENT;
   // the lean kernel covers the paper's default learning mode; SNN_NO_LEAN=1 disables it
-  const bool lean_mode = p->engine == SNN_ENGINE_EVENT && bits <= 8 && p->wta_mode == SNN_WTA_HARD &&
+  // (LAYER WTA is instantiated unsharded only)
+  const bool lean_mode = p->engine == SNN_ENGINE_EVENT && bits <= 8 &&
+                         (p->wta_mode == SNN_WTA_HARD || (p->wta_mode == SNN_WTA_LAYER && world == 1)) &&
                          p->inh_mode == SNN_INH_RESET && p->stdp_mode == SNN_STDP_STOCH &&
                          !(getenv("SNN_NO_LEAN") && atoi(getenv("SNN_NO_LEAN")) != 0);
   int chosen = 0;
@@ -931,7 +933,7 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
     lp.descs = d_descs + off;
     size_t smem = 0;
     bool lean = ev;
-    for (int k : g) lean = lean && hs[k]->lean;
+    for (int k : g) lean = lean && hs[k]->lean && hs[k]->p.wta_mode == hs[g[0]]->p.wta_mode;   // one WTA instance
     for (int k : g) smem = std::max(smem, lean ? hs[k]->smem_lean : hs[k]->smem);
     cudaStream_t st = h0->stream;
     if (groups.size() > 1) {
@@ -948,7 +950,8 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
       if (hs[k]->cpt != hs[g[0]]->cpt) { e = cudaErrorInvalidValue; break; }
     if (e != cudaSuccess) break;
     e = lean ? snn::launch_present_lean(lp, (int)g.size(), h0->cs, hs[g[0]]->nthr, smem, hs[g[0]]->bits,
-                                        hs[g[0]]->cpt, h0->p.membrane_mode, hs[g[0]]->world > 1, st)
+                                        hs[g[0]]->cpt, h0->p.membrane_mode, hs[g[0]]->world > 1,
+                                        hs[g[0]]->p.wta_mode == SNN_WTA_LAYER, st)
         : ev ? snn::launch_present_event_mode(lp, (int)g.size(), h0->cs, hs[g[0]]->nthr, smem, hs[g[0]]->bits,
                                               hs[g[0]]->cpt, h0->p.membrane_mode, st)
              : snn::launch_present(lp, (int)g.size(), h0->cs, h0->nthr, smem, st);

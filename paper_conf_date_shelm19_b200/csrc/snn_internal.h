@@ -117,7 +117,7 @@ size_t lean_smem_bytes(int n_in, int slice_words, int L_pot, int L_dep, int nthr
                        int logn);
 cudaError_t query_max_clusters_lean(int bits, int cpt, int fixed, int cs, int nthr, size_t smem, int* out);
 cudaError_t launch_present_lean(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, int bits, int cpt,
-                                int fixed, int sharded, cudaStream_t s);
+                                int fixed, int sharded, int layer, cudaStream_t s);
 cudaError_t query_max_clusters(int cs, int nthr, size_t smem, int* out);
 cudaError_t launch_init_weights(const NetDesc& d, uint64_t init_seed, cudaStream_t s);
 cudaError_t launch_pack_weights(const NetDesc& d, const void* codes, cudaStream_t s);      // u8 / u16 (bits 16) codes

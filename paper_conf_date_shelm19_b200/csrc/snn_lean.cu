@@ -60,7 +60,7 @@ constexpr int kSlots = 8;            // fixed row slots per step (steps with mor
 constexpr int kBlk = 4;              // steps one block integrates before running the LIF chains through them
 
 struct LeanLayout {
-  size_t slots, wsum, flags, misc, dS, dbits, dev, w, pot, dep, lpre, offs, pst, prow, p8, run, rraw, log, total;
+  size_t slots, wsum, flags, misc, spk, dS, dbits, dev, w, pot, dep, lpre, offs, pst, prow, p8, run, rraw, log, total;
 };
 
 __host__ __device__ inline LeanLayout lean_layout(int n_in, int slice_words, int L_pot, int L_dep, int nthr,
@@ -71,6 +71,7 @@ __host__ __device__ inline LeanLayout lean_layout(int n_in, int slice_words, int
   L.wsum = o;  o = align16(o + 32 * 2 * 8);                  // per warp: steps, key
   L.flags = o; o = align16(o + 4 * 4);                       // early-stop flag per epoch parity
   L.misc = o;  o = align16(o + 40 * 4);
+  L.spk = o;   o = align16(o + (size_t)nthr * 4 * 4);                 // LAYER: this CTA's spiking columns
   L.dS = o;    o = align16(o + (size_t)kDefSteps * 4);                // deferred column: S per table step
   L.dbits = o; o = align16(o + (size_t)(kDefRowsPerThr * nthr / 32) * 4);   // deferred column: event bit per raw row
   L.dev = o;   o = align16(o + (size_t)n_in * 8 * 2);                 // deferred column: event steps per input row (x2)
@@ -103,8 +104,9 @@ size_t lean_smem_bytes(int n_in, int slice_words, int L_pot, int L_dep, int nthr
   return lean_layout(n_in, slice_words, L_pot, L_dep, nthr, rows_cap, offs_cap, logn).total;
 }
 
-// SH: compiled with the cross-rank (column-sharded) exchange; the unsharded instance carries none of it
-template <int BITS, int CPT_, bool FIXED, bool SH>
+// SH: compiled with the cross-rank (column-sharded) exchange; the unsharded instance carries none of it.
+// LAY: LAYER WTA (R7) instead of HARD (instantiated unsharded only)
+template <int BITS, int CPT_, bool FIXED, bool SH, bool LAY>
 __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __grid_constant__ LaunchParams lp) {
   using Z = LSwar<BITS, CPT_>;
   constexpr int CPT = Z::CPT;
@@ -140,6 +142,10 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
   uint32_t* s_rraw = reinterpret_cast<uint32_t*>(smem + L.rraw);
   uint32_t* s_log = reinterpret_cast<uint32_t*>(smem + L.log);
   int* s_dS = reinterpret_cast<int*>(smem + L.dS);
+  int* s_spk = reinterpret_cast<int*>(smem + L.spk);
+  // LAYER WTA (R7): every column that crosses at t* spikes; the summary carries the number of crossers at the
+  // earliest step instead of the largest key (HARD)
+  constexpr bool layer = LAY;
   uint32_t* s_dbits = reinterpret_cast<uint32_t*>(smem + L.dbits);
   unsigned long long* s_dev = reinterpret_cast<unsigned long long*>(smem + L.dev);
 
@@ -518,7 +524,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
       int p_done = k0 - 1;           // last step fully processed by this thread
       int cstep = kNoStep;           // crossing step (the warp stops right after it)
       int hstep = kNoStep;           // undo log full: stopped before this step
-      unsigned long long ckey = 0ull;
+      unsigned long long ckey = 0ull;    // HARD: best WTA key at cstep; LAYER: number of own columns crossing at cstep
+      uint32_t cmk = 0u;                 // own columns crossing at cstep
       int nlog = 0;
       int dr0 = INT_MIN;             // warp-uniform raw start of the drawn LTD row range [dr0, dr0 + kDrawRows)
       unsigned long long evm[CPT];   // LTD event bits of raw rows [dr0, dr0 + 64) (owning lane)
@@ -641,7 +648,10 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         const int dl = __ffs(__ballot_sync(FULL, dslot >= 0)) - 1;
         const int cdw = __shfl_sync(FULL, cd, dl);
         const int lastw = __shfl_sync(FULL, last, dl);
-        if (dslot >= 0) { p_look = last; if (cd != kNoStep) { cstep = cd; ckey = keyd; } }
+        if (dslot >= 0) {
+          p_look = last;
+          if (cd != kNoStep) { cstep = cd; ckey = layer ? 1ull : keyd; cmk = 1u << dslot; }
+        }
         if (cdw != kNoStep) {
           signal_cross(cdw);
         } else if (lastw == kstop - 1 && kstop < kend) {          // the table ends first: the epoch ends there
@@ -774,13 +784,18 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
               if (cm) {
                 // (the thread's deferred column may have reported a LATER crossing in its run ahead: an earlier
                 // one replaces its key, an equal one competes with it)
-                if (kk + j < cstep) { cstep = kk + j; ckey = 0ull; }
+                if (kk + j < cstep) { cstep = kk + j; ckey = 0ull; cmk = 0u; }
+                cmk |= cm;
+                if (layer) {
+                  ckey += (unsigned long long)__popc(cm);
+                } else {
 #pragma unroll
-                for (int c = 0; c < CPT; ++c) {
-                  if (!(cm >> c & 1u)) continue;
-                  const unsigned long long key = ((unsigned long long)lif.ord(v[c]) << 32) |
-                                                 (0xFFFFFFFFu - (uint32_t)(cbase + col0 + jcol[c]));
-                  ckey = key > ckey ? key : ckey;
+                  for (int c = 0; c < CPT; ++c) {
+                    if (!(cm >> c & 1u)) continue;
+                    const unsigned long long key = ((unsigned long long)lif.ord(v[c]) << 32) |
+                                                   (0xFFFFFFFFu - (uint32_t)(cbase + col0 + jcol[c]));
+                    ckey = key > ckey ? key : ckey;
+                  }
                 }
               }
               cmb = __any_sync(FULL, cm != 0) ? 1u : 0u;
@@ -903,13 +918,18 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         }
         p_done = kk;
         if (cm) {                                                // crossing: the WTA key (R7)
-          if (kk < cstep) { cstep = kk; ckey = 0ull; }          // (see the block path)
+          if (kk < cstep) { cstep = kk; ckey = 0ull; cmk = 0u; }   // (see the block path)
+          cmk |= cm;
+          if (layer) {
+            ckey += (unsigned long long)__popc(cm);
+          } else {
 #pragma unroll
-          for (int c = 0; c < CPT; ++c) {
-            if (!(cm >> c & 1u)) continue;
-            const unsigned long long key = ((unsigned long long)lif.ord(v[c]) << 32) |
-                                           (0xFFFFFFFFu - (uint32_t)(cbase + col0 + jcol[c]));
-            ckey = key > ckey ? key : ckey;
+            for (int c = 0; c < CPT; ++c) {
+              if (!(cm >> c & 1u)) continue;
+              const unsigned long long key = ((unsigned long long)lif.ord(v[c]) << 32) |
+                                             (0xFFFFFFFFu - (uint32_t)(cbase + col0 + jcol[c]));
+              ckey = key > ckey ? key : ckey;
+            }
           }
         }
         LEAN_CYC(c_gen);
@@ -941,7 +961,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         const int wc = __reduce_min_sync(FULL, cstep);
         const int wh = __reduce_min_sync(FULL, hstep);
         const uint32_t kh = __reduce_max_sync(FULL, cstep == wc ? (uint32_t)(ckey >> 32) : 0u);
-        const uint32_t kl = __reduce_max_sync(FULL, (cstep == wc && (uint32_t)(ckey >> 32) == kh) ? (uint32_t)ckey : 0u);
+        const uint32_t kl = layer ? __reduce_add_sync(FULL, cstep == wc ? (uint32_t)ckey : 0u)   // LAYER: count
+                                  : __reduce_max_sync(FULL, (cstep == wc && (uint32_t)(ckey >> 32) == kh) ? (uint32_t)ckey : 0u);
         if (lane == 0) {
           s_wsum[2 * warp] = ((unsigned long long)(uint32_t)wc << 32) | (uint32_t)wh;
           s_wsum[2 * warp + 1] = ((unsigned long long)kh << 32) | kl;
@@ -956,7 +977,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         const int C = __reduce_min_sync(FULL, wc);
         const int H = __reduce_min_sync(FULL, wh);
         const uint32_t kh = __reduce_max_sync(FULL, wc == C ? (uint32_t)(k >> 32) : 0u);
-        const uint32_t kl = __reduce_max_sync(FULL, (wc == C && (uint32_t)(k >> 32) == kh) ? (uint32_t)k : 0u);
+        const uint32_t kl = layer ? __reduce_add_sync(FULL, wc == C ? (uint32_t)k : 0u)
+                                  : __reduce_max_sync(FULL, (wc == C && (uint32_t)(k >> 32) == kh) ? (uint32_t)k : 0u);
         const unsigned long long A = ((unsigned long long)(uint32_t)C << 32) | (uint32_t)H;
         const unsigned long long K = ((unsigned long long)kh << 32) | kl;
         unsigned long long* slot = s_slots + (size_t)(fp * kMaxCluster + rank) * 2;
@@ -982,7 +1004,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
         P = __reduce_min_sync(FULL, c);
         H = __reduce_min_sync(FULL, h);
         const uint32_t kh = __reduce_max_sync(FULL, c == P ? (uint32_t)(Kr >> 32) : 0u);
-        const uint32_t kl = __reduce_max_sync(FULL, (c == P && (uint32_t)(Kr >> 32) == kh) ? (uint32_t)Kr : 0u);
+        const uint32_t kl = layer ? __reduce_add_sync(FULL, c == P ? (uint32_t)Kr : 0u)
+                                  : __reduce_max_sync(FULL, (c == P && (uint32_t)(Kr >> 32) == kh) ? (uint32_t)Kr : 0u);
         K = ((unsigned long long)kh << 32) | kl;
       }
       if (sharded) {
@@ -1018,7 +1041,8 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           const int Pg = __reduce_min_sync(FULL, c);
           const int Hg = __reduce_min_sync(FULL, h);
           const uint32_t kh = __reduce_max_sync(FULL, c == Pg ? (uint32_t)(Kr >> 32) : 0u);
-          const uint32_t kl = __reduce_max_sync(FULL, (c == Pg && (uint32_t)(Kr >> 32) == kh) ? (uint32_t)Kr : 0u);
+          const uint32_t kl = layer ? __reduce_add_sync(FULL, c == Pg ? (uint32_t)Kr : 0u)
+                                    : __reduce_max_sync(FULL, (c == Pg && (uint32_t)(Kr >> 32) == kh) ? (uint32_t)Kr : 0u);
           // (own words: the next write comes after the next cluster barrier, which every thread reaches after
           // reading these)
           unsigned long long* s_world = reinterpret_cast<unsigned long long*>(s_misc + 32);
@@ -1050,26 +1074,28 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
           ++eng_undo;
         }
       };
+      uint32_t spk = 0u;                               // LAYER: own columns spiking at t*
       if (event) {
         const uint32_t W = 0xFFFFFFFFu - (uint32_t)K;
+        // HARD: one spiker W; LAYER: every column that crossed at t* (K = their number, R7)
+        const uint32_t nsp = layer ? (uint32_t)K : 1u;
+        if (layer && cstep == P) spk = cmk;
         undo_after(P - k0);
-        bool me_any = false;
 #pragma unroll
         for (int c = 0; c < CPT; ++c) {
           if (!(valid >> c & 1u)) continue;
-          const bool me = (uint32_t)(cbase + col0 + jcol[c]) == W;
+          const bool me = layer ? ((spk >> c & 1u) != 0u) : (uint32_t)(cbase + col0 + jcol[c]) == W;
           // no crossing in [k0, t*) anywhere: the countdown only ran down (R6, R7), v is reset anyway
           const int cnt_p = max(cnt0[c] - (P - k0 + 1), 0);
           if (me) {
-            v[c] = vreset; cnt[c] = t_ref;
+            // a lone spiker keeps t_ref; with >= 2 spikers every neuron, the spikers included, is inhibited (R7)
+            v[c] = vreset; cnt[c] = nsp >= 2 ? max(t_ref, t_inh) : t_ref;
             if (rec_out) atomicOr(&d.raster_out[(size_t)P * d.nwe + ((col0 + jcol[c]) >> 5)], 1u << ((col0 + jcol[c]) & 31));
-            me_any = true;
           } else {
             v[c] = vreset; cnt[c] = max(cnt_p, t_inh);
           }
         }
-        (void)me_any;
-        ++img_spikes;
+        img_spikes += (int)nsp;
       } else if (p_done > k_last) {                    // undo log full somewhere: replay [k0 + 1, k_last]
         ++eng_resim;
         undo_after(0);
@@ -1123,7 +1149,56 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
       nlog = 0;
 
       // ---------------------------------------------------------- LTP at t* in the winner's CTA (eq.(6))
-      if (event) {
+      if (event && layer) {
+        // LAYER: every CTA holding spikers brings its input timers up to t*, writes back its deferred table through
+        // t*, takes the lowest spiking column as its new deferred column and runs the eq.(6) LTP of all of its
+        // spikers (each thread owns its input rows for every spiker: no word is written by two threads)
+        const int tP = tbase + P;
+        if (tid == 0) s_misc[37] = 0;
+        __syncthreads();
+#pragma unroll
+        for (int c = 0; c < CPT; ++c)
+          if (spk >> c & 1u) { lpost[c] = tP; s_spk[atomicAdd(&s_misc[37], 1)] = jcol[c]; }   // after LTD at t*
+        __syncthreads();
+        const int nsl = s_misc[37];
+        if (nsl > 0) {                                                        // CTA-uniform
+          if (tvalid) dtab_apply(P);
+          lpre_catch_up(P - ka);
+          __syncthreads();
+          dtab_clear();
+          int wmin = INT_MAX;
+          for (int q = 0; q < nsl; ++q) wmin = min(wmin, s_spk[q]);
+          Wd = wmin; d_lp = tP;
+          const bool tab = P + 1 < kend && dtab_draw(P + 1);
+          for (int grp = tid; grp < nq4; grp += nthr) {
+            for (int q = 0; q < nsl; ++q) {
+              const int Ws = s_spk[q];
+              const int Wg = cbase + col0 + Ws;
+              const int ww = Ws / CPW, wsh = (Ws % CPW) * BITS;
+              const uint4 u = philox((uint32_t)tP, (uint32_t)Wg, (uint32_t)grp, TAG_LTP, seed);   // eq.(6), R13
+#pragma unroll
+              for (int r = 0; r < 4; ++r) {
+                const int i = 4 * grp + r;
+                if (i >= n_in) break;
+                const int lpi = s_lpre[i];
+                if (lpi < 0) continue;
+                const int D = tP - lpi;                                        // R10: Dt = D >= 0
+                if (D >= L_pot) continue;
+                ++ltp_trials;
+                if (pick(u, r) <= s_pot[D]) {
+                  ++ltp_events;
+                  uint32_t* pw = s_w + i * wpr + ww;            // rows 4 grp .. 4 grp + 3 are this thread's alone
+                  const uint32_t wv = *pw;
+                  if (((wv >> wsh) & FMASK) < (uint32_t)qmax) *pw = wv + (1u << wsh);
+                }
+              }
+            }
+          }
+          __syncthreads();
+          if (tab) { dtab_sums(); __syncthreads(); }
+        }
+      }
+      if (event && !layer) {
         const int Wl = (int)(0xFFFFFFFFu - (uint32_t)K) - cbase - col0;     // winner's local column
         const int tP = tbase + P;
 #pragma unroll
@@ -1264,10 +1339,10 @@ __global__ void __launch_bounds__(kEvMaxThreads, 1) present_lean_kernel(const __
 }
 
 // ====================================================================== host launchers
-template <int BITS, int CPT, bool FIXED, bool SH>
+template <int BITS, int CPT, bool FIXED, bool SH, bool LAY>
 static cudaError_t lean_launch_t(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, cudaStream_t s,
                                  int* occupancy_out) {
-  auto* kern = present_lean_kernel<BITS, CPT, FIXED, SH>;
+  auto* kern = present_lean_kernel<BITS, CPT, FIXED, SH, LAY>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   if (cs > 8) {
@@ -1296,14 +1371,18 @@ static cudaError_t lean_launch_t(const LaunchParams& lp, int n_nets, int cs, int
   return cudaLaunchKernelEx(&cfg, kern, lp);
 }
 
+// sh: 0 unsharded HARD, 1 sharded HARD, 2 unsharded LAYER
 template <int BITS, int CPT>
 static cudaError_t lean_dispatch_f(int fixed, int sh, const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem,
                                    cudaStream_t s, int* occ) {
-  if (sh)
-    return fixed ? lean_launch_t<BITS, CPT, true, true>(lp, n_nets, cs, nthr, smem, s, occ)
-                 : lean_launch_t<BITS, CPT, false, true>(lp, n_nets, cs, nthr, smem, s, occ);
-  return fixed ? lean_launch_t<BITS, CPT, true, false>(lp, n_nets, cs, nthr, smem, s, occ)
-               : lean_launch_t<BITS, CPT, false, false>(lp, n_nets, cs, nthr, smem, s, occ);
+  if (sh == 2)
+    return fixed ? lean_launch_t<BITS, CPT, true, false, true>(lp, n_nets, cs, nthr, smem, s, occ)
+                 : lean_launch_t<BITS, CPT, false, false, true>(lp, n_nets, cs, nthr, smem, s, occ);
+  if (sh == 1)
+    return fixed ? lean_launch_t<BITS, CPT, true, true, false>(lp, n_nets, cs, nthr, smem, s, occ)
+                 : lean_launch_t<BITS, CPT, false, true, false>(lp, n_nets, cs, nthr, smem, s, occ);
+  return fixed ? lean_launch_t<BITS, CPT, true, false, false>(lp, n_nets, cs, nthr, smem, s, occ)
+               : lean_launch_t<BITS, CPT, false, false, false>(lp, n_nets, cs, nthr, smem, s, occ);
 }
 
 static cudaError_t lean_dispatch(int bits, int cpt, int fixed, int sh, const LaunchParams& lp, int n_nets, int cs,
@@ -1326,8 +1405,9 @@ cudaError_t query_max_clusters_lean(int bits, int cpt, int fixed, int cs, int nt
 }
 
 cudaError_t launch_present_lean(const LaunchParams& lp, int n_nets, int cs, int nthr, size_t smem, int bits, int cpt,
-                                int fixed, int sharded, cudaStream_t s) {
-  return lean_dispatch(bits, cpt, fixed, sharded, lp, n_nets, cs, nthr, smem, s, nullptr);
+                                int fixed, int sharded, int layer, cudaStream_t s) {
+  if (sharded && layer) return cudaErrorNotSupported;     // (the runtime never selects it)
+  return lean_dispatch(bits, cpt, fixed, layer ? 2 : (sharded ? 1 : 0), lp, n_nets, cs, nthr, smem, s, nullptr);
 }
 
 }  // namespace snn

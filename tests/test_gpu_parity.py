@@ -165,11 +165,11 @@ def test_C4_hf_variant(gpu, engine):
     _compare_presentations(g, o, synthdata.images(1, "fashion", start=5), 100, synthdata.seeds(1, 9), 784, 6400, 1)
 
 
-@pytest.mark.parametrize("preset,wta,inh,stdp,lean", [("2b", 0, 0, 0, 1), ("8b", 0, 0, 0, 1), ("8b", 1, 0, 0, 0),
+@pytest.mark.parametrize("preset,wta,inh,stdp,lean", [("2b", 0, 0, 0, 1), ("8b", 0, 0, 0, 1), ("8b", 1, 0, 0, 1),
                                                       ("8b", 0, 1, 0, 0), ("8b", 0, 0, 1, 0)])
 def test_lean_kernel_selection(gpu, preset, wta, inh, stdp, lean):
-    """The default learning mode (HARD WTA, RESET inhibition, stochastic STDP) runs the lean kernel;
-    every other mode, and SNN_ENGINE_EVENT_GENERAL, runs the general event kernel."""
+    """RESET inhibition with stochastic STDP (HARD or LAYER WTA) runs the lean kernel; HOLD inhibition, the
+    deterministic arm, and SNN_ENGINE_EVENT_GENERAL run the general event kernel."""
     p = O.params(preset, wta_mode=wta, inh_mode=inh, stdp_mode=stdp)
     g, _ = _pair(784, 400, 8 if preset == "8b" else 2, p, engine=0)
     assert g.info()["lean"] == lean
@@ -412,6 +412,7 @@ def _fuzz_case(k):
     n_exc = int(rng.choice([33, 100, 256, 512, 1024]))
     fmin, fmax = [(1.0, 22.0), (5.0, 78.0), (10.0, 156.0)][int(rng.integers(3))]
     p = O.params({2: "2b", 4: "4b", 8: "8b"}[bits], membrane_mode=int(rng.integers(2)), init_seed=int(rng.integers(1, 99)),
+                 wta_mode=int(rng.random() < 0.35),
                  f_min_hz=fmin, f_max_hz=fmax, t_ref_steps=int(rng.choice([1, 2, 5, 10])),
                  t_inh_steps=int(rng.choice([3, 5, 10])), v_spike=float(rng.choice([1.0, 2.0, 4.0])),
                  cluster_size=min(int(rng.choice([0, 0, 1, 2, 4])), (n_exc + 31) // 32))
@@ -420,9 +421,10 @@ def _fuzz_case(k):
 
 @pytest.mark.parametrize("k", range(48))
 def test_lean_fuzz_vs_oracle(gpu, k):
-    """Randomised configurations of the paper's default mode (the lean kernel): widths, column counts, cluster
-    sizes (one to many warps per CTA), input rates, refractory / inhibition lengths, current scale, membrane
-    mode; 3 images per launch against the oracle presenting them one by one."""
+    """Randomised configurations of the lean kernel's modes (RESET inhibition, stochastic STDP, HARD or LAYER
+    WTA): widths, column counts, cluster sizes (one to many warps per CTA), input rates, refractory /
+    inhibition lengths, current scale, membrane mode; 3 images per launch against the oracle presenting them
+    one by one."""
     import paper_conf_date_shelm19_b200 as P
     p, bits, n_exc, T, kind, start = _fuzz_case(k)
     try:
