@@ -116,6 +116,12 @@ def lib():
         L.oracle_lif_step_fp32.argtypes = [ctypes.c_void_p, ctypes.c_float, ctypes.c_int32]
         L.oracle_lif_step_fp32.restype = ctypes.c_float
         L.oracle_lif_step_fixed.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32]
+        L.oracle_lif_step_fp32g.argtypes = [ctypes.c_void_p, ctypes.c_float, ctypes.c_float]
+        L.oracle_lif_step_fp32g.restype = ctypes.c_float
+        L.oracle_exp_recipe.argtypes = [ctypes.c_void_p, ctypes.c_double]
+        L.oracle_exp_recipe.restype = ctypes.c_double
+        L.oracle_dg.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_float]
+        L.oracle_dg.restype = ctypes.c_double
         L.oracle_lif_step_fixed.restype = ctypes.c_int32
         L.oracle_infer.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int, ctypes.c_int, ctypes.c_void_p,
                                    ctypes.c_void_p]
@@ -196,7 +202,8 @@ class OracleNet:
 
     @property
     def code_dtype(self):
-        return np.uint16 if self.bits > 8 else np.uint8
+        """uint8 codes (<= 8 bits), uint16 codes (16 bits), binary32 conductance (32 bits, R28)"""
+        return np.float32 if self.bits == 32 else (np.uint16 if self.bits > 8 else np.uint8)
 
     def weights(self) -> np.ndarray:
         out = np.empty((self.n_in, self.n_exc), dtype=self.code_dtype)
@@ -248,6 +255,18 @@ class OracleNet:
 
     def lif_step_fixed(self, v: int, S: int) -> int:
         return int(lib().oracle_lif_step_fixed(self._h, int(v), int(S)))
+
+    def lif_step_fp32g(self, v: float, Sg: float) -> float:
+        """32-bit arm (R28): LIF update on the binary32 conductance sum."""
+        return float(lib().oracle_lif_step_fp32g(self._h, ctypes.c_float(v), ctypes.c_float(Sg)))
+
+    def exp_recipe(self, y: float) -> float:
+        """R28's binary64 e^y recipe."""
+        return float(lib().oracle_exp_recipe(self._h, float(y)))
+
+    def dg(self, depress: bool, G: float) -> float:
+        """eqs.(4)(5) at binary32 conductance G (R28), binary64."""
+        return float(lib().oracle_dg(self._h, 1 if depress else 0, ctypes.c_float(G)))
 
     def infer(self, images: np.ndarray, T: int, seeds) -> np.ndarray:
         """NEXT-1: spike counts (n_images, n_exc) u32 with frozen weights (R21)."""

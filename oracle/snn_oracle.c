@@ -35,10 +35,21 @@
 #define TAG_INIT  5u
 #define TAG_ROUND_LTD 6u   /* 16-bit stochastic arm: rounding draw of an LTD step [R27] */
 
+/* Cody-Waite split of ln 2 (hi part has 11 trailing zero bits, so k * LN2_HI is exact for |k| < 2^11) and
+ * 1/ln 2, as binary64 literals, for the exp recipe of the 32-bit arm [R28] */
+#define INV_LN2 0x1.71547652b82fep+0
+#define LN2_HI  0x1.62e42feep-1
+#define LN2_LO  0x1.a39ef35793c76p-33
+#define EXP_DEG 13
+
 struct oracle_net {
   int n_in, n_exc, bits, frac_bits, q_max;
   oracle_params p;
-  uint16_t* q;                /* conductance codes q[i*n_exc + j]; G = q * 2^-frac_bits [R9] */
+  uint16_t* q;                /* conductance codes q[i*n_exc + j]; G = q * 2^-frac_bits [R9] (bits <= 16) */
+  float* g;                   /* 32-bit arm: conductance G[i*n_exc + j] itself, IEEE binary32 [R28] */
+  double ecoef[EXP_DEG + 1];  /* 1/m!, m = 0..EXP_DEG, by c_m = c_{m-1} / m in binary64 [R28] */
+  float kV;                   /* (float) v_spike: I = v_spike * sum G, 32-bit arm [R28] */
+  float gminf, gmaxf;
   /* state [R5] */
   float*   v_f;               /* membrane, fp32 mode */
   int32_t* v_x;               /* membrane, Q15.16 fixed mode */
@@ -113,7 +124,10 @@ static int build_exp_lut(double gamma, double tau, double dt, uint64_t* thr, int
 
 static int validate(int n_in, int n_exc, int bits, const oracle_params* p) {
   if (n_in < 1 || n_in > 8192 || n_exc < 1 || n_exc > (1 << 20)) return E_INVAL;
-  if (bits != 2 && bits != 4 && bits != 8 && bits != 16) return E_INVAL;
+  if (bits != 2 && bits != 4 && bits != 8 && bits != 16 && bits != 32) return E_INVAL;
+  /* 32-bit floating-point conductance [R28]: fp32 membranes (the fixed recipe needs an integer sum) and
+   * IEEE round-to-nearest (the trunc / eq.(8) roundings are defined on a fixed-point grid, R17) */
+  if (bits == 32 && (p->membrane_mode != 0 || p->rounding != 1)) return E_INVAL;
   if (!(p->dt_ms > 0.0)) return E_INVAL;
   if (!(p->f_min_hz >= 0.0 && p->f_max_hz >= p->f_min_hz)) return E_INVAL;
   if (p->f_max_hz * p->dt_ms * 1e-3 > 1.0) return E_INVAL;
@@ -139,8 +153,8 @@ int oracle_create(int n_in, int n_exc, int bits, const oracle_params* p, oracle_
   n->n_in = n_in; n->n_exc = n_exc; n->bits = bits; n->p = *p;
   /* [R9] G = q * 2^-frac_bits, frac_bits = bits unless given (Q1.7 style) */
   n->frac_bits = p->frac_bits > 0 ? p->frac_bits : bits;
-  n->q_max = (1 << bits) - 1;
-  if (n->frac_bits != bits) {
+  n->q_max = bits == 32 ? 0 : (1 << bits) - 1;   /* no code grid at 32 bits [R28] */
+  if (bits <= 16 && n->frac_bits != bits) {
     double cap = floor(ldexp(p->g_max, n->frac_bits));
     if (cap < n->q_max) n->q_max = (int)cap;
   }
@@ -186,9 +200,17 @@ int oracle_create(int n_in, int n_exc, int bits, const oracle_params* p, oracle_
   n->af = (float)p->a; n->bf = (float)p->b; n->cf = (float)p->c; n->dtf = (float)p->dt_ms;
   n->kI = (float)(p->v_spike * lsb); n->ief = (float)p->i_ext;
   n->vthf = (float)p->v_th; n->vresetf = (float)p->v_reset; n->vinitf = (float)p->v_init;
+  /* 32-bit arm [R28] */
+  n->kV = (float)p->v_spike; n->gminf = (float)p->g_min; n->gmaxf = (float)p->g_max;
+  n->ecoef[0] = 1.0;
+  for (int m = 1; m <= EXP_DEG; ++m) n->ecoef[m] = n->ecoef[m - 1] / (double)m;
 
   size_t nq = (size_t)n_in * (size_t)n_exc;
   n->q = (uint16_t*)malloc(nq * sizeof(uint16_t));
+  if (bits == 32) {
+    n->g = (float*)malloc(nq * sizeof(float));
+    if (!n->g) { oracle_destroy(n); return E_NOMEM; }
+  }
   n->v_f = (float*)calloc((size_t)n_exc, sizeof(float));
   n->v_x = (int32_t*)calloc((size_t)n_exc, sizeof(int32_t));
   n->cnt = (int32_t*)calloc((size_t)n_exc, sizeof(int32_t));
@@ -201,6 +223,8 @@ int oracle_create(int n_in, int n_exc, int bits, const oracle_params* p, oracle_
     for (int j = 0; j < n_exc; ++j) {
       uint32_t u = draw(p->init_seed, (uint32_t)i, (uint32_t)(j >> 2), 0u, TAG_INIT, j & 3);
       n->q[(size_t)i * n_exc + j] = (uint16_t)(((uint64_t)u * (uint64_t)(n->q_max + 1)) >> 32);
+      /* 32-bit arm [R28]: G = g_max * (u >> 8) 2^-24, uniform on the 2^24-point grid of [0, g_max) */
+      if (bits == 32) n->g[(size_t)i * n_exc + j] = (float)(p->g_max * ldexp((double)(u >> 8), -24));
     }
   /* state as after a reset [R5] */
   for (int j = 0; j < n_exc; ++j) { n->v_f[j] = n->vinitf; n->v_x[j] = n->Vinit; n->last_post[j] = NEVER; }
@@ -211,7 +235,7 @@ int oracle_create(int n_in, int n_exc, int bits, const oracle_params* p, oracle_
 
 int oracle_destroy(oracle_net* n) {
   if (!n) return 0;
-  free(n->q); free(n->v_f); free(n->v_x); free(n->cnt); free(n->last_post); free(n->last_pre);
+  free(n->q); free(n->g); free(n->v_f); free(n->v_x); free(n->cnt); free(n->last_post); free(n->last_pre);
   free(n->raster); free(n->in_raster);
   free(n->det_p_base); free(n->det_d_base); free(n->det_p_thr); free(n->det_d_thr);
   free(n);
@@ -225,6 +249,47 @@ float oracle_lif_step_fp32(const oracle_net* n, float v, int32_t S) {
   float y  = fmaf(n->cf, x, n->af);       /* a + c I */
   float dv = fmaf(n->bf, v, y);           /* a + b v + c I */
   return fmaf(n->dtf, dv, v);             /* v + dt dv/dt */
+}
+
+/* 32-bit arm [R28]: the same recipe on the binary32 conductance sum Sg = sum_i G_i (eq.(3): I = v_spike Sg) */
+float oracle_lif_step_fp32g(const oracle_net* n, float v, float Sg) {
+  float I  = Sg * n->kV;
+  float x  = I + n->ief;
+  float y  = fmaf(n->cf, x, n->af);
+  float dv = fmaf(n->bf, v, y);
+  return fmaf(n->dtf, dv, v);
+}
+
+/* e^y in binary64 by an explicit recipe [R28] (so that both implementations round identically):
+ * y = k ln2 + r with k = nearest integer to y / ln2 and r = (y - k LN2_HI) - k LN2_LO (two fused
+ * multiply-adds), e^r by its Taylor series to degree EXP_DEG in Horner form (fused multiply-adds), times 2^k.
+ * |r| <= ln2 / 2 bounds the truncation error by 0.35^14 / 14! < 1e-17 relative (tests pin it to libm exp). */
+double oracle_exp_recipe(const oracle_net* n, double y) {
+  double k = nearbyint(y * INV_LN2);
+  double r = fma(-k, LN2_HI, y);
+  r = fma(-k, LN2_LO, r);
+  double e = n->ecoef[EXP_DEG];
+  for (int m = EXP_DEG - 1; m >= 0; --m) e = fma(e, r, n->ecoef[m]);
+  return ldexp(e, (int)k);
+}
+
+/* eqs.(4)(5) at conductance G (binary64) [R28]:
+ *   dG_p = alpha_p e^{-beta_p (G - G_min) / (G_max - G_min)},  dG_d = alpha_d e^{-beta_d (G_max - G) / (G_max - G_min)} */
+double oracle_dg(const oracle_net* n, int depress, float G) {
+  const oracle_params* p = &n->p;
+  const double span = p->g_max - p->g_min;
+  if (!depress) return p->alpha_p * oracle_exp_recipe(n, -p->beta_p * ((double)G - p->g_min) / span);
+  return p->alpha_d * oracle_exp_recipe(n, -p->beta_d * (p->g_max - (double)G) / span);
+}
+
+/* P:89 "after floating point calculation of change in conductance dG, the result is rounded to a value that
+ * can be represented in the current bit width": G' = binary32(G +- dG) (round to nearest), clamped to
+ * [G_min, G_max] [R28] */
+static float g_step(const oracle_net* n, float G, double dG, int depress) {
+  float G1 = (float)(depress ? (double)G - dG : (double)G + dG);
+  if (G1 < n->gminf) G1 = n->gminf;
+  if (G1 > n->gmaxf) G1 = n->gmaxf;
+  return G1;
 }
 
 int32_t oracle_lif_step_fixed(const oracle_net* n, int32_t v, int32_t S) {
@@ -263,10 +328,11 @@ int oracle_present_ex(oracle_net* n, const void* input, int T, uint64_t seed, in
 
   uint8_t* s = (uint8_t*)calloc((size_t)n_in, 1);
   int32_t* S = (int32_t*)calloc((size_t)n_exc, sizeof(int32_t));
+  float* Sg = (float*)calloc((size_t)n_exc, sizeof(float));
   uint8_t* cand = (uint8_t*)calloc((size_t)n_exc, 1);
   int* spikers = (int*)malloc(sizeof(int) * (size_t)n_exc);
-  if (!n->raster || !n->in_raster || !s || !S || !cand || !spikers) {
-    free(s); free(S); free(cand); free(spikers); return E_NOMEM;
+  if (!n->raster || !n->in_raster || !s || !S || !Sg || !cand || !spikers) {
+    free(s); free(S); free(Sg); free(cand); free(spikers); return E_NOMEM;
   }
 
   for (int k = 0; k < T; ++k) {
@@ -288,18 +354,25 @@ int oracle_present_ex(oracle_net* n, const void* input, int T, uint64_t seed, in
       }
     }
 
-    /* 2 INTEGRATE -- eq.(3): S_j = sum over spiking pre-neurons of q[i][j] (I = v_spike LSB S) */
+    /* 2 INTEGRATE -- eq.(3): S_j = sum over spiking pre-neurons of q[i][j] (I = v_spike LSB S);
+     * 32-bit arm: Sg_j = sum of G[i][j] in binary32, ascending i [R28] */
     for (int j = 0; j < n_exc; ++j) {
       int32_t acc = 0;
-      for (int i = 0; i < n_in; ++i)
-        if (s[i]) acc += n->q[(size_t)i * n_exc + j];
+      float accg = 0.0f;
+      for (int i = 0; i < n_in; ++i) {
+        if (!s[i]) continue;
+        if (n->bits == 32) accg = accg + n->g[(size_t)i * n_exc + j];
+        else acc += n->q[(size_t)i * n_exc + j];
+      }
       S[j] = acc;
+      Sg[j] = accg;
     }
 
     /* 3 LIF -- eqs.(1)(2); refractory/inhibited neurons hold v [R6][R7] */
     for (int j = 0; j < n_exc; ++j) {
       if (n->cnt[j] > 0) { n->cnt[j]--; cand[j] = 0; continue; }
       if (fixed) { n->v_x[j] = oracle_lif_step_fixed(n, n->v_x[j], S[j]); cand[j] = n->v_x[j] > n->Vth; }
+      else if (n->bits == 32) { n->v_f[j] = oracle_lif_step_fp32g(n, n->v_f[j], Sg[j]); cand[j] = n->v_f[j] > n->vthf; }
       else       { n->v_f[j] = oracle_lif_step_fp32(n, n->v_f[j], S[j]);  cand[j] = n->v_f[j] > n->vthf; }
     }
 
@@ -348,7 +421,10 @@ int oracle_present_ex(oracle_net* n, const void* input, int T, uint64_t seed, in
           if ((uint64_t)u < n->thr_dep[D]) {
             n->stats[3]++;
             uint16_t* qq = &n->q[(size_t)i * n_exc + j];
-            if (n->bits <= 8) {
+            if (n->bits == 32) {                       /* 32 bit: G -= eq.(5), binary32 [R28] */
+              float* g = &n->g[(size_t)i * n_exc + j];
+              *g = g_step(n, *g, oracle_dg(n, 1, *g), 1);
+            } else if (n->bits <= 8) {
               if (*qq > 0) *qq -= 1;                   /* dG = 1 LSB */
             } else {                                   /* 16 bit: dG = eq.(5), rounded (eq.(8)) [R27] */
               uint32_t u2 = draw(seed, (uint32_t)t, (uint32_t)i, (uint32_t)(j >> 2), TAG_ROUND_LTD, j & 3);
@@ -371,7 +447,10 @@ int oracle_present_ex(oracle_net* n, const void* input, int T, uint64_t seed, in
           if ((uint64_t)u < n->thr_pot[D]) {
             n->stats[5]++;
             uint16_t* qq = &n->q[(size_t)i * n_exc + W];
-            if (n->bits <= 8) {
+            if (n->bits == 32) {                       /* 32 bit: G += eq.(4), binary32 [R28] */
+              float* g = &n->g[(size_t)i * n_exc + W];
+              *g = g_step(n, *g, oracle_dg(n, 0, *g), 0);
+            } else if (n->bits <= 8) {
               if (*qq < n->q_max) *qq += 1;            /* dG = 1 LSB */
             } else {                                   /* 16 bit: dG = eq.(4), rounded (eq.(8)) [R27] */
               uint32_t u2 = draw(seed, (uint32_t)t, (uint32_t)W, (uint32_t)(i >> 2), TAG_ROUND, i & 3);
@@ -391,6 +470,14 @@ int oracle_present_ex(oracle_net* n, const void* input, int T, uint64_t seed, in
           uint16_t* qq = &n->q[(size_t)i * n_exc + W];
           int q0 = *qq;
           int pot = n->last_pre[i] != NEVER && (t - n->last_pre[i]) <= p->t_ltp_steps;
+          if (n->bits == 32) {                         /* eq.(4) or eq.(5) in binary32, no draw [R28] */
+            float* g = &n->g[(size_t)i * n_exc + W];
+            double dG = oracle_dg(n, !pot, *g);
+            *g = g_step(n, *g, dG, !pot);
+            n->stats[pot ? 4 : 2]++;
+            if (dG > 0.0) n->stats[pot ? 5 : 3]++;
+            continue;
+          }
           int64_t base = pot ? n->det_p_base[q0] : n->det_d_base[q0];
           uint64_t thr = pot ? n->det_p_thr[q0] : n->det_d_thr[q0];
           uint32_t u = draw(seed, (uint32_t)t, (uint32_t)W, (uint32_t)(i >> 2), TAG_ROUND, i & 3);
@@ -407,15 +494,16 @@ int oracle_present_ex(oracle_net* n, const void* input, int T, uint64_t seed, in
     for (int m = 0; m < nsp; ++m) n->last_post[spikers[m]] = t;      /* spike timer P:87 */
   }
   n->t_next = t0 + T;
-  free(s); free(S); free(cand); free(spikers);
+  free(s); free(S); free(Sg); free(cand); free(spikers);
   return 0;
 }
 
 /* ---------------------------------------------------------------- accessors */
-/* codes: one byte per code (bits <= 8) or one uint16 per code (bits = 16) */
+/* codes: one byte per code (bits <= 8), one uint16 per code (bits = 16), one binary32 G (bits = 32) */
 int oracle_get_weights(const oracle_net* n, void* codes) {
   if (!n || !codes) return E_INVAL;
   size_t nq = (size_t)n->n_in * n->n_exc;
+  if (n->bits == 32) { memcpy(codes, n->g, nq * sizeof(float)); return 0; }
   if (n->bits > 8) { memcpy(codes, n->q, nq * sizeof(uint16_t)); return 0; }
   for (size_t k = 0; k < nq; ++k) ((uint8_t*)codes)[k] = (uint8_t)n->q[k];
   return 0;
@@ -424,6 +512,12 @@ int oracle_get_weights(const oracle_net* n, void* codes) {
 int oracle_set_weights(oracle_net* n, const void* codes) {
   if (!n || !codes) return E_INVAL;
   size_t nq = (size_t)n->n_in * n->n_exc;
+  if (n->bits == 32) {                             /* every G finite and inside [G_min, G_max] [R28] */
+    const float* g = (const float*)codes;
+    for (size_t k = 0; k < nq; ++k) if (!(g[k] >= n->gminf && g[k] <= n->gmaxf)) return E_INVAL;
+    memcpy(n->g, g, nq * sizeof(float));
+    return 0;
+  }
   for (size_t k = 0; k < nq; ++k) {
     int c = n->bits > 8 ? ((const uint16_t*)codes)[k] : ((const uint8_t*)codes)[k];
     if (c > n->q_max) return E_INVAL;

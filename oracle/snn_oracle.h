@@ -55,7 +55,8 @@ int oracle_destroy(oracle_net* net);
 int oracle_present(oracle_net* net, const uint8_t* image, int T, uint64_t seed);
 int oracle_present_ex(oracle_net* net, const void* input, int T, uint64_t seed, int flags, int t0);
 
-/* codes n_in*n_exc row-major [i][j]: uint8 per code for bits <= 8, uint16 per code for bits = 16 */
+/* codes n_in*n_exc row-major [i][j]: uint8 per code for bits <= 8, uint16 per code for bits = 16,
+ * binary32 conductance G per synapse for bits = 32 (R28; set: every G in [G_min, G_max]) */
 int oracle_get_weights(const oracle_net* net, void* codes);
 int oracle_set_weights(oracle_net* net, const void* codes);
 /* last presentation's output raster, T x ceil(n_exc/32) u32, bit j%32 of word j/32 */
@@ -109,6 +110,12 @@ int oracle_lut(const oracle_net* net, int which /*0 enc,1 pot,2 dep,3 det_p_base
 /* One LIF update (eq.(1) Euler, R2/R12) of a non-refractory neuron with integer synaptic sum S. */
 float   oracle_lif_step_fp32(const oracle_net* net, float v, int32_t S);
 int32_t oracle_lif_step_fixed(const oracle_net* net, int32_t v, int32_t S);
+/* 32-bit floating-point conductance ("32-bit floating-point"; R28):
+ * LIF update on the binary32 sum Sg = sum_i G_i; e^y by the binary64 recipe of R28; eqs.(4)(5) at G
+ * (depress = 0: dG_p, 1: dG_d) in binary64. */
+float   oracle_lif_step_fp32g(const oracle_net* net, float v, float Sg);
+double  oracle_exp_recipe(const oracle_net* net, double y);
+double  oracle_dg(const oracle_net* net, int depress, float G);
 
 #ifdef __cplusplus
 }

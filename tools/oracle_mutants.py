@@ -36,6 +36,23 @@ MUTANTS = [
      "if (n->cnt[j] > 0) { n->cnt[j]--; cand[j] = 0; }"),
     ("M8", "R7 lone LAYER spiker not self-inhibited",
      "int other = (nsp >= 2) || (j != spikers[0]);", "int other = 1;"),
+    # 32-bit floating-point conductance arm (NEXT-2, R28)
+    ("M9", "P:84 eq.(4) normalised by (G_max - G_min)",
+     "return p->alpha_p * oracle_exp_recipe(n, -p->beta_p * ((double)G - p->g_min) / span);",
+     "return p->alpha_p * oracle_exp_recipe(n, -p->beta_p * ((double)G - p->g_min));"),
+    ("M10", "P:84 eq.(5) uses alpha_d / beta_d",
+     "return p->alpha_d * oracle_exp_recipe(n, -p->beta_d * (p->g_max - (double)G) / span);",
+     "return p->alpha_d * oracle_exp_recipe(n, -p->beta_p * (p->g_max - (double)G) / span);"),
+    ("M11", "P:83 eq.(3) I = v_pre sum g (32 bit)",
+     "float I  = Sg * n->kV;", "float I  = Sg * n->kI;"),
+    ("M12", "P:89 LTD of the 32-bit arm subtracts eq.(5)",
+     "*g = g_step(n, *g, oracle_dg(n, 1, *g), 1);", "*g = g_step(n, *g, oracle_dg(n, 0, *g), 1);"),
+    ("M13", "R28 exp recipe: Cody-Waite low part",
+     "r = fma(-k, LN2_LO, r);", "r = fma(k, LN2_LO, r);"),
+    ("M14", "R28 clamp at G_max",
+     "if (G1 > n->gmaxf) G1 = n->gmaxf;", ""),
+    ("M15", "R16 window at 32 bits (fp32 branch sees pot)",
+     "double dG = oracle_dg(n, !pot, *g);", "double dG = oracle_dg(n, pot, *g);"),
 ]
 
 
