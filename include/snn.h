@@ -112,11 +112,18 @@ int snn_params_preset(snn_params* p, int preset);
 
 typedef struct snn_handle snn_handle;
 
-/* Create a network n_in -> n_exc with `bits`-bit conductance codes (2, 4, 8 or 16).
+/* Create a network n_in -> n_exc with `bits`-bit conductance codes (2, 4, 8 or 16), or with IEEE binary32
+ * conductances (bits = 32).
  * 16 bits (NEXT-2, "For 16-bit ... after floating point calculation of change in conductance dG,
  * the result is rounded"; R27): every STDP event (stochastic arm) moves the code by the
  * eq.(4)/(5) magnitude rounded by `rounding` instead of one LSB; 16-bit handles run on the per-step
  * engine (SNN_ENGINE_STEP is selected automatically) and cannot be sharded or used for snn_infer.
+ * 32 bits (NEXT-2, "32-bit floating-point"; R28): every conductance is a binary32 G in
+ * [g_min, g_max]; integration sums G in binary32 (I = v_spike * sum G); an STDP event (stochastic arm: gated
+ * by the eqs.(6)(7) draw; deterministic arm: R16 window) sets G = binary32(G +- dG) with dG = eq.(4)/(5) in
+ * binary64 by R28's exp recipe, clamped.  Requires membrane_mode = SNN_MEM_FP32 and rounding =
+ * SNN_ROUND_NEAREST (else SNN_EINVAL); per-step engine, one cluster (784 -> <= 512 columns at 227 KB/CTA),
+ * no sharding, no snn_infer.
  * Conductances are initialised on the device (R4).  SNN_ESIZE if the network does not fit the
  * on-chip layout.  *out receives the handle. */
 int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** out);
@@ -161,7 +168,8 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
                      const uint64_t* const* seeds);
 
 /* Readout.  codes: n_in x n_exc codes, row-major [i][j], one code per byte (bits <= 8) or one
- * little-endian uint16 per code (bits = 16); G = code * 2^-frac_bits.  cap / n are in BYTES. */
+ * little-endian uint16 per code (bits = 16); G = code * 2^-frac_bits.  bits = 32: one little-endian binary32
+ * G per synapse (set: every G finite and in [g_min, g_max], else SNN_EINVAL).  cap / n are in BYTES. */
 int snn_get_weights(snn_handle* h, uint8_t* codes, size_t cap);
 int snn_set_weights(snn_handle* h, const uint8_t* codes, size_t n);
 /* Output raster of the last presented image: T x ceil(n_exc/32) u32, bit j%32 of word j/32. */

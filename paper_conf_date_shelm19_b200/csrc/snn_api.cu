@@ -140,11 +140,19 @@ struct snn_handle {
 
 namespace {
 
+// bytes per code in the readout layout: u8 (<= 8 bits), u16 (16 bits), binary32 G (32 bits, R28)
+size_t code_bytes(int bits) { return bits == 32 ? 4 : (bits > 8 ? 2 : 1); }
+
 int validate(int n_in, int n_exc, int bits, const snn_params* p) {
   if (!p) return fail(SNN_EINVAL, "params is NULL");
   if (n_in < 1 || n_in > 8192) return fail(SNN_EINVAL, "n_in=%d outside [1, 8192]", n_in);
   if (n_exc < 1 || n_exc > (1 << 20)) return fail(SNN_EINVAL, "n_exc=%d outside [1, 2^20]", n_exc);
-  if (bits != 2 && bits != 4 && bits != 8 && bits != 16) return fail(SNN_EINVAL, "bits=%d not in {2,4,8,16}", bits);
+  if (bits != 2 && bits != 4 && bits != 8 && bits != 16 && bits != 32)
+    return fail(SNN_EINVAL, "bits=%d not in {2,4,8,16,32}", bits);
+  // 32-bit floating-point conductance (R28): the fixed recipe needs an integer sum; truncation and eq.(8)
+  // are roundings onto a fixed-point grid (R17), binary32 rounds to nearest
+  if (bits == 32 && p->membrane_mode != SNN_MEM_FP32) return fail(SNN_EINVAL, "bits=32 needs membrane_mode fp32 (R28)");
+  if (bits == 32 && p->rounding != SNN_ROUND_NEAREST) return fail(SNN_EINVAL, "bits=32 rounds to nearest only (R28)");
   if (!(p->dt_ms > 0.0)) return fail(SNN_EINVAL, "dt_ms must be > 0");
   if (!(p->f_min_hz >= 0.0 && p->f_max_hz >= p->f_min_hz)) return fail(SNN_EINVAL, "need 0 <= f_min <= f_max");
   if (p->f_max_hz * p->dt_ms * 1e-3 > 1.0) return fail(SNN_EINVAL, "f_max * dt > 1 (spike probability > 1)");
@@ -194,6 +202,11 @@ void fill_static(const snn_handle* h, NetDesc& d) {
   d.t_ref = p.t_ref_steps; d.t_inh = p.t_inh_steps; d.wta_mode = p.wta_mode; d.inh_mode = p.inh_mode;
   d.stdp_mode = p.stdp_mode; d.t_ltp = p.t_ltp_steps;
   d.L_pot = h->L_pot; d.L_dep = h->L_dep;
+  d.alpha_p = p.alpha_p; d.beta_p = p.beta_p; d.alpha_d = p.alpha_d; d.beta_d = p.beta_d;
+  d.g_min = p.g_min; d.g_max = p.g_max;
+  d.ecoef[0] = 1.0;                                   // R28: 1/m! by c_m = c_{m-1} / m (binary64)
+  for (int m = 1; m <= snn::kExpDeg; ++m) d.ecoef[m] = d.ecoef[m - 1] / (double)m;
+  d.kV = (float)p.v_spike; d.gminf = (float)p.g_min; d.gmaxf = (float)p.g_max;
   d.thr_enc = h->d_enc; d.pot_m1 = h->d_pot; d.dep_m1 = h->d_dep;
   d.det_base_p = h->d_dbp; d.det_thr_p = h->d_dtp; d.det_base_d = h->d_dbd; d.det_thr_d = h->d_dtd;
   d.wslices = h->d_w;
@@ -467,8 +480,8 @@ int create_impl(int n_in, int n_exc, int bits, const snn_params* p, int col_base
   h->n_in = n_in; h->n_exc = n_exc; h->bits = bits;
   h->col_base = col_base; h->n_exc_total = n_exc_total; h->shard = shard; h->world = world;
   h->frac_bits = p->frac_bits > 0 ? p->frac_bits : bits;
-  h->q_max = (1 << bits) - 1;
-  if (h->frac_bits != bits) {
+  h->q_max = bits == 32 ? 0 : (1 << bits) - 1;      // 32 bits: binary32 conductance, no code grid (R28)
+  if (bits <= 16 && h->frac_bits != bits) {
     const double cap = std::floor(std::ldexp(p->g_max, h->frac_bits));
     if (cap < h->q_max) h->q_max = (int)cap;
   }
@@ -522,7 +535,8 @@ int create_impl(int n_in, int n_exc, int bits, const snn_params* p, int col_base
   int smem_optin = 0;
   cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, h->dev);
   h->ngroups = (n_exc + 31) / 32;
-  // 16-bit codes (NEXT-2, R27) run on the per-step engine: the event kernels pack <= 8-bit codes in SWAR lanes
+  // 16-bit codes (NEXT-2, R27) and binary32 conductances (R28) run on the per-step engine: the event kernels
+  // pack <= 8-bit codes in SWAR lanes
   h->engine = (p->engine == SNN_ENGINE_STEP || bits > 8) ? SNN_ENGINE_STEP : SNN_ENGINE_EVENT;
   // the lean kernel covers the paper's default learning mode; SNN_NO_LEAN=1 disables it
   // (LAYER WTA is instantiated unsharded only)
@@ -638,7 +652,7 @@ int create_impl(int n_in, int n_exc, int bits, const snn_params* p, int col_base
   ALLOC(h->d_lpost, (size_t)n_exc);
   ALLOC(h->d_lpre, (size_t)n_in);
   ALLOC(h->d_stats, SNN_NSTATS);
-  ALLOC(h->d_codes, (size_t)n_in * n_exc * (bits > 8 ? 2 : 1));
+  ALLOC(h->d_codes, (size_t)n_in * n_exc * code_bytes(bits));
   ALLOC(h->d_bad, 1);
   if (world > 1) {
     ALLOC(h->d_mbox, 1);
@@ -978,7 +992,7 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
 int snn_get_weights(snn_handle* h, uint8_t* codes, size_t cap) {
   int rc = check_handle(h);
   if (rc) return rc;
-  const size_t n = (size_t)h->n_in * h->n_exc * (h->bits > 8 ? 2 : 1);     // bytes
+  const size_t n = (size_t)h->n_in * h->n_exc * code_bytes(h->bits);     // bytes
   if (!codes) return fail(SNN_EINVAL, "codes is NULL");
   if (cap < n) return fail(SNN_ESIZE, "need %zu bytes", n);
   DevGuard g(h->dev);
@@ -995,17 +1009,22 @@ int snn_set_weights(snn_handle* h, const uint8_t* codes, size_t n) {
   int rc = check_handle(h);
   if (rc) return rc;
   const size_t ncodes = (size_t)h->n_in * h->n_exc;
-  const size_t need = ncodes * (h->bits > 8 ? 2 : 1);                          // bytes
+  const size_t need = ncodes * code_bytes(h->bits);                          // bytes
   if (!codes) return fail(SNN_EINVAL, "codes is NULL");
   if (n < need) return fail(SNN_ESIZE, "need %zu bytes", need);
   DevGuard g(h->dev);
   CUDA_TRY(cudaMemcpyAsync(h->d_codes, codes, need, is_device_ptr(codes) ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice,
                            h->stream));
   CUDA_TRY(cudaMemsetAsync(h->d_bad, 0, sizeof(int), h->stream));
-  CUDA_TRY(snn::launch_check_codes(h->d_codes, ncodes, h->bits, h->q_max, h->d_bad, h->stream));
+  if (h->bits == 32)
+    CUDA_TRY(snn::launch_check_g(reinterpret_cast<const float*>(h->d_codes), ncodes, (float)h->p.g_min, (float)h->p.g_max,
+                                 h->d_bad, h->stream));
+  else
+    CUDA_TRY(snn::launch_check_codes(h->d_codes, ncodes, h->bits, h->q_max, h->d_bad, h->stream));
   int bad = 0;
   CUDA_TRY(cudaMemcpyAsync(&bad, h->d_bad, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
   CUDA_TRY(cudaStreamSynchronize(h->stream));
+  if (bad && h->bits == 32) return fail(SNN_EINVAL, "%d conductances outside [g_min, g_max] (R28)", bad);
   if (bad) return fail(SNN_EINVAL, "%d codes exceed q_max=%d", bad, h->q_max);
   NetDesc d;
   fill_static(h, d);
@@ -1226,7 +1245,7 @@ int snn_infer(snn_handle* h, const uint8_t* images, int n_images, int T, const u
   if (n_images < 0 || T < 0) return fail(SNN_EINVAL, "negative n_images / T");
   if (T > 65535) return fail(SNN_EINVAL, "T=%d exceeds 65535 for inference", T);
   if (h->world > 1) return fail(SNN_EINVAL, "inference runs on unsharded handles");
-  if (h->bits > 8) return fail(SNN_EINVAL, "inference supports 2/4/8-bit codes (16-bit: NEXT-2 learning only)");
+  if (h->bits > 8) return fail(SNN_EINVAL, "inference supports 2/4/8-bit codes (16/32-bit: NEXT-2 learning only)");
   if (h->n_exc > snn::kInferMaxCols) return fail(SNN_ESIZE, "n_exc=%d exceeds %d for inference", h->n_exc,
                                                  snn::kInferMaxCols);
   if (n_images == 0) return SNN_OK;

@@ -18,6 +18,8 @@ enum : int { FLAG_RASTER_INPUT = 1, FLAG_KEEP_STATE = 2, FLAG_RECORD_INPUT = 4, 
 // Everything one network needs inside the persistent kernel.  Built per launch on the host.
 struct Mailbox;
 
+constexpr int kExpDeg = 13;   // degree of the Taylor polynomial of R28's e^y recipe
+
 struct NetDesc {
   // geometry
   int n_in, n_exc, bits, q_max;
@@ -33,6 +35,11 @@ struct NetDesc {
   int Vth, Vreset, Vinit;
   int t_ref, t_inh, wta_mode, inh_mode, stdp_mode, t_ltp;
   int L_pot, L_dep;
+  // 32-bit floating-point conductance (bits = 32, NEXT-2, R28): eqs.(4)(5) parameters, the
+  // binary64 e^y recipe's Taylor coefficients 1/m! (host-built, c_m = c_{m-1}/m), I = S * (float)v_spike
+  double alpha_p, beta_p, alpha_d, beta_d, g_min, g_max;
+  double ecoef[kExpDeg + 1];
+  float kV, gminf, gmaxf;
   // tables (device)
   const unsigned long long* thr_enc;   // [256]      event iff u <  thr
   const uint32_t* pot_m1;              // [L_pot]    event iff u <= thr - 1   (thr >= 1 for D < L)
@@ -122,6 +129,7 @@ cudaError_t query_max_clusters(int cs, int nthr, size_t smem, int* out);
 cudaError_t launch_init_weights(const NetDesc& d, uint64_t init_seed, cudaStream_t s);
 cudaError_t launch_pack_weights(const NetDesc& d, const void* codes, cudaStream_t s);      // u8 / u16 (bits 16) codes
 cudaError_t launch_unpack_weights(const NetDesc& d, void* codes, cudaStream_t s);
+cudaError_t launch_check_g(const float* g, size_t n, float gmin, float gmax, int* bad, cudaStream_t s);
 cudaError_t launch_check_codes(const void* codes, size_t n, int bits, int q_max, int* bad, cudaStream_t s);
 size_t present_smem_bytes(int n_in, int wpr, int L_pot, int L_dep, int q_max, int nthr);
 

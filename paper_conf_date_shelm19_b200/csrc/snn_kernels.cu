@@ -54,6 +54,43 @@ size_t present_smem_bytes(int n_in, int slice_words, int L_pot, int L_dep, int q
 
 __device__ __forceinline__ int slice_words_of(const NetDesc& d) { return d.slice_words; }
 
+// ---- 32-bit floating-point conductance (bits = 32, NEXT-2, R28); every operation an IEEE-rounded
+// intrinsic so that nvcc contracts nothing and the result equals R28's recipe bit for bit
+constexpr double kInvLn2 = 0x1.71547652b82fep+0;   // 1/ln 2
+constexpr double kLn2Hi = 0x1.62e42feep-1;         // Cody-Waite split of ln 2 (11 trailing zero bits)
+constexpr double kLn2Lo = 0x1.a39ef35793c76p-33;
+
+// e^y: y = k ln2 + r (k = rint(y / ln2), two fused multiply-adds), e^r by the degree-kExpDeg Taylor polynomial
+// in Horner form (coefficients 1/m! built on the host), times 2^k
+__device__ __noinline__ double exp_r28(const NetDesc& d, double y) {
+  const double k = rint(__dmul_rn(y, kInvLn2));
+  double r = __fma_rn(-k, kLn2Hi, y);
+  r = __fma_rn(-k, kLn2Lo, r);
+  double e = d.ecoef[kExpDeg];
+#pragma unroll
+  for (int m = kExpDeg - 1; m >= 0; --m) e = __fma_rn(e, r, d.ecoef[m]);
+  return scalbn(e, (int)k);
+}
+
+// eqs.(4)(5) P:84 at binary32 G, in binary64: dG_p = alpha_p e^{((-beta_p)(G - G_min)) / (G_max - G_min)},
+// dG_d = alpha_d e^{((-beta_d)(G_max - G)) / (G_max - G_min)}
+__device__ __forceinline__ double dg_r28(const NetDesc& d, bool depress, float G) {
+  const double span = __dsub_rn(d.g_max, d.g_min);
+  const double Gd = (double)G;
+  if (!depress) return __dmul_rn(d.alpha_p, exp_r28(d, __ddiv_rn(__dmul_rn(-d.beta_p, __dsub_rn(Gd, d.g_min)), span)));
+  return __dmul_rn(d.alpha_d, exp_r28(d, __ddiv_rn(__dmul_rn(-d.beta_d, __dsub_rn(d.g_max, Gd)), span)));
+}
+
+// G' = binary32(G +- dG) (binary64 add, one rounding to nearest), clamped to [G_min, G_max]
+__device__ __forceinline__ uint32_t gstep_r28(const NetDesc& d, uint32_t word, bool depress) {
+  const float G = __uint_as_float(word);
+  const double dG = dg_r28(d, depress, G);
+  float G1 = __double2float_rn(depress ? __dsub_rn((double)G, dG) : __dadd_rn((double)G, dG));
+  G1 = G1 < d.gminf ? d.gminf : G1;
+  G1 = G1 > d.gmaxf ? d.gmaxf : G1;
+  return __float_as_uint(G1);
+}
+
 // ------------------------------------------------------------------ the persistent step kernel
 __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_constant__ LaunchParams lp) {
   extern __shared__ __align__(16) unsigned char smem[];
@@ -94,11 +131,12 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
   const int ngrp_cta = g1 - g0;
   const bool mycol = tid < ncols;
   const int j = col0 + tid;
-  const int lg = bits == 2 ? 4 : (bits == 4 ? 3 : (bits == 8 ? 2 : 1));   // log2(codes per u32 word)
+  const int lg = bits == 2 ? 4 : (bits == 4 ? 3 : (bits == 8 ? 2 : (bits == 16 ? 1 : 0)));   // log2(codes per word)
   const int wj = tid >> lg;
   const int sh = (tid & ((1 << lg) - 1)) * bits;
-  const uint32_t fmask = (1u << bits) - 1u;
+  const uint32_t fmask = bits == 32 ? 0xFFFFFFFFu : (1u << bits) - 1u;
   const bool wide = bits > 8;       // 16-bit codes: STDP steps by eqs.(4)(5) magnitudes, not 1 LSB (R27)
+  const bool f32 = bits == 32;      // binary32 conductance, one column per word (R28)
   const int nq4 = (n_in + 3) >> 2;
   const bool fixed = d.membrane_mode == 1;
   const bool hard = d.wta_mode == 0;
@@ -213,8 +251,12 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
       bool cand = false;
       if (mycol && !floor_mode) {
         int S = 0;
+        float Sg = 0.0f;                                   // R28: binary32 sum, ascending rows, from +0
         const uint32_t* wcol = s_w + wj;
-        for (int a = 0; a < nact; ++a) S += (int)((wcol[(int)s_alist[a] * wpr] >> sh) & fmask);
+        if (f32)
+          for (int a = 0; a < nact; ++a) Sg = __fadd_rn(Sg, __uint_as_float(wcol[(int)s_alist[a] * wpr]));
+        else
+          for (int a = 0; a < nact; ++a) S += (int)((wcol[(int)s_alist[a] * wpr] >> sh) & fmask);
         if (cnt_r > 0) {
           --cnt_r;
         } else if (fixed) {
@@ -225,7 +267,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
           cand = v_r > d.Vth;
         } else {
           const float vf = __int_as_float(v_r);
-          const float I = __fmul_rn(__int2float_rn(S), d.kI);
+          const float I = f32 ? __fmul_rn(Sg, d.kV) : __fmul_rn(__int2float_rn(S), d.kI);
           const float x = __fadd_rn(I, d.ief);
           const float y = __fmaf_rn(d.cf, x, d.af);
           const float dv = __fmaf_rn(d.bf, vf, y);
@@ -283,7 +325,9 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
             if (pick(u, j & 3) <= thr) {
               ++ltd_events;
               uint32_t* p = wcol + i * wpr;
-              if (!wide) {
+              if (f32) {                                        // eq.(5) in binary32 (R28); own word
+                *p = gstep_r28(d, *p, true);
+              } else if (!wide) {
                 if ((*p >> sh) & fmask) atomicSub(p, 1u << sh);   // other fields of the word may move concurrently
               } else {                                          // eq.(5) rounded (eq.(8), R27)
                 const int q0 = (int)((*p >> sh) & fmask);
@@ -366,7 +410,9 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
                   ++ltp_events;
                   const uint32_t word = *p;
                   const int q0 = (int)((word >> wsh) & fmask);
-                  if (!wide) {
+                  if (f32) {                                // eq.(4) in binary32 (R28)
+                    *p = gstep_r28(d, word, false);
+                  } else if (!wide) {
                     if (q0 < qmax) *p = word + (1u << wsh);
                   } else {                                  // eq.(4) rounded (eq.(8), R27)
                     const uint4 u2 = philox((uint32_t)t, (uint32_t)Wg, (uint32_t)grp, TAG_ROUND, seed);
@@ -375,6 +421,12 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
                     *p = (word & ~(fmask << wsh)) | ((uint32_t)q1 << wsh);
                   }
                 }
+              } else if (f32) {                             // R16 window, eqs.(4)(5) in binary32 (R28)
+                const bool pot = lp >= 0 && (t - lp) <= d.t_ltp;
+                const float G = __uint_as_float(*p);
+                *p = gstep_r28(d, *p, !pot);
+                if (dg_r28(d, !pot, G) > 0.0) { if (pot) ++ltp_events; else ++ltd_events; }
+                if (pot) ++ltp_trials; else ++ltd_trials;
               } else {
                 const uint32_t word = *p;
                 const int q0 = (int)((word >> wsh) & fmask);
@@ -516,16 +568,23 @@ __global__ void init_weights_kernel(const NetDesc d, unsigned long long init_see
     if (jl >= ncols) break;
     const int jg = d.col_base + col0 + jl;                  // global column (a shard starts at col_base)
     const uint4 u = philox((uint32_t)i, (uint32_t)(jg >> 2), 0u, TAG_INIT, init_seed);   // R4
+    if (d.bits == 32) {                                     // R28: G = binary32(G_max (u >> 8) 2^-24)
+      word = __float_as_uint(__double2float_rn(__dmul_rn(d.g_max, scalbn((double)(pick(u, jg & 3) >> 8), -24))));
+      break;
+    }
     const uint32_t code = (uint32_t)(((unsigned long long)pick(u, jg & 3) * (unsigned long long)(d.q_max + 1)) >> 32);
     word |= code << (c * d.bits);
   }
   d.wslices[gid] = word;
 }
 
-// codes: one byte per code (bits <= 8) or one uint16 per code (bits = 16), row-major [i][j]
+// codes: one byte per code (bits <= 8), one uint16 per code (bits = 16) or the binary32 G (bits = 32, R28),
+// row-major [i][j]
 __device__ __forceinline__ uint32_t code_at(const NetDesc& d, const void* codes, size_t k) {
+  if (d.bits == 32) return static_cast<const uint32_t*>(codes)[k];
   return d.bits > 8 ? (uint32_t)static_cast<const uint16_t*>(codes)[k] : (uint32_t)static_cast<const uint8_t*>(codes)[k];
 }
+__device__ __forceinline__ uint32_t field_mask(int bits) { return bits == 32 ? 0xFFFFFFFFu : (1u << bits) - 1u; }
 
 __global__ void pack_weights_kernel(const NetDesc d, const void* __restrict__ codes) {
   const size_t gid = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -538,7 +597,7 @@ __global__ void pack_weights_kernel(const NetDesc d, const void* __restrict__ co
   for (int c = 0; c < cpw; ++c) {
     const int jl = w * cpw + c;
     if (jl >= ncols) break;
-    word |= (code_at(d, codes, (size_t)i * d.n_exc + col0 + jl) & ((1u << d.bits) - 1u)) << (c * d.bits);
+    word |= (code_at(d, codes, (size_t)i * d.n_exc + col0 + jl) & field_mask(d.bits)) << (c * d.bits);
   }
   d.wslices[gid] = word;
 }
@@ -552,9 +611,10 @@ __global__ void unpack_weights_kernel(const NetDesc d, void* __restrict__ codes)
   for (int c = 0; c < cpw; ++c) {
     const int jl = w * cpw + c;
     if (jl >= ncols) break;
-    const uint32_t code = (word >> (c * d.bits)) & ((1u << d.bits) - 1u);
+    const uint32_t code = (word >> (c * d.bits)) & field_mask(d.bits);
     const size_t k = (size_t)i * d.n_exc + col0 + jl;
-    if (d.bits > 8) static_cast<uint16_t*>(codes)[k] = (uint16_t)code;
+    if (d.bits == 32) static_cast<uint32_t*>(codes)[k] = code;
+    else if (d.bits > 8) static_cast<uint16_t*>(codes)[k] = (uint16_t)code;
     else static_cast<uint8_t*>(codes)[k] = (uint8_t)code;
   }
 }
@@ -564,6 +624,14 @@ __global__ void check_codes_kernel(const void* __restrict__ codes, size_t n, int
   if (gid >= n) return;
   const int c = bits > 8 ? (int)static_cast<const uint16_t*>(codes)[gid] : (int)static_cast<const uint8_t*>(codes)[gid];
   if (c > q_max) atomicAdd(bad, 1);
+}
+
+// R28: every binary32 conductance finite and inside [G_min, G_max] (NaN fails both comparisons)
+__global__ void check_g_kernel(const float* __restrict__ g, size_t n, float gmin, float gmax, int* bad) {
+  const size_t gid = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (gid >= n) return;
+  const float x = g[gid];
+  if (!(x >= gmin && x <= gmax)) atomicAdd(bad, 1);
 }
 
 static unsigned grid_for(size_t n, int bs) { return (unsigned)((n + bs - 1) / bs); }
@@ -581,6 +649,10 @@ cudaError_t launch_pack_weights(const NetDesc& d, const void* codes, cudaStream_
 cudaError_t launch_unpack_weights(const NetDesc& d, void* codes, cudaStream_t s) {
   const size_t n = (size_t)d.cs * d.slice_words;
   unpack_weights_kernel<<<grid_for(n, 256), 256, 0, s>>>(d, codes);
+  return cudaGetLastError();
+}
+cudaError_t launch_check_g(const float* g, size_t n, float gmin, float gmax, int* bad, cudaStream_t s) {
+  check_g_kernel<<<grid_for(n, 256), 256, 0, s>>>(g, n, gmin, gmax, bad);
   return cudaGetLastError();
 }
 cudaError_t launch_check_codes(const void* codes, size_t n, int bits, int q_max, int* bad, cudaStream_t s) {

@@ -169,7 +169,7 @@ class Network:
         """shard=(rank, world): this object is shard `rank` of an n_exc-column network split over
         `world` ranks (include/snn.h snn_create_shard); self.n_exc becomes the shard's own columns."""
         self.n_in, self.n_exc, self.bits = n_in, n_exc, bits
-        self.params = params if params is not None else preset({2: "2b", 4: "4b", 8: "8b", 16: "16b"}[bits])
+        self.params = params if params is not None else preset({2: "2b", 4: "4b", 8: "8b", 16: "16b", 32: "16b"}[bits])
         for k, v in overrides.items():
             setattr(self.params, k, v)
         self._h = ctypes.c_void_p()
@@ -235,7 +235,8 @@ class Network:
 
     @property
     def code_dtype(self):
-        return np.uint16 if self.bits > 8 else np.uint8
+        """uint8 codes (<= 8 bits), uint16 codes (16 bits), binary32 conductance (32 bits, R28)"""
+        return np.float32 if self.bits == 32 else (np.uint16 if self.bits > 8 else np.uint8)
 
     def weights(self) -> np.ndarray:
         out = np.empty((self.n_in, self.n_exc), dtype=self.code_dtype)

@@ -74,10 +74,18 @@ def test_invalid_params_rejected_before_cuda(bad):
     assert e.value.rc == S.SNN_EINVAL
 
 
-@pytest.mark.parametrize("bits", [0, 1, 3, 12, 32])
+@pytest.mark.parametrize("bits", [0, 1, 3, 12, 24, 64])
 def test_invalid_bits_rejected(bits):
     with pytest.raises(P.SnnError) as e:
         P.Network(784, 10, bits, P.preset("8b"))
+    assert e.value.rc == S.SNN_EINVAL
+
+
+@pytest.mark.parametrize("bad", [dict(membrane_mode=1), dict(rounding=0), dict(rounding=2)])
+def test_fp32_conductance_mode_constraints(bad):
+    """bits = 32 (R28): binary32 conductance needs fp32 membranes and round-to-nearest; rejected before CUDA."""
+    with pytest.raises(P.SnnError) as e:
+        P.Network(784, 10, 32, P.preset("16b", **bad))
     assert e.value.rc == S.SNN_EINVAL
 
 

@@ -1,0 +1,141 @@
+"""NEXT-2 GPU <-> oracle parity: 32-bit floating-point conductance ("32-bit floating-point (accuracy
+96.1%)"; "For 16-bit and 32-bit learning, after floating point calculation of change in conductance dG,
+the result is rounded to a value that can be represented in the current bit width"; reading DESIGN.md R28).
+
+Both sides execute the same sequence of IEEE-rounded operations (binary32 sums in ascending row order, the
+fp32 LIF recipe, binary64 eqs.(4)(5) through R28's exp recipe, one rounding to binary32 per event), so
+conductances, rasters, timers and counters are compared bit for bit; membranes within 1e-5 relative (the
+north_star's fp32 bar; bit-exact in practice)."""
+import numpy as np
+import pytest
+
+import synthdata
+from oracle import oracle as O
+
+pytestmark = pytest.mark.gpu
+
+
+def _pair(n_in, n_exc, p):
+    import paper_conf_date_shelm19_b200 as P
+    return P.Network(n_in, n_exc, 32, P.params_from_dict(p)), O.OracleNet(n_in, n_exc, 32, p)
+
+
+def _compare_state(g, o, n_in, n_exc):
+    assert np.array_equal(g.spikes(), o.spikes()), "raster"
+    gw, ow = g.weights(), o.weights()
+    assert gw.dtype == np.float32
+    bad = np.argwhere(gw.view(np.uint32) != ow.view(np.uint32))
+    assert bad.size == 0, f"{len(bad)} conductances differ, first {bad[:3].tolist()}: {gw[tuple(bad[0])]} vs {ow[tuple(bad[0])]}"
+    assert np.array_equal(g.stats()[:6], o.stats()[:6]), "counters"
+    sg, so = O.unpack_state(g.state(), n_in, n_exc), O.unpack_state(o.state(), n_in, n_exc)
+    for k in ("cnt", "last_post", "last_pre"):
+        assert np.array_equal(sg[k], so[k]), k
+    np.testing.assert_allclose(sg["v"], so["v"], rtol=1e-5, atol=0)
+
+
+def _compare(g, o, imgs, T, seeds, n_in, n_exc):
+    for img, sd in zip(imgs, seeds):
+        g.reset_stats()
+        g.present(img, T, int(sd))
+        o.present(img, T, int(sd))
+        _compare_state(g, o, n_in, n_exc)
+
+
+def test_fp32_init_and_roundtrip(gpu):
+    import paper_conf_date_shelm19_b200 as P
+    for g_max in (1.0, 0.75):
+        p = O.params("16b", init_seed=7, g_max=g_max)
+        g, o = _pair(784, 100, p)
+        w = g.weights()
+        assert w.dtype == np.float32 and w.max() < g_max and w.min() >= 0.0
+        assert np.array_equal(w.view(np.uint32), o.weights().view(np.uint32))
+    rng = np.random.default_rng(1)
+    c = (rng.random((784, 100)) * 0.75).astype(np.float32)
+    g.set_weights(c)
+    assert np.array_equal(g.weights(), c)
+    for bad in (0.7501, -1e-7, np.nan, np.inf):
+        c2 = c.copy()
+        c2[3, 4] = bad
+        with pytest.raises(P.SnnError):
+            g.set_weights(c2)
+    assert np.array_equal(g.weights(), c)
+
+
+@pytest.mark.parametrize("wta", [0, 1])
+def test_fp32_stochastic_c1(gpu, wta):
+    """784 -> 100, Table I "16 bit" row (gamma 0.9): eqs.(6)(7)-gated events of eq.(4)/(5) size, 4 images."""
+    p = O.params("16b", wta_mode=wta, init_seed=3)
+    g, o = _pair(784, 100, p)
+    _compare(g, o, synthdata.images(4, "mnist", start=30), 100, synthdata.seeds(4, base_seed=12), 784, 100)
+    assert int(o.stats()[3]) + int(o.stats()[5]) > 0
+
+
+@pytest.mark.parametrize("wta", [0, 1])
+def test_fp32_deterministic_c1(gpu, wta):
+    """Deterministic arm (R16 window, eqs.(4)(5) magnitudes in binary32): the floating-point baseline of P:82."""
+    p = O.params("16b", stdp_mode=1, wta_mode=wta, init_seed=4)
+    g, o = _pair(784, 100, p)
+    _compare(g, o, synthdata.images(3, "mnist", start=40), 150, synthdata.seeds(3, base_seed=13), 784, 100)
+    assert int(o.stats()[1]) > 0
+
+
+@pytest.mark.parametrize("stdp,wta", [(0, 0), (0, 1), (1, 1)])
+def test_fp32_c2_shape(gpu, stdp, wta):
+    """784 -> 400 (C2's network: 1.25 MB of binary32 conductance over one cluster), 350-step presentations."""
+    p = O.params("16b", stdp_mode=stdp, wta_mode=wta, init_seed=5)
+    g, o = _pair(784, 400, p)
+    assert g.info()["cluster_size"] >= 7
+    _compare(g, o, synthdata.images(2, "mnist", start=70), 350, synthdata.seeds(2, base_seed=2), 784, 400)
+
+
+def test_fp32_high_frequency_row(gpu):
+    """Table I "high frequency" row (5-78 Hz, tau_pot 80, tau_dep 5), T = 100, fashion-shaped input."""
+    p = O.params("hf", init_seed=8)
+    g, o = _pair(784, 64, p)
+    _compare(g, o, synthdata.images(3, "fashion", start=5), 100, synthdata.seeds(3, base_seed=5), 784, 64)
+
+
+def test_fp32_ragged_small(gpu):
+    """Ragged shapes: 37 columns (a partial 32-column group), 50 inputs (a partial input word)."""
+    p = O.params("16b", f_min_hz=20.0, f_max_hz=200.0, init_seed=6)
+    g, o = _pair(50, 37, p)
+    imgs = synthdata.images(3, "fashion", start=2)[:, :50]
+    _compare(g, o, imgs, 80, synthdata.seeds(3, base_seed=21), 50, 37)
+
+
+def test_fp32_batch_matches_sequential_oracle(gpu):
+    """One snn_present_batch launch of 6 images (weights resident on chip across images) against the oracle
+    presenting them one by one: final conductances, per-image spike counts, last raster and state."""
+    import paper_conf_date_shelm19_b200 as P
+    p = O.params("16b", init_seed=9)
+    g, o = _pair(784, 128, p)
+    imgs = synthdata.images(6, "mnist", start=90)
+    seeds = synthdata.seeds(6, base_seed=31)
+    counts = np.zeros(6, np.int32)
+    g.present_batch(imgs, 100, seeds, spike_counts=counts)
+    want = []
+    for img, sd in zip(imgs, seeds):
+        o.present(img, 100, int(sd))
+        want.append(int(O.unpack_bits(o.spikes(), 128).sum()))
+    assert counts.tolist() == want
+    assert np.array_equal(g.weights().view(np.uint32), o.weights().view(np.uint32))
+    assert np.array_equal(g.spikes(), o.spikes())
+    sg, so = O.unpack_state(g.state(), 784, 128), O.unpack_state(o.state(), 784, 128)
+    for k in ("cnt", "last_post", "last_pre"):
+        assert np.array_equal(sg[k], so[k]), k
+
+
+def test_fp32_rejections(gpu):
+    import paper_conf_date_shelm19_b200 as P
+    g = P.Network(784, 64, 32, P.preset("16b"))
+    assert g.info()["engine"] == 1                       # per-step engine selected automatically
+    with pytest.raises(P.SnnError):
+        g.infer(synthdata.images(1), 10, synthdata.seeds(1))
+    with pytest.raises(P.SnnError):
+        P.Network(784, 640, 32, P.preset("16b"), shard=(0, 2))
+    with pytest.raises(P.SnnError):
+        P.Network(784, 64, 32, P.params_from_dict(O.params("16b", membrane_mode=1)))
+    with pytest.raises(P.SnnError):
+        P.Network(784, 64, 32, P.params_from_dict(O.params("16b", rounding=2)))
+    with pytest.raises(P.SnnError):                      # 5 MB of binary32 > one cluster's shared memory
+        P.Network(784, 1600, 32, P.preset("16b"))
