@@ -221,7 +221,10 @@ int snn_get_trace(snn_handle* h, uint64_t* out, size_t cap);
  * the event engine each shard publishes a 16-byte summary (earliest crossing step,
  * crossing count, best WTA key) into every shard's mailbox in device memory (peer stores over NVLink)
  * and every shard applies the same reduction: the exchange step of P:88 §III-B's lateral inhibition
- * across GPUs.  Event engine only.  All shards of a world must run the same presentation calls
+ * across GPUs.  On the per-step engine (SNN_ENGINE_STEP; 16-bit codes and binary32 conductances always run
+ * there) the exchange is per step: each shard publishes its cluster's best WTA key (HARD) or spiker count
+ * (LAYER) the same way, so a 784 -> 6400 network at 16 / 32 bits (10 / 20 MB, beyond one cluster's shared
+ * memory) runs as 4 / 7 shards.  All shards of a world must run the same presentation calls
  * (inputs, seeds, T, flags) in the same order; a rank that stops answering makes the others trap
  * after 20 s instead of hanging.
  * Readouts (weights, spikes, state) of a shard cover its own columns: n_in x n_exc_local codes, a

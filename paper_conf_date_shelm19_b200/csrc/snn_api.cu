@@ -415,6 +415,7 @@ int present_impl(snn_handle* h, const void* input, int n_images, int T, const ui
                                               h->stream));
     prof_mark(h);
   } else {
+    if ((rc = shard_arm(h, d))) return rc;
     lp.single = d;
     prof_mark(h);
     CUDA_TRY(snn::launch_present(lp, 1, h->cs, h->nthr, h->smem, h->stream));
@@ -720,7 +721,10 @@ int snn_create_shard(int n_in, int n_exc_total, int bits, const snn_params* p, i
   if (rc) return rc;
   if (world < 1 || world > snn::kMaxWorld) return fail(SNN_EINVAL, "world=%d outside [1, %d]", world, snn::kMaxWorld);
   if (shard < 0 || shard >= world) return fail(SNN_EINVAL, "shard=%d outside [0, %d)", shard, world);
-  if (p->engine != SNN_ENGINE_EVENT || bits > 8) return fail(SNN_EINVAL, "column sharding needs the event engine (bits <= 8)");
+  // <= 8-bit codes shard on the event engines (one exchange per post-spike epoch), 16-bit codes and binary32
+  // conductances on the per-step engine (one exchange per step): a 784 -> 6400 network at 16 / 32 bits spreads
+  // over 4 / 8 clusters
+  if (p->engine == SNN_ENGINE_EVENT_GENERAL && bits > 8) return fail(SNN_EINVAL, "bits > 8 run on the per-step engine");
   const int G = (n_exc_total + 31) / 32;
   if (G < world) return fail(SNN_EINVAL, "%d column groups of 32 cannot feed %d shards", G, world);
   const int lo = 32 * (int)(((long long)shard * G) / world);
@@ -908,7 +912,7 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
     if (!rc) {
       d.images = img; d.seeds = sd; d.raster_out = h->d_raster;
       if (ev) rc = event_prepass(h, d, img, nullptr, n_images, T, 0, sd);
-      if (!rc && ev) rc = shard_arm(h, d);
+      if (!rc) rc = shard_arm(h, d);
     }
     h->stream = own;
     if (rc) return rc;

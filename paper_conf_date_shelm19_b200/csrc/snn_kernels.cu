@@ -130,7 +130,16 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
   const int ncols = min(g1 * 32, n_exc) - col0;
   const int ngrp_cta = g1 - g0;
   const bool mycol = tid < ncols;
-  const int j = col0 + tid;
+  const int j = col0 + tid;                          // this CTA-slice column (state arrays are per shard)
+  // column sharding: this network is columns [col_base, col_base + n_exc) of a network split over
+  // `world` ranks; every random draw and WTA key uses GLOBAL column indices, and per step the clusters' WTA summaries
+  // meet in every rank's mailbox, so the union of the shards is the unsharded network bit for bit
+  const int cbase = d.col_base;
+  const int jg = cbase + j;                          // global column
+  const int world = d.world;
+  const bool sharded = world > 1;
+  const uint32_t seq0 = sharded ? (uint32_t)ld_relaxed_sys_s32(reinterpret_cast<const int*>(&d.mbox->seq)) : 0u;
+  uint32_t nxch = 0;                                 // exchanges of this launch (one per step)
   const int lg = bits == 2 ? 4 : (bits == 4 ? 3 : (bits == 8 ? 2 : (bits == 16 ? 1 : 0)));   // log2(codes per word)
   const int wj = tid >> lg;
   const int sh = (tid & ((1 << lg) - 1)) * bits;
@@ -284,7 +293,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
         uint32_t ord = 0, lo = 0;
         if (cand) {
           ord = fixed ? ((uint32_t)v_r ^ 0x80000000u) : float_ord((uint32_t)v_r);
-          lo = 0xFFFFFFFFu - (uint32_t)j;
+          lo = 0xFFFFFFFFu - (uint32_t)jg;
         }
         const uint32_t mh = __reduce_max_sync(FULL, ord);
         const uint32_t ml = __reduce_max_sync(FULL, ord == mh ? lo : 0u);
@@ -320,9 +329,9 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
           uint32_t* wcol = s_w + wj;
           for (int a = 0; a < nact; ++a) {
             const int i = s_alist[a];
-            const uint4 u = philox((uint32_t)t, (uint32_t)i, (uint32_t)(j >> 2), TAG_LTD, seed);
+            const uint4 u = philox((uint32_t)t, (uint32_t)i, (uint32_t)(jg >> 2), TAG_LTD, seed);
             ++ltd_trials;
-            if (pick(u, j & 3) <= thr) {
+            if (pick(u, jg & 3) <= thr) {
               ++ltd_events;
               uint32_t* p = wcol + i * wpr;
               if (f32) {                                        // eq.(5) in binary32 (R28); own word
@@ -331,8 +340,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
                 if ((*p >> sh) & fmask) atomicSub(p, 1u << sh);   // other fields of the word may move concurrently
               } else {                                          // eq.(5) rounded (eq.(8), R27)
                 const int q0 = (int)((*p >> sh) & fmask);
-                const uint4 u2 = philox((uint32_t)t, (uint32_t)i, (uint32_t)(j >> 2), TAG_ROUND_LTD, seed);
-                const int dq = s_dbd[q0] + (pick(u2, j & 3) < s_dtd[q0] ? 1 : 0);
+                const uint4 u2 = philox((uint32_t)t, (uint32_t)i, (uint32_t)(jg >> 2), TAG_ROUND_LTD, seed);
+                const int dq = s_dbd[q0] + (pick(u2, jg & 3) < s_dtd[q0] ? 1 : 0);
                 const int q1 = q0 - dq < 0 ? 0 : q0 - dq;
                 if (q1 != q0) atomicSub(p, (uint32_t)(q0 - q1) << sh);   // only this thread moves this field
               }
@@ -344,12 +353,53 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
 
       // global decision
       int W = -1, total = 0;
+      unsigned long long m = 0;                       // HARD: the cluster's best key; LAYER: its spiker count
       if (hard) {
-        unsigned long long m = 0;
         for (int r = 0; r < cs; ++r) { const unsigned long long x = s_slots[par * kMaxCluster + r]; m = x > m ? x : m; }
-        if (m) W = (int)(0xFFFFFFFFu - (uint32_t)m);
       } else {
-        for (int r = 0; r < cs; ++r) total += (int)s_slots[par * kMaxCluster + r];
+        for (int r = 0; r < cs; ++r) m += s_slots[par * kMaxCluster + r];
+      }
+      if (sharded) {
+        // the cluster's value goes to slot [cur & 1][shard] of every rank's mailbox as two LL words (peer stores, no
+        // fence); warp 0 of every CTA polls its own mailbox for the world's values and applies the same reduction
+        const uint32_t cur = seq0 + ++nxch;
+        const int mp = (int)(cur & 1u);
+        const unsigned long long tag = (unsigned long long)cur << 32;
+        if (rank == 0 && warp == 0 && lane < world) {
+          unsigned long long* sl = d.peers[lane]->slot[mp][d.shard];
+          st_relaxed_sys_u64(sl, tag | (uint32_t)(m >> 32));
+          st_relaxed_sys_u64(sl + 1, tag | (uint32_t)m);
+        }
+        if (warp == 0) {
+          unsigned long long x = 0ull;
+          if (lane < world) {
+            const unsigned long long* sl = d.mbox->slot[mp][lane];
+            const unsigned long long t_start = globaltimer();
+            unsigned long long w0, w1;
+            while (true) {
+              w0 = ld_relaxed_sys_u64(sl); w1 = ld_relaxed_sys_u64(sl + 1);
+              if ((uint32_t)(w0 >> 32) == cur && (uint32_t)(w1 >> 32) == cur) break;
+              if (globaltimer() - t_start > kShardTimeoutNs) __trap();   // a rank is gone: fail, never hang
+            }
+            x = ((unsigned long long)(uint32_t)w0 << 32) | (uint32_t)w1;
+          }
+          const uint32_t xh = (uint32_t)(x >> 32), xl = (uint32_t)x;
+          unsigned long long g;
+          if (hard) {
+            const uint32_t mh = __reduce_max_sync(FULL, xh);
+            g = ((unsigned long long)mh << 32) | __reduce_max_sync(FULL, xh == mh ? xl : 0u);
+          } else {
+            g = __reduce_add_sync(FULL, xl);
+          }
+          if (lane == 0) s_misc[8 + par * 2] = (int)(uint32_t)(g >> 32), s_misc[9 + par * 2] = (int)(uint32_t)g;
+        }
+        __syncthreads();
+        m = ((unsigned long long)(uint32_t)s_misc[8 + par * 2] << 32) | (uint32_t)s_misc[9 + par * 2];
+      }
+      if (hard) {
+        if (m) W = (int)(0xFFFFFFFFu - (uint32_t)m);     // global column
+      } else {
+        total = (int)m;
       }
 
       // apply eq.(2) reset, refractory, lateral inhibition (R6, R7)
@@ -358,14 +408,14 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
       if (hard) {
         if (W >= 0) {
           if (mycol) {
-            if (j == W) { v_r = fixed ? d.Vreset : __float_as_int(d.vresetf); cnt_r = d.t_ref; spiked = true; }
+            if (jg == W) { v_r = fixed ? d.Vreset : __float_as_int(d.vresetf); cnt_r = d.t_ref; spiked = true; }
             else {
               cnt_r = max(cnt_r, d.t_inh);
               if (inh_reset) v_r = fixed ? d.Vreset : __float_as_int(d.vresetf);
             }
           }
           img_spikes += 1;
-          local_spike = (W >= col0 && W < col0 + ncols);
+          local_spike = (W >= cbase + col0 && W < cbase + col0 + ncols);
         }
       } else if (total > 0) {
         if (mycol) {
@@ -391,8 +441,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
         const int nsp = hard ? 1 : s_misc[1];
         for (int grp = tid; grp < nq4; grp += nthr) {
           for (int m = 0; m < nsp; ++m) {
-            const int Wl = hard ? (W - col0) : (int)s_splist[m];
-            const int Wg = col0 + Wl;
+            const int Wl = hard ? (W - cbase - col0) : (int)s_splist[m];
+            const int Wg = cbase + col0 + Wl;
             const int ww = Wl >> lg, wsh = (Wl & ((1 << lg) - 1)) * bits;
             const uint4 u = philox((uint32_t)t, (uint32_t)Wg, (uint32_t)grp, stoch ? TAG_LTP : TAG_ROUND, seed);
 #pragma unroll
@@ -485,6 +535,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
       atomicAdd(&d.stats[7], (unsigned long long)d.n_images * (unsigned long long)T);
     }
   }
+  if (sharded && rank == 0 && tid == 0) d.mbox->seq = seq0 + nxch;   // every CTA read seq0 long ago
   if (cs > 1) { cluster_arrive(); cluster_wait(); }   // no CTA leaves while peers may address its SMEM
 }
 

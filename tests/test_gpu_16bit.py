@@ -92,8 +92,8 @@ def test_16bit_rejections(gpu):
     assert g.info()["engine"] == 1                       # per-step engine selected automatically
     with pytest.raises(P.SnnError):
         g.infer(synthdata.images(1), 10, synthdata.seeds(1))
-    with pytest.raises(P.SnnError):
-        P.Network(784, 640, 16, P.preset("16b"), shard=(0, 2))
+    sh = P.Network(784, 640, 16, P.preset("16b"), shard=(0, 2))   # shards run on the per-step engine
+    assert sh.info()["engine"] == 1 and sh.info()["world"] == 2
 
 
 def test_table2_grid_ensemble_mixed_widths(gpu):

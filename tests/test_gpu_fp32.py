@@ -131,8 +131,8 @@ def test_fp32_rejections(gpu):
     assert g.info()["engine"] == 1                       # per-step engine selected automatically
     with pytest.raises(P.SnnError):
         g.infer(synthdata.images(1), 10, synthdata.seeds(1))
-    with pytest.raises(P.SnnError):
-        P.Network(784, 640, 32, P.preset("16b"), shard=(0, 2))
+    sh = P.Network(784, 640, 32, P.preset("16b"), shard=(0, 2))   # shards run on the per-step engine
+    assert sh.info()["engine"] == 1 and sh.info()["world"] == 2
     with pytest.raises(P.SnnError):
         P.Network(784, 64, 32, P.params_from_dict(O.params("16b", membrane_mode=1)))
     with pytest.raises(P.SnnError):

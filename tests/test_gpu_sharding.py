@@ -144,8 +144,8 @@ def test_shard_api_errors(gpu):
     with pytest.raises(P.SnnError) as e:                  # 4 column groups cannot feed 5 shards
         P.Network(784, 100, 8, pp, shard=(0, 5))
     assert e.value.rc == -1
-    with pytest.raises(P.SnnError):                       # sharding needs the event engine
-        P.Network(784, 100, 8, P.params_from_dict(p, engine=1), shard=(0, 2))
+    with pytest.raises(P.SnnError):                       # bits > 8 shard on the per-step engine only
+        P.Network(784, 100, 16, P.params_from_dict(O.params("16b"), engine=2), shard=(0, 2))
     a, b = (P.Network(784, 100, 8, pp, shard=(r, 2)) for r in range(2))
     img = synthdata.images(1, "mnist")[0]
     with pytest.raises(P.SnnError):                       # not connected yet
