@@ -488,7 +488,7 @@ def test_invalid_params_rejected(bad):
     assert e.value.rc == -1
 
 
-@pytest.mark.parametrize("bits", [0, 1, 3, 12, 32])
+@pytest.mark.parametrize("bits", [0, 1, 3, 12, 24, 64])
 def test_invalid_bits_rejected(bits):
     with pytest.raises(O.OracleError):
         O.OracleNet(784, 10, bits, O.params("8b"))
