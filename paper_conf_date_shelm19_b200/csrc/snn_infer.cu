@@ -128,6 +128,7 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
   long long p_step = 0;       // next step to issue
   int p_img = 0, p_t = 0;     // its image (of this CTA) and timestep
   long long p_pos = 0;        // next ring position (consumers see its low 32 bits; R | 2^32)
+  unsigned long long p_act = 0;   // active input rows of the issued steps
   // Issue steps [p_step, min(G, limit)) while their rows fit the ring; ring positions before the first
   // row of step `first_live` are released (their readers passed a barrier).  Steps with more than rmax
   // rows are marked direct (read from global memory by the consumers, no ring slots).
@@ -206,6 +207,7 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
         if (lane == 0) { s_base[s] = (uint32_t)p_pos; s_nrows[s] = (uint32_t)n; }
         p_pos = pos;
       }
+      p_act += (unsigned long long)n;                 // active rows of the step (stats [0])
       ++p_step;
       if (++p_t == T) { p_t = 0; ++p_img; }
     }
@@ -224,7 +226,7 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
   lif.af = d.af; lif.bf = d.bf; lif.cf = d.cf; lif.dtf = d.dtf; lif.kI = d.kI; lif.ief = d.ief; lif.vthf = d.vthf;
   lif.A = d.A; lif.B = d.B; lif.C = d.C; lif.E = d.E; lif.Vth = d.Vth; lif.fixed = FIXED;
   const bool consumer = !is_producer && tcol < d.nthr_cols;
-  unsigned long long act_sum = 0, spikes = 0, lif_cs = 0;   // lif_cs: column-steps that ran eqs.(1)(2)
+  unsigned long long spikes = 0, lif_cs = 0;   // lif_cs: column-steps that ran eqs.(1)(2)
 
   if (is_producer) {
     // the producer runs decoupled from the consumers' step barriers: it publishes step records (release) and
@@ -242,6 +244,7 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
       while (r2 == rel && p_step == before && p_step < G) r2 = ld_acquire_cta(s_rel);   // ring full: wait
       rel = __shfl_sync(FULL, r2, 0);
     }
+    if (d.stats && lane == 0 && p_act) atomicAdd(&d.stats[0], p_act);
     return;
   }
 
@@ -269,9 +272,10 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
         if (j0 + 32 > d.n_exc) my_min_free = j0 >= d.n_exc ? 0xFFFF : 0;
       }
     }
-    while (ld_acquire_cta(s_pub) <= (uint32_t)g) {}     // the producer published step g
-    const uint32_t nr = s_nrows[g & (kSR - 1)];
+    // a thread whose 32 columns are all held (R6, R7) reads no rows: it goes straight to the step's barrier
     if (consumer && (int)tt >= my_min_free) {
+      while (ld_acquire_cta(s_pub) <= (uint32_t)g) {}     // the producer published step g
+      const uint32_t nr = s_nrows[g & (kSR - 1)];
       if (!(nr & kDirect)) {
         uint32_t acc[SW::NACC];
 #pragma unroll
@@ -350,7 +354,6 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
       }
       has_cand = ncand > 0;
     }
-    if (tid == 0) act_sum += nr & ~kDirect;
     // ---- B_g: the one barrier of a step (consumers only); then the ring slots of step g are released
     const int any = bar_red_or(1, ncons, has_cand);
     if (tid == 0) st_release_cta(s_rel, (uint32_t)(g + 1));
@@ -412,9 +415,6 @@ __global__ void __launch_bounds__(kInfMaxThreads, MINB) infer_kernel(const Infer
         my_max_free = mx;
       }
     }
-  }
-  if (d.stats && tid == 0) {
-    atomicAdd(&d.stats[0], act_sum);
   }
   if (d.stats && consumer && spikes) atomicAdd(&d.stats[1], spikes);
   if (d.stats && consumer && lif_cs) atomicAdd(&d.stats[2], lif_cs);
