@@ -74,6 +74,21 @@ def shards(world=2):
     assert np.array_equal(np.concatenate([s.weights() for s in sh], axis=1), o.weights())
 
 
+def step_shards(bits, world=2, n_exc=256, preset="16b", **kw):
+    """per-step engine column shards (per-step mailbox exchange), 16-bit codes or binary32 conductances"""
+    import paper_conf_date_shelm19_b200 as P
+    p = O.params(preset, init_seed=3, **kw)
+    sh = [P.Network(784, n_exc, bits, P.params_from_dict(p, engine=1), shard=(r, world)) for r in range(world)]
+    P.link_shards(sh)
+    o = O.OracleNet(784, n_exc, bits, p)
+    imgs = synthdata.images(2, "fashion", start=3)
+    seeds = synthdata.seeds(2, base_seed=4)
+    P.present_many(sh, [imgs] * world, 80, [seeds] * world)
+    for img, sd in zip(imgs, seeds):
+        o.present(img, 80, int(sd))
+    assert np.array_equal(np.concatenate([s.weights() for s in sh], axis=1), o.weights())
+
+
 CASES = {
     # lean kernel (HARD + RESET + stochastic): C1 shape (one CTA) and a 16-CTA C4-like slice
     "lean_c1": lambda: learn(100, 8, "8b", 0, 0, 3, 100),
@@ -89,6 +104,12 @@ CASES = {
     "step_c1": lambda: learn(100, 8, "8b", 1, 0, 2, 100),
     "step_c4s": lambda: learn(512, 2, "2b", 1, 16, 2, 120),
     "step_16b": lambda: learn(200, 16, "16b", 0, 0, 2, 80),
+    # LAYER WTA on the lean kernel; binary32 conductances (R28) on the per-step engine; per-step column shards
+    "lean_layer": lambda: learn(400, 8, "8b", 0, 0, 2, 200, wta_mode=1),
+    "step_fp32": lambda: learn(200, 32, "16b", 0, 0, 2, 80, mode=0),
+    "step_fp32_det": lambda: learn(200, 32, "16b", 0, 0, 2, 80, mode=0, stdp_mode=1, wta_mode=1),
+    "step_shards_16b": lambda: step_shards(16, rounding=2, membrane_mode=1),
+    "step_shards_fp32": lambda: step_shards(32, world=3),
     "infer": infer,
     "sparse": sparse,
     "shards": shards,
