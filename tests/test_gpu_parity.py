@@ -429,9 +429,10 @@ def test_lean_fuzz_vs_oracle(gpu, k):
     p, bits, n_exc, T, kind, start = _fuzz_case(k)
     try:
         g, o = _pair(784, n_exc, bits, p)
-    except P.SnnError as e:                       # a cluster size too small for the network's codes
-        assert e.rc == -5
-        pytest.skip("network does not fit the requested cluster")
+    except P.SnnError as e:                       # a cluster size too small for the network's codes is refused
+        assert e.rc == -5                         # (SNN_ESIZE); the library's own choice then runs the case
+        p = dict(p, cluster_size=0)
+        g, o = _pair(784, n_exc, bits, p)
     imgs, seeds = synthdata.images(3, kind, start=start), synthdata.seeds(3, base_seed=k + 1)
     counts = np.zeros(3, np.int32)
     g.present_batch(imgs, T, seeds, counts)
