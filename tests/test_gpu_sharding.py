@@ -159,11 +159,11 @@ def test_shard_api_errors(gpu):
 
 
 # ------------------------------------------------------------------ two processes, CUDA IPC mailboxes
-def _ipc_worker(rank, world, tmp, p, imgs, seeds, T):
+def _ipc_worker(rank, world, tmp, p, imgs, seeds, T, bits=8, engine=0):
     import torch
     import paper_conf_date_shelm19_b200 as P
     torch.cuda.set_device(0)
-    net = P.Network(784, 128, 8, P.params_from_dict(p), shard=(rank, world))
+    net = P.Network(784, 128, bits, P.params_from_dict(p, engine=engine), shard=(rank, world))
     with open(os.path.join(tmp, f"h{rank}.tmp"), "wb") as f:
         f.write(net.ipc_handle())
     os.rename(os.path.join(tmp, f"h{rank}.tmp"), os.path.join(tmp, f"h{rank}.bin"))
@@ -199,6 +199,35 @@ def test_sharded_two_processes_ipc(gpu, tmp_path):
             x.kill()
     assert all(x.exitcode == 0 for x in procs), [x.exitcode for x in procs]
     o = O.OracleNet(784, 128, 8, p)
+    oc = []
+    for img, sd in zip(imgs, seeds):
+        o.present(img, T, int(sd))
+        oc.append(int(O.unpack_bits(o.spikes(), 128).sum()))
+    w = np.concatenate([np.load(tmp_path / f"w{r}.npy") for r in range(2)], axis=1)
+    assert np.array_equal(w, o.weights())
+    for r in range(2):
+        assert np.load(tmp_path / f"c{r}.npy").tolist() == oc
+
+
+def test_step_sharded_two_processes_ipc(gpu, tmp_path):
+    """The per-step engine's shard exchange (one mailbox round per step) between two processes over CUDA IPC,
+    16-bit codes (R27): what a 784 -> 6400 16-bit network does across GPUs, here time-sliced on one GPU."""
+    import torch.multiprocessing as mp
+    p = O.params("16b", membrane_mode=1, rounding=2, init_seed=4, f_min_hz=5.0, f_max_hz=78.0)
+    imgs = synthdata.images(2, "mnist", start=6)
+    seeds = synthdata.seeds(2, base_seed=5)
+    T = 40
+    ctx = mp.get_context("spawn")
+    procs = [ctx.Process(target=_ipc_worker, args=(r, 2, str(tmp_path), p, imgs, seeds, T, 16, 1)) for r in range(2)]
+    for x in procs:
+        x.start()
+    for x in procs:
+        x.join(timeout=240)
+    for x in procs:
+        if x.is_alive():
+            x.kill()
+    assert all(x.exitcode == 0 for x in procs), [x.exitcode for x in procs]
+    o = O.OracleNet(784, 128, 16, p)
     oc = []
     for img, sd in zip(imgs, seeds):
         o.present(img, T, int(sd))

@@ -1,8 +1,9 @@
 """Column sharding of one network across ranks: CPU test doubles of the exchange
 protocols, run as world_size-2 `gloo` process groups, must reproduce the unsharded oracle bit for
-bit.  The first double exchanges once per STEP (SURVEY §8(e)'s all_gather reading, every mode); the
-second, test_per_epoch_summary_protocol_matches_oracle, is the protocol the CUDA path ships: one 16-byte
-summary per post-spike EPOCH.  Rank r owns a contiguous slice of post-synaptic columns (codes, v, countdown, last_post); the
+bit.  The first double exchanges once per STEP (SURVEY §8(e)'s all_gather reading, every mode): the protocol
+the per-step engine's shards ship (best key for HARD, summed count for LAYER); the second,
+test_per_epoch_summary_protocol_matches_oracle, is the event engines' protocol: one 16-byte summary per
+post-spike EPOCH.  Rank r owns a contiguous slice of post-synaptic columns (codes, v, countdown, last_post); the
 encoder and last_pre are replicated (every rank draws the same Philox inputs, R13); per step the
 ranks exchange one candidate key (HARD) or a candidate count (LAYER) with all_gather, then apply
 inhibition locally; LTD/LTP draws are keyed by GLOBAL indices, so the slicing cannot change them.
