@@ -56,8 +56,8 @@ constexpr int kDrawRows = 64;        // raw rows one LTD draw covers (two Philox
 constexpr int kDefSteps = 64;        // steps one deferred-LTD table covers at most (u64 step masks per input row)
 constexpr int kDefMargin = 16;       // a table with fewer steps left than this is rebuilt at the epoch start
 constexpr int kDefRowsPerThr = 1;    // raw rows a table draws per thread (an epoch spans ~15 steps of ~6 rows)
-constexpr int kSlots = 8;            // fixed row slots per step (steps with more active rows take the general path)
-constexpr int kBlk = 4;              // steps one block integrates before running the LIF chains through them
+constexpr int kSlots = 12;            // fixed row slots per step (steps with more active rows take the general path)
+constexpr int kBlk = 2;              // steps one block integrates before running the LIF chains through them
 
 struct LeanLayout {
   size_t slots, wsum, flags, misc, spk, dS, dbits, dev, w, pot, dep, lpre, offs, pst, prow, p8, run, rraw, log, total;
