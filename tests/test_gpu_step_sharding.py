@@ -68,3 +68,49 @@ def test_step_sharded_fp32_deterministic_layer(gpu):
     sh = _step_shards(784, 640, 32, p, 3)
     o = O.OracleNet(784, 640, 32, p)
     _compare(sh, o, synthdata.images(2, "mnist", start=30), 120, synthdata.seeds(2, base_seed=45), 784, 640, 0)
+
+
+def _wide_fuzz_case(k):
+    rng = np.random.default_rng(7000 + k)
+    bits = int(rng.choice([16, 32]))
+    world = int(rng.choice([1, 1, 2, 3]))
+    n_exc = int(rng.choice([33, 64, 100, 200, 320]))
+    n_exc = max(n_exc, 32 * world)
+    fmin, fmax = [(1.0, 22.0), (5.0, 78.0)][int(rng.integers(2))]
+    kw = dict(init_seed=int(rng.integers(1, 99)), wta_mode=int(rng.random() < 0.4), stdp_mode=int(rng.random() < 0.4),
+              inh_mode=int(rng.random() < 0.25), f_min_hz=fmin, f_max_hz=fmax,
+              t_ref_steps=int(rng.choice([1, 5, 10])), t_inh_steps=int(rng.choice([3, 10])),
+              v_spike=float(rng.choice([1.0, 2.0, 3.0])))
+    if bits == 16:
+        kw.update(membrane_mode=int(rng.integers(2)), rounding=int(rng.integers(3)), frac_bits=int(rng.choice([0, 15])))
+    p = O.params(str(rng.choice(["16b", "hf"])), **kw)
+    return p, bits, world, n_exc, int(rng.choice([60, 150])), str(rng.choice(["mnist", "fashion"])), int(rng.integers(5000))
+
+
+@pytest.mark.parametrize("k", range(16))
+def test_wide_step_fuzz_vs_oracle(gpu, k):
+    """Randomised 16-bit (R27) and binary32 (R28) networks on the per-step engine, unsharded and column-sharded
+    (world 1-3): widths, column counts, both STDP arms, HARD/LAYER, RESET/HOLD, rates, refractory / inhibition
+    lengths, current scale, membrane mode, rounding, Q1.15; 2 images against the oracle."""
+    import paper_conf_date_shelm19_b200 as P
+    p, bits, world, n_exc, T, kind, start = _wide_fuzz_case(k)
+    o = O.OracleNet(784, n_exc, bits, p)
+    imgs, seeds = synthdata.images(2, kind, start=start), synthdata.seeds(2, base_seed=k + 3)
+    mode = p["membrane_mode"]
+    if world == 1:
+        g = P.Network(784, n_exc, bits, P.params_from_dict(p))
+        for x, s in zip(imgs, seeds):
+            g.present(x, T, int(s))
+            o.present(x, T, int(s))
+            assert np.array_equal(g.spikes(), o.spikes()), "raster"
+            assert np.array_equal(g.weights(), o.weights()), "codes"
+            sg, so = O.unpack_state(g.state(), 784, n_exc), O.unpack_state(o.state(), 784, n_exc)
+            for key in ("cnt", "last_post", "last_pre"):
+                assert np.array_equal(sg[key], so[key]), key
+            if mode == 1:
+                assert np.array_equal(sg["v"], so["v"])
+            else:
+                np.testing.assert_allclose(sg["v"], so["v"], rtol=1e-5, atol=0)
+    else:
+        sh = _step_shards(784, n_exc, bits, p, world)
+        _compare(sh, o, imgs, T, seeds, 784, n_exc, mode)
