@@ -601,7 +601,7 @@ def main():
                                    f"replicas x{ws}" if ws > 1 else
                                    f"1 network in {K} shards on 1 GPU" if K > 1 else "1 network / 1 GPU"),
                    "cluster_size": info["cluster_size"], "threads_per_cta": info["threads"],
-                   "smem_bytes_per_cta": info["smem_bytes"],
+                   "smem_bytes_per_cta": info["smem_lean"] if info.get("lean") else info["smem_bytes"],
                    "l2": "flushed between timed steps (256 MiB write)", "membrane": "fp32" if args.membrane == 0 else "Q15.16"},
         "secondary": {"synaptic_events_per_s": ev_rate, "steps_per_s": images * T_STEPS / dev_s,
                       "post_spikes_per_image": int(stats[1]) / (B * args.steps),
