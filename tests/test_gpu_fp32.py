@@ -139,3 +139,55 @@ def test_fp32_rejections(gpu):
         P.Network(784, 64, 32, P.params_from_dict(O.params("16b", rounding=2)))
     with pytest.raises(P.SnnError):                      # 5 MB of binary32 > one cluster's shared memory
         P.Network(784, 1600, 32, P.preset("16b"))
+
+
+def test_fp32_stepwise_keep_state_and_reseed(gpu):
+    """North-star protocol at 32 bits: one step per call with SNN_KEEP_STATE (t0 = t); after every step the state
+    and the conductances equal the oracle's; at t = 40 the GPU is reseeded from the oracle (state + G) and goes on."""
+    import paper_conf_date_shelm19_b200 as P
+    p = O.params("16b", init_seed=8, f_min_hz=5.0, f_max_hz=78.0)
+    g, o = _pair(784, 64, p)
+    img = synthdata.images(1, "mnist", start=4)[0]
+    for t in range(80):
+        o.present_ex(img, 1, 21, flags=O.ORACLE_KEEP_STATE if t else 0, t0=t)
+        g.reset_stats()                                  # the library's counters accumulate across calls
+        g.present_ex(img, 1, 21, flags=(P.SNN_KEEP_STATE if t else 0), t0=t)
+        _compare_state(g, o, 784, 64)
+        if t == 40:
+            g.set_state(o.state())
+            g.set_weights(o.weights())
+    assert int(O.unpack_bits(o.spikes(), 64).sum()) >= 0
+
+
+def test_fp32_raster_input_forced_ltp_ltd(gpu):
+    """Encoder bypass (SNN_RASTER_INPUT) with forced post spikes: every LTP / LTD event of the binary32 arm (eq.(4)
+    / eq.(5) magnitudes) and its counters equal the oracle's."""
+    p = O.params("16b", i_ext=60.0, v_spike=1e-9, t_ref_steps=7, gamma_pot=0.9, gamma_dep=0.9)
+    g, o = _pair(784, 3, p)
+    rng = np.random.default_rng(3)
+    raster = rng.integers(0, 2 ** 32, size=(40, 25), dtype=np.uint64).astype(np.uint32)
+    raster &= rng.integers(0, 2 ** 32, size=(40, 25), dtype=np.uint64).astype(np.uint32)
+    raster[:, -1] &= 0xFFFF
+    g.present_raster(raster, 40, 99)
+    o.present_raster(raster, 40, 99)
+    _compare_state(g, o, 784, 3)
+    assert o.stats()[3] > 0 and o.stats()[5] > 0
+
+
+def test_fp32_and_16bit_ensemble_one_launch(gpu):
+    """snn_present_many with binary32 and 16-bit networks side by side on the per-step engine (one launch); each
+    network equals its own oracle."""
+    import paper_conf_date_shelm19_b200 as P
+    specs = [(32, O.params("16b", init_seed=11, cluster_size=2)), (16, O.params("16b", init_seed=12, rounding=2, cluster_size=2)),
+             (32, O.params("16b", init_seed=13, stdp_mode=1, cluster_size=2))]
+    nets = [P.Network(784, 128, b, P.params_from_dict(p)) for b, p in specs]
+    assert {n.info()["cluster_size"] for n in nets} == {2}
+    orc = [O.OracleNet(784, 128, b, p) for b, p in specs]
+    imgs = [synthdata.images(2, "mnist", start=50 + 7 * k) for k in range(3)]
+    seeds = [synthdata.seeds(2, base_seed=60 + k) for k in range(3)]
+    P.present_many(nets, imgs, 100, seeds)
+    for n, o, im, sd in zip(nets, orc, imgs, seeds):
+        for x, s in zip(im, sd):
+            o.present(x, 100, int(s))
+        assert np.array_equal(n.weights().view(np.uint8), o.weights().view(np.uint8))
+        assert np.array_equal(n.spikes(), o.spikes())
