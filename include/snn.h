@@ -31,12 +31,14 @@
  *    launch (the ensemble C5 runs 8 networks x B images per call), not one image per handle.
  *  - snn_create_sharded(..., nccl_unique_id) became snn_create_shard + snn_shard_ipc_handle /
  *    snn_shard_connect (multi-process) or snn_shard_link (one process): the exchange step is a
- *    16-byte per-epoch summary written by the kernel itself into every rank's device mailbox
- *    (NVLink peer stores), so there is no NCCL communicator to bootstrap.  The only
+ *    16-byte per-epoch summary (event engines) or a per-step WTA summary (per-step engine) written by the
+ *    kernel itself into every rank's device mailbox (NVLink peer stores), so there is no
+ *    NCCL communicator to bootstrap.  The only
  *    host-side collective is the caller's all_gather of the 64-byte IPC handles.  SNN_ENCCL is kept
  *    (reserved) so that the error-code values of §8(b) do not shift.
  *  - Added beyond §8(b): snn_present_batch / snn_present_ex (batches, raster input, KEEP_STATE),
- *    state/trace/info accessors, and the NEXT-1 / NEXT-4 entry points below.
+ *    state/trace/info accessors, bits = 16 (R27) and bits = 32 (binary32 conductance, R28), and the
+ *    NEXT-1 / NEXT-4 entry points below.
  */
 #ifndef SNN_H
 #define SNN_H
