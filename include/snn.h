@@ -119,13 +119,14 @@ typedef struct snn_handle snn_handle;
  * 16 bits (NEXT-2, "For 16-bit ... after floating point calculation of change in conductance dG,
  * the result is rounded"; R27): every STDP event (stochastic arm) moves the code by the
  * eq.(4)/(5) magnitude rounded by `rounding` instead of one LSB; 16-bit handles run on the per-step
- * engine (SNN_ENGINE_STEP is selected automatically) and cannot be sharded or used for snn_infer.
+ * engine (SNN_ENGINE_STEP is selected automatically); they shard on it (snn_create_shard) and infer on it
+ * (snn_infer, unsharded handles).
  * 32 bits (NEXT-2, "32-bit floating-point"; R28): every conductance is a binary32 G in
  * [g_min, g_max]; integration sums G in binary32 (I = v_spike * sum G); an STDP event (stochastic arm: gated
  * by the eqs.(6)(7) draw; deterministic arm: R16 window) sets G = binary32(G +- dG) with dG = eq.(4)/(5) in
  * binary64 by R28's exp recipe, clamped.  Requires membrane_mode = SNN_MEM_FP32 and rounding =
- * SNN_ROUND_NEAREST (else SNN_EINVAL); per-step engine, one cluster (784 -> <= 512 columns at 227 KB/CTA),
- * no sharding, no snn_infer.
+ * SNN_ROUND_NEAREST (else SNN_EINVAL); per-step engine; one cluster holds 784 -> <= 512 columns (227 KB per
+ * CTA), larger networks run column-sharded (snn_create_shard).
  * Conductances are initialised on the device (R4).  SNN_ESIZE if the network does not fit the
  * on-chip layout.  *out receives the handle. */
 int snn_create(int n_in, int n_exc, int bits, const snn_params* p, snn_handle** out);
@@ -259,9 +260,11 @@ int snn_shard_link(snn_handle* const* hs, int world);
  * not updated either (inference counters: snn_get_infer_stats).  All pointers host or device (the call
  * stages host buffers); SNN_ASYNC returns after enqueueing.  T <= 65535; n_exc <= 7168;
  * unsharded handles only.  Errors: SNN_EINVAL (arguments), SNN_ESIZE (n_exc too large), SNN_ECUDA.
+ * 16-bit codes and binary32 conductances (bits 16 / 32) run their inference on the per-step engine
+ * instead: the same semantics, the images one after another on the handle's cluster (synchronous).
  * snn_get_infer_stats: [0] sum over images and steps of active input rows, [1] post spikes, [2] column-
  * steps that ran the eqs.(1)(2) update (neither refractory nor inhibited: the LIF work that cannot be
- * skipped), since the handle was created.
+ * skipped; counted by the <= 8-bit path only), since the handle was created.
  *
  * snn_label (R22): labels[j] (n_exc int32) = the class c maximising the MEAN count of neuron j over
  * the labelling images of class c (counts: n_images x n_exc u32, classes: n_images int32 in

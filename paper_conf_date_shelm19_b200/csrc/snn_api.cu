@@ -129,6 +129,7 @@ struct snn_handle {
   int32_t* d_cls = nullptr;       size_t cls_cap = 0;
   int32_t* d_lab = nullptr;       size_t lab_cap = 0;
   unsigned long long* d_istats = nullptr;
+  unsigned long long* d_iscratch = nullptr;   // per-step engine inference: the kernel's learning-stats slots
   // NEXT-4 sparse workload
   int32_t* d_soff = nullptr;      size_t soff_cap = 0;
   uint16_t* d_stgt = nullptr;     size_t stgt_cap = 0;
@@ -234,7 +235,7 @@ void free_all(snn_handle* h) {
                   h->d_img, h->d_rin, h->d_seeds, h->d_counts, h->d_codes, h->d_bad,
                   h->d_words, h->d_ecnt, h->d_offs, h->d_rows, h->d_rows16, h->d_trace,
                   h->d_mbox, h->d_peers, h->d_winf, h->d_iwords, h->d_icounts, h->d_iecnt, h->d_cls,
-                  h->d_lab, h->d_istats, h->d_soff, h->d_stgt, h->d_sq, h->d_scounts, h->d_sraster,
+                  h->d_lab, h->d_istats, h->d_iscratch, h->d_soff, h->d_stgt, h->d_sq, h->d_scounts, h->d_sraster,
                   h->d_sstats};
   for (void* q : ptrs) if (q) cudaFree(q);
   for (cudaEvent_t e : h->prof_ev) cudaEventDestroy(e);
@@ -1242,6 +1243,64 @@ int infer_weights(snn_handle* h, int wpr) {
 
 extern "C" {
 
+}  // extern "C"
+
+namespace {
+// Inference at 16 bits (R27) and with binary32 conductances (R28): the per-step engine's presentation kernel with
+// FLAG_NO_LEARN (steps 1-4 of DESIGN.md §3.5 only, R21), images one after another on the handle's cluster, state
+// reset per image (R5), spikes per neuron and image written by the kernel; the handle's weights and state are not
+// touched.  Inference stats: [0] active input rows, [1] post spikes ([2], the LIF column-steps, is counted by the
+// batch-parallel kernel of the <= 8-bit codes only).
+int infer_step_engine(snn_handle* h, const uint8_t* images, int n_images, int T, const uint64_t* seeds,
+                      uint32_t* counts, int flags) {
+  if (n_images == 0) return SNN_OK;
+  if (!images || !seeds || !counts) return fail(SNN_EINVAL, "images / seeds / counts is NULL");
+  int rc;
+  DevGuard g(h->dev);
+  if (!h->d_istats) {
+    CUDA_TRY(dalloc(&h->d_istats, 3));
+    CUDA_TRY(cudaMemsetAsync(h->d_istats, 0, 3 * sizeof(unsigned long long), h->stream));
+  }
+  if (!h->d_iscratch) CUDA_TRY(dalloc(&h->d_iscratch, SNN_NSTATS));
+  CUDA_TRY(cudaMemsetAsync(h->d_iscratch, 0, SNN_NSTATS * sizeof(unsigned long long), h->stream));
+  const uint8_t* img = nullptr;
+  if ((rc = stage(h, images, (size_t)n_images * h->n_in, &h->d_img, &h->img_cap, &img))) return rc;
+  const unsigned long long* sd = nullptr;
+  if ((rc = stage(h, reinterpret_cast<const unsigned long long*>(seeds), (size_t)n_images, &h->d_seeds,
+                  &h->seeds_cap, &sd)))
+    return rc;
+  const bool counts_dev = is_device_ptr(counts);
+  uint32_t* cnt = counts;
+  if (!counts_dev) {
+    if ((rc = ensure(h, &h->d_icounts, &h->icounts_cap, (size_t)n_images * h->n_exc))) return rc;
+    cnt = h->d_icounts;
+  }
+  NetDesc d;
+  fill_static(h, d);
+  d.n_images = n_images; d.T = T; d.flags = snn::FLAG_NO_LEARN; d.t0 = 0;
+  d.images = img; d.seeds = sd; d.neuron_counts = cnt; d.stats = h->d_iscratch;
+  snn::LaunchParams lp;
+  lp.descs = nullptr;
+  lp.single = d;
+  CUDA_TRY(snn::launch_present(lp, 1, h->cs, h->nthr, h->smem, h->stream));
+  h->launches++;
+  unsigned long long sc[SNN_NSTATS], is[3];
+  CUDA_TRY(cudaMemcpyAsync(sc, h->d_iscratch, sizeof(sc), cudaMemcpyDeviceToHost, h->stream));
+  CUDA_TRY(cudaMemcpyAsync(is, h->d_istats, sizeof(is), cudaMemcpyDeviceToHost, h->stream));
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  is[0] += sc[0];
+  is[1] += sc[1];
+  CUDA_TRY(cudaMemcpyAsync(h->d_istats, is, sizeof(is), cudaMemcpyHostToDevice, h->stream));
+  if (!counts_dev)
+    CUDA_TRY(cudaMemcpyAsync(counts, cnt, (size_t)n_images * h->n_exc * sizeof(uint32_t), cudaMemcpyDeviceToHost,
+                             h->stream));
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  return finish(h, flags & ~SNN_ASYNC);
+}
+}  // namespace
+
+extern "C" {
+
 int snn_infer(snn_handle* h, const uint8_t* images, int n_images, int T, const uint64_t* seeds, uint32_t* counts,
               int flags) {
   int rc = check_handle(h);
@@ -1249,7 +1308,7 @@ int snn_infer(snn_handle* h, const uint8_t* images, int n_images, int T, const u
   if (n_images < 0 || T < 0) return fail(SNN_EINVAL, "negative n_images / T");
   if (T > 65535) return fail(SNN_EINVAL, "T=%d exceeds 65535 for inference", T);
   if (h->world > 1) return fail(SNN_EINVAL, "inference runs on unsharded handles");
-  if (h->bits > 8) return fail(SNN_EINVAL, "inference supports 2/4/8-bit codes (16/32-bit: NEXT-2 learning only)");
+  if (h->bits > 8) return infer_step_engine(h, images, n_images, T, seeds, counts, flags);
   if (h->n_exc > snn::kInferMaxCols) return fail(SNN_ESIZE, "n_exc=%d exceeds %d for inference", h->n_exc,
                                                  snn::kInferMaxCols);
   if (n_images == 0) return SNN_OK;

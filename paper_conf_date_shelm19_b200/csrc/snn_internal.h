@@ -13,7 +13,8 @@ constexpr int kNever = -1;
 constexpr int kPadRows = 16;        // fixed-width per-step row slots used by the event engine's block integration
 
 enum : uint32_t { TAG_ENC = 1, TAG_LTD = 2, TAG_LTP = 3, TAG_ROUND = 4, TAG_INIT = 5, TAG_ROUND_LTD = 6 };
-enum : int { FLAG_RASTER_INPUT = 1, FLAG_KEEP_STATE = 2, FLAG_RECORD_INPUT = 4, FLAG_ASYNC = 8, FLAG_FLOOR = 16 };
+enum : int { FLAG_RASTER_INPUT = 1, FLAG_KEEP_STATE = 2, FLAG_RECORD_INPUT = 4, FLAG_ASYNC = 8, FLAG_FLOOR = 16,
+             FLAG_NO_LEARN = 64 };   // internal: frozen weights (per-step engine inference, R21)
 
 // Everything one network needs inside the persistent kernel.  Built per launch on the host.
 struct Mailbox;
@@ -62,6 +63,7 @@ struct NetDesc {
   uint32_t* raster_out;                // [T][nwe] output raster of the last image (may be null)
   uint32_t* in_raster_out;             // [T][nwi] input raster of the last image (may be null)
   int* spike_counts;                   // [n_images] (may be null)
+  uint32_t* neuron_counts;             // [n_images][n_exc] spikes per neuron and image (FLAG_NO_LEARN; may be null)
   int n_images, T, flags, t0;
   // event engine: per-image active-row lists from the encoder pre-pass
   const uint32_t* ev_offs;             // [n_images][T+1] prefix offsets into ev_rows

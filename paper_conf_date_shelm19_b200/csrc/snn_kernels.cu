@@ -152,6 +152,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
   const bool stoch = d.stdp_mode == 0;
   const bool inh_reset = d.inh_mode == 0;
   const bool floor_mode = (flags & FLAG_FLOOR) != 0;   // bench: same launch shape, barriers + exchange only
+  const bool learn = (flags & FLAG_NO_LEARN) == 0;     // inference (R21): steps 1-4 only, weights and state kept
 
   // ---- one-time staging: tables + this CTA's weight slice -> SMEM
   for (int k = tid; k < 256; k += nthr) s_enc[k] = d.thr_enc[k];
@@ -193,6 +194,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
     const bool rec_in = last_img && rank == 0 && d.in_raster_out != nullptr;
     const bool rec_out = last_img && d.raster_out != nullptr;
     int img_spikes = 0;
+    uint32_t ncount = 0;                                      // this column's spikes in the image (inference)
     __syncthreads();
 
     for (int k = 0; k < T; ++k) {
@@ -322,7 +324,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
 
       // (a5) LTD, overlapped with the exchange: pre spikes at t against last_post (eq.(7), R10, R14).
       // Column-local and independent of this step's winner (uses the old last_post).
-      if (stoch && mycol && lpost_r >= 0) {
+      if (learn && stoch && mycol && lpost_r >= 0) {
         const int D = t - lpost_r;
         if (D < L_dep) {
           const uint32_t thr = s_dep[D];
@@ -433,10 +435,11 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
         const uint32_t bal = __ballot_sync(FULL, spiked);
         if (lane == 0 && warp < ngrp_cta) d.raster_out[(size_t)k * nwe + g0 + warp] = bal;
       }
+      if (spiked) ++ncount;
 
       // (a5) LTP (eq.(6)) or (a6) the deterministic arm (eqs.(4)(5)(8)) on the spiking columns.
       // Thread g owns input rows 4g..4g+3 (their words), so no atomics are needed here.
-      if (local_spike) {
+      if (local_spike && learn) {
         __syncthreads();                                                       // B5: LTD done, splist built
         const int nsp = hard ? 1 : s_misc[1];
         for (int grp = tid; grp < nq4; grp += nthr) {
@@ -501,7 +504,8 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
       post_sum += (unsigned long long)img_spikes;
       if (d.spike_counts) d.spike_counts[b] = img_spikes;
     }
-    if (last_img) {
+    if (d.neuron_counts && mycol) d.neuron_counts[(size_t)b * n_exc + j] = ncount;
+    if (last_img && learn) {
       if (mycol) { d.v[j] = v_r; d.cnt[j] = cnt_r; d.last_post[j] = lpost_r; }
       if (rank == 0) for (int i = tid; i < n_in; i += nthr) d.last_pre[i] = s_lpre[i];
     }
@@ -509,7 +513,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1) present_kernel(const __grid_co
   }  // images
 
   // write the (learned) slice back to HBM
-  {
+  if (learn) {
     uint4* dst = reinterpret_cast<uint4*>(d.wslices + (size_t)rank * slice_words);
     const uint4* src = reinterpret_cast<const uint4*>(s_w);
     for (int k = tid; k < slice_words / 4; k += nthr) dst[k] = src[k];

@@ -90,10 +90,11 @@ def test_16bit_rejections(gpu):
     import paper_conf_date_shelm19_b200 as P
     g = P.Network(784, 64, 16, P.preset("16b"))
     assert g.info()["engine"] == 1                       # per-step engine selected automatically
-    with pytest.raises(P.SnnError):
-        g.infer(synthdata.images(1), 10, synthdata.seeds(1))
+    assert g.infer(synthdata.images(1), 10, synthdata.seeds(1)).shape == (1, 64)   # per-step engine inference
     sh = P.Network(784, 640, 16, P.preset("16b"), shard=(0, 2))   # shards run on the per-step engine
     assert sh.info()["engine"] == 1 and sh.info()["world"] == 2
+    with pytest.raises(P.SnnError):                      # inference runs on unsharded handles
+        sh.infer(synthdata.images(1), 10, synthdata.seeds(1))
 
 
 def test_table2_grid_ensemble_mixed_widths(gpu):

@@ -129,10 +129,11 @@ def test_fp32_rejections(gpu):
     import paper_conf_date_shelm19_b200 as P
     g = P.Network(784, 64, 32, P.preset("16b"))
     assert g.info()["engine"] == 1                       # per-step engine selected automatically
-    with pytest.raises(P.SnnError):
-        g.infer(synthdata.images(1), 10, synthdata.seeds(1))
+    assert g.infer(synthdata.images(1), 10, synthdata.seeds(1)).shape == (1, 64)   # per-step engine inference
     sh = P.Network(784, 640, 32, P.preset("16b"), shard=(0, 2))   # shards run on the per-step engine
     assert sh.info()["engine"] == 1 and sh.info()["world"] == 2
+    with pytest.raises(P.SnnError):                      # inference runs on unsharded handles
+        sh.infer(synthdata.images(1), 10, synthdata.seeds(1))
     with pytest.raises(P.SnnError):
         P.Network(784, 64, 32, P.params_from_dict(O.params("16b", membrane_mode=1)))
     with pytest.raises(P.SnnError):
@@ -191,3 +192,30 @@ def test_fp32_and_16bit_ensemble_one_launch(gpu):
             o.present(x, 100, int(s))
         assert np.array_equal(n.weights().view(np.uint8), o.weights().view(np.uint8))
         assert np.array_equal(n.spikes(), o.spikes())
+
+
+@pytest.mark.parametrize("bits,wta", [(32, 0), (32, 1), (16, 0)])
+def test_wide_inference_matches_oracle(gpu, bits, wta):
+    """NEXT-1 at 16 bits / binary32 (R21 on R27 / R28): snn_infer on the per-step engine with frozen weights equals
+    the oracle's inference spike counts for every neuron and image; weights and state are left untouched; labelling
+    and the vote (R22, R23) then run on those counts."""
+    import paper_conf_date_shelm19_b200 as P
+    p = O.params("16b", wta_mode=wta, init_seed=14, f_min_hz=5.0, f_max_hz=78.0,
+                 **({"rounding": 2, "membrane_mode": 1} if bits == 16 else {}))
+    g = P.Network(784, 100, bits, P.params_from_dict(p))
+    o = O.OracleNet(784, 100, bits, p)
+    learn_imgs, learn_seeds = synthdata.images(2, "mnist", start=300), synthdata.seeds(2, base_seed=70)
+    for x, s in zip(learn_imgs, learn_seeds):           # some learning first, identical on both sides
+        g.present(x, 100, int(s))
+        o.present(x, 100, int(s))
+    w0, st0 = g.weights().copy(), g.state().copy()
+    imgs, seeds = synthdata.images(6, "mnist", start=310), synthdata.seeds(6, base_seed=71)
+    c = g.infer(imgs, 120, seeds)
+    want = o.infer(imgs, 120, seeds)
+    assert np.array_equal(c, want)
+    assert int(want.sum()) > 0
+    assert np.array_equal(g.weights().view(np.uint8), w0.view(np.uint8)) and np.array_equal(g.state(), st0)
+    classes = synthdata.labels(6)
+    lab = g.label(c, classes, 10)
+    assert np.array_equal(lab, O.label(want, classes, 10))
+    assert np.array_equal(g.classify(c, lab, 10), O.classify(want, lab, 10))
