@@ -275,6 +275,13 @@ int snn_shard_link(snn_handle* const* hs, int world);
 int snn_infer(snn_handle* h, const uint8_t* images, int n_images, int T, const uint64_t* seeds, uint32_t* counts,
               int flags);
 int snn_get_infer_stats(snn_handle* h, uint64_t stats[3]);
+/* snn_infer_many: snn_infer for n per-step-engine handles in ONE launch (bits 16 / 32, or SNN_ENGINE_STEP):
+ * independent networks and, what snn_infer cannot do, the linked shards of one column-sharded network (every
+ * shard of its world must be in the call; each shard counts its own columns).  images[k] / seeds[k] /
+ * counts[k] (n_images x n_exc_k u32) per handle, host or device.  Synchronous; weights and state untouched.
+ * SNN_EINVAL for event-engine handles or an incomplete world. */
+int snn_infer_many(snn_handle* const* hs, int n, const uint8_t* const* images, int n_images, int T,
+                   const uint64_t* const* seeds, uint32_t* const* counts);
 int snn_label(snn_handle* h, const uint32_t* counts, int n_images, const int32_t* classes, int n_classes,
               int32_t* labels);
 int snn_classify(snn_handle* h, const uint32_t* counts, int n_images, const int32_t* labels, int n_classes,

@@ -863,9 +863,15 @@ int snn_present_batch(snn_handle* h, const uint8_t* images, int n_images, int T,
   return present_impl(h, images, n_images, T, seeds, spike_counts, flags, 0);
 }
 
-int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images, int n_images, int T,
-                     const uint64_t* const* seeds) {
+}  // extern "C"
+
+namespace {
+// One launch for n handles (ensembles, linked shards).  kflags = FLAG_NO_LEARN (per-step engine only): inference,
+// spike counts per neuron and image into ncounts[k] (device buffers), the handles' weights and state untouched.
+int present_many_impl(snn_handle* const* hs, int n, const uint8_t* const* images, int n_images, int T,
+                      const uint64_t* const* seeds, int kflags, uint32_t* const* ncounts) {
   if (!hs || n < 1 || !images || !seeds) return fail(SNN_EINVAL, "bad ensemble arguments");
+  const bool infer = (kflags & snn::FLAG_NO_LEARN) != 0;
   if (n_images < 0 || T < 0) return fail(SNN_EINVAL, "negative n_images / T");
   for (int k = 0; k < n; ++k) {
     if (!hs[k]) return fail(SNN_EINVAL, "handle %d is NULL", k);
@@ -877,7 +883,9 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
       return fail(SNN_EINVAL, "ensemble handles must share n_in, cluster size, CTA shape, engine, membrane mode, device");
     for (int m = 0; m < k; ++m)
       if (hs[m] == hs[k]) return fail(SNN_EINVAL, "handle %d appears twice", k);
-    hs[k]->w_version++;
+    if (infer && hs[k]->engine != SNN_ENGINE_STEP)
+      return fail(SNN_EINVAL, "snn_infer_many runs per-step-engine handles (bits 16 / 32 or SNN_ENGINE_STEP)");
+    if (!infer) hs[k]->w_version++;
     if (hs[k]->world > 1) {        // every shard of its world must be in this launch (they wait on each other)
       if (hs[k]->linked.empty()) return fail(SNN_EINVAL, "shard handle %d is not linked in this process", k);
       for (snn_handle* o : hs[k]->linked)
@@ -903,7 +911,17 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
     h->stream = h0->stream;            // all pre-pass work is ordered on the launching stream
     NetDesc& d = descs[k];
     fill_static(h, d);
-    d.n_images = n_images; d.T = T; d.flags = 0; d.t0 = 0;
+    d.n_images = n_images; d.T = T; d.flags = kflags; d.t0 = 0;
+    if (infer) {                       // inference: the learning counters are left alone (scratch slots)
+      if (!h->d_iscratch && dalloc(&h->d_iscratch, SNN_NSTATS) != cudaSuccess) {
+        cudaGetLastError();
+        h->stream = own;
+        return fail(SNN_ENOMEM, "scratch allocation failed");
+      }
+      cudaMemsetAsync(h->d_iscratch, 0, SNN_NSTATS * sizeof(unsigned long long), h0->stream);
+      d.stats = h->d_iscratch;
+      d.neuron_counts = ncounts[k];
+    }
     const uint8_t* img = nullptr;
     const unsigned long long* sd = nullptr;
     int rc = stage(h, images[k], (size_t)n_images * h->n_in, &h->d_img, &h->img_cap, &img);
@@ -911,7 +929,7 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
                         &h->seeds_cap, &sd);
     if (!rc) rc = ensure(h, &h->d_raster, &h->raster_cap, (size_t)T * d.nwe);
     if (!rc) {
-      d.images = img; d.seeds = sd; d.raster_out = h->d_raster;
+      d.images = img; d.seeds = sd; d.raster_out = infer ? nullptr : h->d_raster;
       if (ev) rc = event_prepass(h, d, img, nullptr, n_images, T, 0, sd);
       if (!rc) rc = shard_arm(h, d);
     }
@@ -986,10 +1004,53 @@ int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images,
   cudaFree(d_descs);
   if (e != cudaSuccess) return fail(SNN_ECUDA, "present_many: %s", cudaGetErrorString(e));
   for (int k = 0; k < n; ++k) {
+    hs[k]->launches++;
+    if (infer) continue;
     hs[k]->last_T = T;
     hs[k]->last_recorded = false;
     hs[k]->t_next = T;
-    hs[k]->launches++;
+  }
+  return SNN_OK;
+}
+}  // namespace
+
+extern "C" {
+
+int snn_present_many(snn_handle* const* hs, int n, const uint8_t* const* images, int n_images, int T,
+                     const uint64_t* const* seeds) {
+  return present_many_impl(hs, n, images, n_images, T, seeds, 0, nullptr);
+}
+
+int snn_infer_many(snn_handle* const* hs, int n, const uint8_t* const* images, int n_images, int T,
+                   const uint64_t* const* seeds, uint32_t* const* counts) {
+  if (!hs || n < 1 || !counts) return fail(SNN_EINVAL, "bad arguments");
+  if (n_images < 0 || T < 0 || T > 65535) return fail(SNN_EINVAL, "n_images / T out of range");
+  if (n_images == 0) return SNN_OK;
+  std::vector<uint32_t*> dev(n, nullptr);
+  for (int k = 0; k < n; ++k) {
+    if (!hs[k] || !counts[k]) return fail(SNN_EINVAL, "handle / counts %d is NULL", k);
+    if (is_device_ptr(counts[k])) { dev[k] = counts[k]; continue; }
+    int rc = ensure(hs[k], &hs[k]->d_icounts, &hs[k]->icounts_cap, (size_t)n_images * hs[k]->n_exc);
+    if (rc) return rc;
+    dev[k] = hs[k]->d_icounts;
+  }
+  int rc = present_many_impl(hs, n, images, n_images, T, seeds, snn::FLAG_NO_LEARN, dev.data());
+  if (rc) return rc;
+  DevGuard g(hs[0]->dev);
+  for (int k = 0; k < n; ++k) {      // inference counters (snn_get_infer_stats [0], [1]) and the host copies
+    snn_handle* h = hs[k];
+    if (!h->d_istats) {
+      CUDA_TRY(dalloc(&h->d_istats, 3));
+      CUDA_TRY(cudaMemset(h->d_istats, 0, 3 * sizeof(unsigned long long)));
+    }
+    unsigned long long sc[SNN_NSTATS], is[3];
+    CUDA_TRY(cudaMemcpy(sc, h->d_iscratch, sizeof(sc), cudaMemcpyDeviceToHost));
+    CUDA_TRY(cudaMemcpy(is, h->d_istats, sizeof(is), cudaMemcpyDeviceToHost));
+    is[0] += sc[0];
+    is[1] += sc[1];
+    CUDA_TRY(cudaMemcpy(h->d_istats, is, sizeof(is), cudaMemcpyHostToDevice));
+    if (dev[k] != counts[k])
+      CUDA_TRY(cudaMemcpy(counts[k], dev[k], (size_t)n_images * h->n_exc * sizeof(uint32_t), cudaMemcpyDeviceToHost));
   }
   return SNN_OK;
 }

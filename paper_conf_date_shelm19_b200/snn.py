@@ -19,7 +19,7 @@ PRESETS = {"2b": 0, "4b": 1, "8b": 2, "16b": 3, "hf": 4}
 # Every function declared in include/snn.h (checked by tests/test_abi.py).
 EXPORTS = [
     "snn_params_preset", "snn_create", "snn_destroy", "snn_set_stream", "snn_synchronize",
-    "snn_present", "snn_present_batch", "snn_present_ex", "snn_present_raster", "snn_present_many",
+    "snn_present", "snn_present_batch", "snn_present_ex", "snn_present_raster", "snn_present_many", "snn_infer_many",
     "snn_get_weights", "snn_set_weights", "snn_get_spikes", "snn_get_input_raster",
     "snn_state_bytes", "snn_get_state", "snn_set_state", "snn_get_stats", "snn_reset_stats",
     "snn_get_info", "snn_set_trace", "snn_get_trace", "snn_set_profile", "snn_get_profile", "snn_last_error",
@@ -79,6 +79,7 @@ def lib():
             "snn_present_ex": ([vp, vp, i32, u64, i32, i32], i32),
             "snn_present_raster": ([vp, vp, i32, u64], i32),
             "snn_present_many": ([vp, i32, vp, i32, i32, vp], i32),
+            "snn_infer_many": ([vp, i32, vp, i32, i32, vp, vp], i32),
             "snn_get_weights": ([vp, vp, sz], i32),
             "snn_set_weights": ([vp, vp, sz], i32),
             "snn_get_spikes": ([vp, vp, sz], i32),
@@ -361,6 +362,20 @@ def link_shards(shards: Sequence[Network]):
     """Single process: link shards 0..world-1 of one network (include/snn.h snn_shard_link)."""
     hs = (ctypes.c_void_p * len(shards))(*[x.handle.value for x in shards])
     _check(lib().snn_shard_link(hs, len(shards)), "snn_shard_link")
+
+
+def infer_many(nets: Sequence[Network], images: Sequence, T: int, seeds: Sequence):
+    """Inference with frozen weights for several per-step-engine networks (or the shards of one) in one launch;
+    returns one (n_images, n_exc) u32 count array per network (include/snn.h snn_infer_many)."""
+    n = len(nets)
+    n_images = int(images[0].shape[0])
+    outs = [np.zeros((n_images, x.n_exc), dtype=np.uint32) for x in nets]
+    hs = (ctypes.c_void_p * n)(*[x.handle.value for x in nets])
+    imgs = (ctypes.c_void_p * n)(*[_ptr(a).value for a in images])
+    sds = (ctypes.c_void_p * n)(*[_ptr(s).value for s in seeds])
+    cts = (ctypes.c_void_p * n)(*[_ptr(c).value for c in outs])
+    _check(lib().snn_infer_many(hs, n, imgs, n_images, T, sds, cts), "snn_infer_many")
+    return outs
 
 
 def present_many(nets: Sequence[Network], images: Sequence, T: int, seeds: Sequence):

@@ -114,3 +114,22 @@ def test_wide_step_fuzz_vs_oracle(gpu, k):
     else:
         sh = _step_shards(784, n_exc, bits, p, world)
         _compare(sh, o, imgs, T, seeds, 784, n_exc, mode)
+
+
+@pytest.mark.parametrize("bits,world", [(16, 4), (32, 7)])
+def test_sharded_wide_C4_inference(gpu, bits, world):
+    """NEXT-1 on the C4 network at 16 bits / binary32 (column-sharded over 4 / 7 clusters): snn_infer_many runs
+    the shards in one launch with frozen weights; the concatenated per-neuron counts equal the oracle's inference."""
+    import paper_conf_date_shelm19_b200 as P
+    p = O.params("16b", init_seed=15, f_min_hz=5.0, f_max_hz=78.0, **({"rounding": 2} if bits == 16 else {}))
+    sh = _step_shards(784, 6400, bits, p, world)
+    o = O.OracleNet(784, 6400, bits, p)
+    imgs, seeds = synthdata.images(2, "fashion", start=77), synthdata.seeds(2, base_seed=78)
+    w0 = [s.weights().copy() for s in sh]
+    outs = P.infer_many(sh, [imgs] * world, 60, [seeds] * world)
+    want = o.infer(imgs, 60, seeds)
+    assert np.array_equal(np.concatenate(outs, axis=1), want)
+    assert int(want.sum()) > 0
+    assert all(np.array_equal(s.weights().view(np.uint8), w.view(np.uint8)) for s, w in zip(sh, w0))
+    with pytest.raises(P.SnnError):                  # the world must be complete
+        P.infer_many(sh[:1], [imgs], 60, [seeds])
